@@ -1,0 +1,195 @@
+/* mggcn.h — C ABI of the B200-native MG-GCN hot path.
+ *
+ * MG-GCN: Balın, Sancak, Çatalyürek, "MG-GCN: A Scalable multi-GPU GCN
+ * Training Framework", ICPP '22.  The paper text is /root/reference/PAPER.md
+ * at build time and is cited here as P:line.  The library computes full-batch
+ * GCN training on a randomly permuted, 1D row-partitioned
+ * graph:
+ *     forward   H' = ReLU(Â^T · H · W)                 (Eq. 1, 5-7)
+ *     loss      softmax cross-entropy
+ *     backward  Eq. 8-11
+ *     update    W_G summed over ranks, Adam
+ * where Â_uv = A_uv / sum_w A_wv is the in-degree normalised adjacency (Eq. 2,
+ * P:312-318).  Every sparse aggregation runs as P stages (Fig. 2-3):
+ * the next feature block is broadcast into BC1/BC2 on the communication stream
+ * while the current stage's CSR block SpMM runs on the compute stream
+ * (§4.3).
+ *
+ * Conventions (all functions):
+ *  - return an int status; 0 = MGGCN_OK.  Nothing throws across the ABI.
+ *    mggcn_last_error() returns a thread-local message for the last non-OK
+ *    return of the calling thread.
+ *  - host inputs are copied before the call returns; the caller may free them.
+ *  - device memory is never allocated by the library outside the caller-owned
+ *    workspace given to mggcn_model_create (the debug_* test entry points are
+ *    the exception and say so).
+ *  - all matrices are row-major fp32; W_l is d_l x d_{l+1} (so H·W is Eq. 5).
+ *  - CUDA / NCCL errors poison a model: every later call on it returns the
+ *    same code.
+ *  - a model is single-threaded.  Results are bitwise reproducible run to run
+ *    for fixed inputs, P and seed (no floating-point atomics); they are NOT
+ *    bitwise equal across different P.
+ */
+#ifndef MGGCN_H
+#define MGGCN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+    MGGCN_OK = 0,
+    MGGCN_EINVAL = -1,        /* invalid argument (see each function)              */
+    MGGCN_ENOMEM = -2,        /* host allocation failed / workspace too small      */
+    MGGCN_ECUDA = -3,         /* CUDA runtime error (model poisoned)               */
+    MGGCN_ENCCL = -4,         /* NCCL error (model poisoned)                       */
+    MGGCN_ESTATE = -5,        /* call out of order (backward before forward, ...)  */
+    MGGCN_EUNSUPPORTED = -6   /* valid but not implemented         */
+};
+
+/* Model flags. */
+enum {
+    MGGCN_F_OVERLAP = 1u,     /* overlap broadcast i+1 with SpMM i.  Off =
+                                 each broadcast waits for the previous stage.          */
+    MGGCN_F_RELU_LAST = 2u,   /* ReLU on the last layer too (literal Eq. 4, reading C4) */
+    MGGCN_F_TF32X1 = 4u,      /* 1xTF32 GEMMs (faster, ~1e-3 rel. error); default is
+                                 3xTF32 (hi/lo split, ~fp32 accuracy)                  */
+    MGGCN_F_NO_BCAST = 16u,   /* TIMING ONLY: skip broadcasts; results invalid         */
+    MGGCN_F_PROFILE = 32u     /* record per-op CUDA events (see mggcn_get_profile)     */
+};
+
+typedef struct mggcn_graph_s* mggcn_graph; /* host CSR of A + in-degrees                     */
+typedef struct mggcn_part_s* mggcn_part;   /* one rank's permuted 1D partition (host)        */
+typedef struct mggcn_model_s* mggcn_model; /* weights, Adam state, buffer plan, comm, streams */
+
+const char* mggcn_last_error(void);
+int mggcn_version(void); /* MAJOR*10000 + MINOR*100 + PATCH */
+
+/* ------------------------------------------------------------------ ingest
+ * mggcn_load_csr — the adjacency A in R^{n x n} as CSR.
+ *   rowptr  int64[n+1], host; rowptr[0] = 0, non-decreasing, rowptr[n] = nnz
+ *   colidx  int32[nnz], host; in [0, n); any order within a row
+ *   vals    fp32[nnz] host, finite and > 0; NULL means A_uv = 1 (pattern-only)
+ *   Duplicate entries are multiplicities (reading C19).  Computes the
+ *   weighted in-degree deg(v) = sum_u A_uv (fp64 in CSR order, rounded to
+ *   fp32; Eq. 2, reading C18) and detects multiset symmetry.
+ *   EINVAL: n <= 0, n >= 2^31, malformed rowptr, colidx out of range, bad vals. */
+int mggcn_load_csr(int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* colidx, const float* vals,
+                   mggcn_graph* out);
+/* n, nnz, symmetric (0/1), unit weights (0/1); deg: fp32[n] host or NULL. */
+int mggcn_graph_info(mggcn_graph g, int64_t* n, int64_t* nnz, int32_t* symmetric, int32_t* unit_weights,
+                     float* deg);
+
+/* --------------------------------------------------------------- partition
+ * mggcn_partition — random vertex permutation pi (splitmix64
+ * Fisher-Yates from perm_seed, reading C15; 0 = identity), uniform partition
+ * vector p(i) = floor(i n / P) (Eq. 13, reading C14), and for `rank` the P
+ * forward tiles F_rank,j (rows p(rank)..p(rank+1)-1 of Â'^T restricted to
+ * columns p(j)..p(j+1)-1, local indices, Eq. 14-15) and backward tiles
+ * B_rank,j (the same rows of Â').  Pure host work.
+ *   nparts in [1, 64], rank in [0, nparts), n >= nparts.
+ *   EUNSUPPORTED: a tile with >= 2^31 entries. */
+int mggcn_partition(mggcn_graph g, int32_t nparts, int32_t rank, uint64_t perm_seed, mggcn_part* out);
+/* p: int64[P+1] or NULL; perm: int64[n] (perm[old] = new) or NULL;
+ * tile_nnz: int64[2P] (F_rank,0..P-1 then B_rank,0..P-1) or NULL. */
+int mggcn_part_info(mggcn_part part, int32_t* nparts, int32_t* rank, int64_t* n, int64_t* p, int64_t* perm,
+                    int64_t* tile_nnz);
+/* Host copy of tile (dir 0 = forward F_rank,j of Â'^T, 1 = backward B_rank,j
+ * of Â'): rowptr int32[n_rank+1], colidx int32[nnz], vals fp32[nnz] (the
+ * value Â'_uv of every entry; may be NULL).  Bit-exact test contract. */
+int mggcn_part_export_tile(mggcn_part part, int32_t dir, int32_t j, int32_t* rowptr, int32_t* colidx, float* vals);
+/* inv_deg of this rank's rows (fp32 1/deg, 0 when deg = 0, reading C20). */
+int mggcn_part_inv_deg(mggcn_part part, float* inv_deg);
+
+/* ------------------------------------------------------------------- model
+ * dims: int32[L+1] = d_0 .. d_L (d_0 = input features, d_L = classes).
+ * parts: nlocal partitions.  nlocal = 1 is the production mode (one process
+ * per GPU; for P > 1, nccl_id128 is the ncclUniqueId from
+ * mggcn_nccl_unique_id on rank 0, shared by the caller, e.g. through
+ * torch.distributed).  nlocal = P (parts for ranks 0..P-1 in order,
+ * nccl_id128 = NULL) is the LOOPBACK mode: all P ranks live on the current
+ * device and broadcasts become device copies with the identical event
+ * schedule (test harness for the P-stage pipeline on one GPU).
+ * workspace: device memory, caller-owned, >= mggcn_workspace_bytes, 256-B
+ * aligned; it must outlive the model.  compute_stream / comm_stream:
+ * cudaStream_t values (streams 0 and 1 of P:929-933); 0 = legacy default.
+ * EUNSUPPORTED: an SpMM-first layer (d_l < d_{l+1}) at l > 0. */
+int mggcn_workspace_bytes(const mggcn_part* parts, int32_t nlocal, int32_t L, const int32_t* dims, uint32_t flags,
+                          size_t* bytes);
+int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32_t L, const int32_t* dims, uint32_t flags,
+                       const void* nccl_id128, void* workspace, size_t ws_bytes, uintptr_t compute_stream,
+                       uintptr_t comm_stream, mggcn_model* out);
+int mggcn_nccl_unique_id(void* out128);
+
+/* Weights W_l (d_l x d_{l+1}, host fp32).  set_weights resets Adam (t = 0). */
+int mggcn_set_weights(mggcn_model m, int32_t layer, const float* W);
+int mggcn_get_weights(mggcn_model m, int32_t layer, float* W);
+
+/* ----------------------------------------------------------- the hot path
+ * mggcn_forward — L layers (Eq. 5-7 with the §4.4 order rule), then the
+ * softmax-CE loss and its gradient (written in place, Eq. 19).
+ *   X_local  fp32 rows of X' owned by this model (rows p(rank)..p(rank+1)-1
+ *            of the PERMUTED features; all n rows in loopback mode), row
+ *            stride ldx >= d_0.  Host or device pointer (host: copied on the
+ *            compute stream; this is the end-to-end path).
+ *   y_local  int32 labels of the same rows (host or device); -1 = unlabelled.
+ *   loss     host out: global mean CE over labelled vertices (reading C5), or
+ *            NULL (no host synchronisation).
+ *   logits_local  device out (n_local x d_L, ld = d_L) or NULL.
+ * mggcn_backward — Eq. 8-11 for l = L-1..0, per-layer W_G all-reduce
+ *   (P:696-704).  ESTATE without a prior forward.
+ * mggcn_step — waits for the W_G all-reduce, Adam (reading C6), t++.
+ *   ESTATE without a prior backward. */
+int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float* loss,
+                  float* logits_local);
+int mggcn_backward(mggcn_model m);
+int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps);
+
+/* Synchronising getters / checkpoint. */
+int mggcn_get_loss(mggcn_model m, float* loss);                 /* loss of the last forward */
+int mggcn_get_grad(mggcn_model m, int32_t layer, float* WG);    /* reduced W_G of the last backward */
+int mggcn_get_adam(mggcn_model m, int32_t layer, float* mom, float* vel, int64_t* t);
+int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, const float* vel, int64_t t);
+
+/* Profiling (MGGCN_F_PROFILE): accumulated device milliseconds and launch
+ * counts per op class since the last reset, measured with CUDA events on the
+ * stream each op is launched on.  Classes: 0 spmm, 1 gemm, 2 loss, 3 adam,
+ * 4 bcast, 5 allreduce, 6 other.  Synchronises. */
+int mggcn_get_profile(mggcn_model m, double* ms /*[7]*/, int64_t* launches /*[7]*/, int32_t reset);
+/* Algorithmic work of one epoch of this model's rows for the roofline
+ * (DESIGN.md §6): spmm_bytes = compulsory SpMM bytes
+ * (indices + rowptr + each input row once + each output row once, summed over
+ * the epoch's SpMM launches), spmm_gather_bytes = cacheless gather model
+ * (nnz * width * 4 B), gemm_flops, bcast_bytes = bytes received by
+ * broadcasts.  Any pointer may be NULL. */
+int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* spmm_gather_bytes, double* gemm_flops,
+                     double* bcast_bytes);
+
+/* Number of kernels this library has launched in this process (all models,
+ * all debug hooks).  Read before and after a timed region to count them. */
+int64_t mggcn_kernel_launch_count(void);
+
+void mggcn_graph_free(mggcn_graph g);
+void mggcn_part_free(mggcn_part part);
+void mggcn_model_free(mggcn_model m);
+
+/* ------------------------------------------------- kernel-level test hooks
+ * These run single ops of the hot path through the same kernels, for the
+ * parity tests at full size.  They may allocate device scratch.
+ * mggcn_debug_spmm: out = Â'^T B (dir 0) or Â' B (dir 1) for the model's
+ *   rows, B = the model's n_local... all n rows of the permuted operand in
+ *   loopback mode / P = 1 (device, ld = ldb), through the staged pipeline.
+ * mggcn_debug_gemm: op 0: C = A·B (A MxK, B KxN); op 1: C = A·B^T (B NxK);
+ *   op 2: C = A^T·B (A KxM, B KxN).  Device pointers, tcgen05 path. */
+int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int64_t ldb, int32_t width, float* out,
+                     int64_t ldo);
+int mggcn_debug_gemm(int32_t op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+                     int64_t ldb, float* C, int64_t ldc, uint32_t flags, uintptr_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MGGCN_H */

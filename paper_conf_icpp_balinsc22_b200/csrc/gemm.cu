@@ -1,0 +1,501 @@
+// gemm.cu — tcgen05 / TMA / TMEM GEMM for the dense products of MG-GCN on
+// sm_100a (F1, B2, B3 of SURVEY §8a):
+//     Eq. 5   HW  = H · W            op 0 (also the S-order (Â^T H) · W)
+//     Eq. 11  H_G = HW_G · W^T        op 1 (+ fused ReLU' mask of Eq. 8, Eq. 21 in place)
+//     Eq. 10  W_G = H^T · HW_G        op 2 (tall-skinny, split-K, reading C2)
+//
+// The paper uses cuBLAS row-major SGEMM and states no precision
+// (reading C17).  Here the fp32 operands are staged in shared memory by TMA,
+// split in shared memory by 4 "transform" warps into tf32 hi + lo parts (and
+// transposed into the K-major SWIZZLE_128B layout when the operand is stored
+// K-outer), and one thread issues tcgen05.mma.kind::tf32 for hi·hi + hi·lo +
+// lo·hi (3xTF32, ~fp32 accuracy) into a TMEM accumulator; 4 epilogue warps
+// drain TMEM with tcgen05.ld, apply the fused epilogue and store.
+//
+// Warp roles (320 threads, one CTA per SM, persistent over output tiles):
+//   warps 0-3 epilogue (TMEM lane quadrants 0-3), warps 4-7 transform,
+//   warp 8 TMA producer, warp 9 TMEM allocator + MMA issuer.
+// Pipelines (mbarriers): raw[2] TMA -> transform, split[2] transform -> MMA,
+// accumulator[2] MMA -> epilogue (double-buffered TMEM, 2 x 128 columns).
+#include <cuda.h>
+
+#include <mutex>
+
+#include "kernels.cuh"
+
+namespace mggcn {
+
+namespace {
+
+constexpr int BM = 128;          // UMMA_M (cta_group::1)
+constexpr int BK = 32;           // 32 fp32 = 128 B = one SWIZZLE_128B row
+constexpr int kMaxBN = 128;
+constexpr int kThreads = 320;
+constexpr int kXfWarp0 = 4, kTmaWarp = 8, kMmaWarp = 9;
+constexpr int kTmemCols = 256;   // 2 accumulators x 128 columns
+
+// shared-memory map (bytes from a 1024-B aligned base)
+constexpr int kRawA = 0;                    // 2 x 16 KB
+constexpr int kRawB = 2 * 16384;            // 2 x 16 KB
+constexpr int kAhi = 4 * 16384;
+constexpr int kAlo = 6 * 16384;
+constexpr int kBhi = 8 * 16384;
+constexpr int kBlo = 10 * 16384;
+constexpr int kBars = 12 * 16384;           // 12 mbarriers + TMEM slot
+constexpr int kSmemBytes = kBars + 256 + 1024;
+
+struct KParams {
+    int M, N, K;
+    int BN, m_tiles, n_tiles, k_chunks, k_chunk_len;
+    float* C;
+    int64_t ldc;
+    float* partial;
+    const float* rowscale;
+    int flags;
+    int op2;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* tm, int c0, int c1, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+            smem_u32(dst)),
+        "l"((uint64_t)tm), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+        : "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// K-major, SWIZZLE_128B shared-memory matrix descriptor (sm_100 format):
+// start>>4 [0,14), LBO>>4 [16,30) (unused for swizzled K-major), SBO>>4 [32,46)
+// = 1024 B between 8-row groups, version 1 at [46,48), layout 2 = SW128 at [61,64).
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
+    return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+           ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+
+__device__ __forceinline__ void mma_tf32(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                         uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+        : "memory");
+}
+
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+                 : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
+    uint32_t r[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+// fp32 -> (hi, lo) with hi exactly representable in tf32 (10-bit mantissa).
+__device__ __forceinline__ void split_tf32(float x, float& hi, float& lo, bool x1) {
+    if (x1) {
+        uint32_t t;
+        asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(t) : "f"(x));
+        hi = __uint_as_float(t);
+        lo = 0.f;
+    } else {
+        hi = __uint_as_float(__float_as_uint(x) & 0xFFFFE000u);
+        lo = x - hi;
+    }
+}
+
+__device__ __forceinline__ void split4(float4 x, float4& hi, float4& lo, bool x1) {
+    split_tf32(x.x, hi.x, lo.x, x1);
+    split_tf32(x.y, hi.y, lo.y, x1);
+    split_tf32(x.z, hi.z, lo.z, x1);
+    split_tf32(x.w, hi.w, lo.w, x1);
+}
+
+// Operand tile of `rows` x 32 k.  NOT transposed: raw is already the K-major
+// SW128 image written by TMA -> elementwise split at identical offsets.
+// Transposed: raw[kk][r] (pitch `rows` floats) -> K-major SW128:
+// element (r, k) lives at r*128 + (((k>>2) ^ (r&7)) << 4) + (k&3)*4.
+template <bool TRANS>
+__device__ __forceinline__ void transform_tile(const uint8_t* raw, uint8_t* hi, uint8_t* lo, int rows, int t,
+                                               bool x1) {
+    const int nchunks = rows * 8;   // 16-B chunks
+    if (!TRANS) {
+        const float4* src = reinterpret_cast<const float4*>(raw);
+        float4* h = reinterpret_cast<float4*>(hi);
+        float4* l = reinterpret_cast<float4*>(lo);
+        for (int c = t; c < nchunks; c += 128) {
+            float4 a = src[c], ah, al;
+            split4(a, ah, al, x1);
+            h[c] = ah;
+            if (!x1) l[c] = al;
+        }
+    } else {
+        const float* src = reinterpret_cast<const float*>(raw);
+        for (int idx = t; idx < nchunks; idx += 128) {
+            const int r = idx % rows, kq = idx / rows;
+            float4 a;
+            a.x = src[(4 * kq + 0) * rows + r];
+            a.y = src[(4 * kq + 1) * rows + r];
+            a.z = src[(4 * kq + 2) * rows + r];
+            a.w = src[(4 * kq + 3) * rows + r];
+            float4 ah, al;
+            split4(a, ah, al, x1);
+            const int off = r * 128 + ((kq ^ (r & 7)) << 4);
+            *reinterpret_cast<float4*>(hi + off) = ah;
+            if (!x1) *reinterpret_cast<float4*>(lo + off) = al;
+        }
+    }
+}
+
+__device__ __forceinline__ void decode_tile(const KParams& p, int tile, int& mt, int& nt, int& kc) {
+    nt = tile % p.n_tiles;
+    const int rest = tile / p.n_tiles;
+    mt = rest % p.m_tiles;
+    kc = rest / p.m_tiles;
+}
+
+template <bool AT, bool BT>
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_tf32_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const KParams p) {
+    extern __shared__ uint8_t smem_dyn[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_dyn) + 1023) & ~uintptr_t(1023));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kBars);
+    uint64_t* raw_full = bars + 0;
+    uint64_t* raw_empty = bars + 2;
+    uint64_t* split_full = bars + 4;
+    uint64_t* split_empty = bars + 6;
+    uint64_t* tmem_full = bars + 8;
+    uint64_t* tmem_empty = bars + 10;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 12);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const bool x1 = (p.flags & GEMM_TF32X1) != 0;
+    const int BN = p.BN;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(raw_full + s, 1);
+            mbar_init(raw_empty + s, 128);
+            mbar_init(split_full + s, 128);
+            mbar_init(split_empty + s, 1);
+            mbar_init(tmem_full + s, 1);
+            mbar_init(tmem_empty + s, 128);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == kMmaWarp) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(kTmemCols));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    const int total_tiles = p.m_tiles * p.n_tiles * p.k_chunks;
+
+    if (warp == kTmaWarp) {
+        if (lane == 0) {
+            const uint32_t bytes = (uint32_t)(BM * BK * 4 + BN * BK * 4);
+            uint32_t it = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                int mt, nt, kc;
+                decode_tile(p, tile, mt, nt, kc);
+                const int k0 = kc * p.k_chunk_len;
+                const int k1 = min(p.K, k0 + p.k_chunk_len);
+                for (int k = k0; k < k1; k += BK, ++it) {
+                    const int s = it & 1;
+                    const uint32_t ph = (it >> 1) & 1;
+                    mbar_wait(raw_empty + s, ph ^ 1);
+                    mbar_expect_tx(raw_full + s, bytes);
+                    if (AT) tma_load_2d(smem + kRawA + s * 16384, &tmA, mt * BM, k, raw_full + s);
+                    else tma_load_2d(smem + kRawA + s * 16384, &tmA, k, mt * BM, raw_full + s);
+                    if (BT) tma_load_2d(smem + kRawB + s * 16384, &tmB, nt * BN, k, raw_full + s);
+                    else tma_load_2d(smem + kRawB + s * 16384, &tmB, k, nt * BN, raw_full + s);
+                }
+            }
+        }
+    } else if (warp >= kXfWarp0 && warp < kXfWarp0 + 4) {
+        const int t = threadIdx.x - kXfWarp0 * 32;
+        uint32_t it = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+            int mt, nt, kc;
+            decode_tile(p, tile, mt, nt, kc);
+            const int k0 = kc * p.k_chunk_len;
+            const int k1 = min(p.K, k0 + p.k_chunk_len);
+            for (int k = k0; k < k1; k += BK, ++it) {
+                const int s = it & 1;
+                const uint32_t ph = (it >> 1) & 1;
+                mbar_wait(raw_full + s, ph);
+                mbar_wait(split_empty + s, ph ^ 1);
+                transform_tile<AT>(smem + kRawA + s * 16384, smem + kAhi + s * 16384, smem + kAlo + s * 16384, BM, t,
+                                   x1);
+                transform_tile<BT>(smem + kRawB + s * 16384, smem + kBhi + s * 16384, smem + kBlo + s * 16384, BN, t,
+                                   x1);
+                fence_proxy_async();
+                mbar_arrive(raw_empty + s);
+                mbar_arrive(split_full + s);
+            }
+        }
+    } else if (warp == kMmaWarp) {
+        if (lane == 0) {
+            // instruction descriptor: D f32, A/B tf32, both K-major, N>>3 at 17, M>>4 at 24
+            const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
+                                   ((uint32_t)(BM >> 4) << 24);
+            uint32_t it = 0, tc = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
+                int mt, nt, kc;
+                decode_tile(p, tile, mt, nt, kc);
+                const int k0 = kc * p.k_chunk_len;
+                const int k1 = min(p.K, k0 + p.k_chunk_len);
+                const int acc = tc & 1;
+                const uint32_t aph = (tc >> 1) & 1;
+                mbar_wait(tmem_empty + acc, aph ^ 1);
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + (uint32_t)(acc * kMaxBN);
+                bool first = true;
+                for (int k = k0; k < k1; k += BK, ++it) {
+                    const int s = it & 1;
+                    const uint32_t ph = (it >> 1) & 1;
+                    mbar_wait(split_full + s, ph);
+                    tc_fence_after();
+                    const uint64_t ah = sw128_desc(smem_u32(smem + kAhi + s * 16384));
+                    const uint64_t al = sw128_desc(smem_u32(smem + kAlo + s * 16384));
+                    const uint64_t bh = sw128_desc(smem_u32(smem + kBhi + s * 16384));
+                    const uint64_t bl = sw128_desc(smem_u32(smem + kBlo + s * 16384));
+#pragma unroll
+                    for (int kk = 0; kk < BK / 8; ++kk) {
+                        const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);   // 32 B per UMMA_K=8 step
+                        mma_tf32(d_tmem, ah + adv, bh + adv, idesc, first ? 0u : 1u);
+                        first = false;
+                        if (!x1) {
+                            mma_tf32(d_tmem, ah + adv, bl + adv, idesc, 1u);
+                            mma_tf32(d_tmem, al + adv, bh + adv, idesc, 1u);
+                        }
+                    }
+                    mma_commit(split_empty + s);
+                }
+                mma_commit(tmem_full + acc);
+            }
+        }
+    } else {
+        // epilogue warps 0-3: TMEM lane quadrant = warp
+        uint32_t tc = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
+            int mt, nt, kc;
+            decode_tile(p, tile, mt, nt, kc);
+            const int acc = tc & 1;
+            const uint32_t aph = (tc >> 1) & 1;
+            mbar_wait(tmem_full + acc, aph);
+            tc_fence_after();
+            const int row = mt * BM + warp * 32 + lane;
+            const int n0 = nt * BN;
+            for (int c0 = 0; c0 < BN; c0 += 16) {
+                float v[16];
+                tmem_ld16(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)(acc * kMaxBN + c0), v);
+                if (row >= p.M) continue;
+                const int nb = n0 + c0;
+                if (nb >= p.N) continue;
+                if (p.op2) {
+                    float* dst = p.partial + ((int64_t)kc * p.M + row) * (int64_t)p.N + nb;
+#pragma unroll
+                    for (int i = 0; i < 16; ++i)
+                        if (nb + i < p.N) dst[i] = v[i];
+                    continue;
+                }
+                float* dst = p.C + (int64_t)row * p.ldc + nb;
+                const float sc = (p.flags & GEMM_SCALE) ? __ldg(p.rowscale + row) : 1.f;
+                if (nb + 16 <= p.N) {
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+                        if (p.flags & GEMM_MASK) {
+                            const float4 old = reinterpret_cast<const float4*>(dst)[q];
+                            o.x = old.x > 0.f ? o.x : 0.f;
+                            o.y = old.y > 0.f ? o.y : 0.f;
+                            o.z = old.z > 0.f ? o.z : 0.f;
+                            o.w = old.w > 0.f ? o.w : 0.f;
+                        }
+                        o.x *= sc; o.y *= sc; o.z *= sc; o.w *= sc;
+                        if (p.flags & GEMM_RELU) {
+                            o.x = fmaxf(o.x, 0.f); o.y = fmaxf(o.y, 0.f);
+                            o.z = fmaxf(o.z, 0.f); o.w = fmaxf(o.w, 0.f);
+                        }
+                        reinterpret_cast<float4*>(dst)[q] = o;
+                    }
+                } else {
+                    for (int i = 0; i < 16 && nb + i < p.N; ++i) {
+                        float o = v[i];
+                        if ((p.flags & GEMM_MASK) && !(dst[i] > 0.f)) o = 0.f;
+                        o *= sc;
+                        if (p.flags & GEMM_RELU) o = fmaxf(o, 0.f);
+                        dst[i] = o;
+                    }
+                }
+            }
+            tc_fence_before();
+            mbar_arrive(tmem_empty + acc);
+        }
+    }
+    __syncthreads();
+    if (warp == kMmaWarp) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(kTmemCols));
+    }
+}
+
+// --------------------------------------------------------------- host side
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode() {
+    static EncodeTiledFn fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* f = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(f);
+    });
+    return fn;
+}
+
+// 2-D fp32 tensor map: dim0 = contiguous extent, dim1 = rows with stride ld floats.
+int encode2d(CUtensorMap* m, const float* base, int64_t dim0, int64_t dim1, int64_t ld, int box0, int box1,
+             bool swizzle128) {
+    EncodeTiledFn fn = get_encode();
+    if (!fn) return -1;
+    cuuint64_t dims[2] = {(cuuint64_t)dim0, (cuuint64_t)dim1};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+    cuuint32_t box[2] = {(cuuint32_t)box0, (cuuint32_t)box1};
+    cuuint32_t es[2] = {1, 1};
+    CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, es,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE,
+                    swizzle128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : -2;
+}
+
+int num_sms() {
+    static int n = 0;
+    if (n == 0) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+template <bool AT, bool BT>
+cudaError_t launch_kernel(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaError_t e = cudaFuncSetAttribute(gemm_tf32_kernel<AT, BT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             kSmemBytes);
+        if (e != cudaSuccess) return e;
+        attr_set = true;
+    }
+    gemm_tf32_kernel<AT, BT><<<g.grid, kThreads, kSmemBytes, s>>>(g.tmA, g.tmB, kp);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+int gemm_plan(GemmPlan& g, int op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+              int64_t ldb, float* C, int64_t ldc, int flags, size_t* partial_floats) {
+    if (M <= 0 || N <= 0 || K <= 0 || M >= (1 << 30) || K >= (1 << 30) || N > 65536) return -1;
+    if ((lda & 3) || (ldb & 3) || (reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
+        return -1;
+    g = GemmPlan();
+    g.op = op;
+    g.M = M; g.N = N; g.K = K;
+    g.n_tiles = (int)((N + kMaxBN - 1) / kMaxBN);
+    g.BN = (int)(((N + g.n_tiles - 1) / g.n_tiles + 15) / 16 * 16);
+    g.m_tiles = (int)((M + BM - 1) / BM);
+    g.C = C;
+    g.ldc = ldc;
+    g.flags = flags;
+    g.k_chunks = 1;
+    g.k_chunk_len = (K + BK - 1) / BK * BK;
+    if (op == 2) {
+        const int mn = g.m_tiles * g.n_tiles;
+        int want = (num_sms() + mn - 1) / mn;
+        const int64_t kblocks = (K + BK - 1) / BK;
+        if (want > kblocks) want = (int)kblocks;
+        if (want < 1) want = 1;
+        g.k_chunk_len = (kblocks + want - 1) / want * BK;
+        g.k_chunks = (int)((K + g.k_chunk_len - 1) / g.k_chunk_len);
+        if (partial_floats) *partial_floats = (size_t)g.k_chunks * (size_t)M * (size_t)N;
+    } else if (partial_floats) {
+        *partial_floats = 0;
+    }
+    int rc;
+    // A operand: op 0/1 A is M x K (K contiguous); op 2 A is K x M (M contiguous)
+    if (op == 2) rc = encode2d(&g.tmA, A, M, K, lda, BM, BK, false);
+    else rc = encode2d(&g.tmA, A, K, M, lda, BK, BM, true);
+    if (rc) return rc;
+    // B operand: op 0 and 2: B is K x N (N contiguous); op 1: B is N x K (K contiguous)
+    if (op == 1) rc = encode2d(&g.tmB, B, K, N, ldb, BK, g.BN, true);
+    else rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, BK, false);
+    if (rc) return rc;
+    const int total = g.m_tiles * g.n_tiles * g.k_chunks;
+    g.grid = total < num_sms() ? total : num_sms();
+    return 0;
+}
+
+cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
+    KParams kp;
+    kp.M = (int)g.M; kp.N = (int)g.N; kp.K = (int)g.K;
+    kp.BN = g.BN; kp.m_tiles = g.m_tiles; kp.n_tiles = g.n_tiles;
+    kp.k_chunks = g.k_chunks; kp.k_chunk_len = (int)g.k_chunk_len;
+    kp.C = g.C; kp.ldc = g.ldc; kp.partial = g.partial; kp.rowscale = g.rowscale;
+    kp.flags = g.flags; kp.op2 = g.op == 2;
+    switch (g.op) {
+        case 0: return launch_kernel<false, true>(g, kp, s);
+        case 1: return launch_kernel<false, false>(g, kp, s);
+        case 2: return launch_kernel<true, true>(g, kp, s);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+}  // namespace mggcn

@@ -1,0 +1,96 @@
+// kernels.cuh — launch interface of the sm_100a kernels (internal).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace mggcn {
+
+// process-wide count of kernel launches issued by this library
+void count_launches(int n);
+
+// ------------------------------------------------------------------ SpMM
+// One stage of the staged SpMM: out_i (+)= T_ij · B_j for one
+// tile T (CSR, local indices).  Work is pre-cut on the host into items
+// {row, beg, end, slot}: rows with <= kSplit entries are one item written
+// directly (slot = -1); longer rows (R-MAT hubs) are cut into kSplit-entry
+// segments whose partial sums go to `partial[slot]` and are combined in
+// segment order by a fix-up kernel (deterministic, no float atomics).
+constexpr int kSplit = 2048;
+
+struct SpmmTile {
+    const int4* items = nullptr;   // {row, beg, end, slot}
+    int64_t n_items = 0;
+    const int4* splits = nullptr;  // {row, first_slot, nslots, 0}
+    int64_t n_splits = 0;
+    int64_t n_slots = 0;
+    const int32_t* col = nullptr;
+    const float* val = nullptr;    // nullptr => pattern-only (value 1)
+    int64_t nnz = 0, nrows = 0, ncols = 0;
+};
+
+enum SpmmFlags : int { SPMM_ACCUM = 1, SPMM_LAST = 2, SPMM_RELU = 4 };
+
+// width: columns to compute (multiple of 4, <= ldb, <= ldo); B and out 16-B aligned.
+// rowscale (nullable): multiplies the finished row on the LAST stage.
+cudaError_t launch_spmm(const SpmmTile& t, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
+                        const float* rowscale, int width, int flags, cudaStream_t s);
+
+// ------------------------------------------------------------------ GEMM
+// tcgen05 (kind::tf32) GEMM with TMA-staged operands and TMEM accumulators.
+// op 0: C = A·B   (A M x K row-major, B K x N row-major)     [Eq. 5, S-order T·W]
+// op 1: C = A·B^T (A M x K, B N x K)                         [Eq. 11]
+// op 2: C = A^T·B (A K x M, B K x N), split-K partials       [Eq. 10]
+// The fp32 operands are split into tf32 hi + lo in shared memory and the
+// product is hi·hi + hi·lo + lo·hi (3xTF32) unless GEMM_TF32X1.
+enum GemmFlags : int {
+    GEMM_RELU = 1,     // C = max(C, 0)
+    GEMM_MASK = 2,     // C = C * [C_old > 0]  (ReLU' of Eq. 8 read from the buffer being overwritten)
+    GEMM_SCALE = 4,    // C *= rowscale[row]   (inv_deg pre-scale for the next pattern SpMM)
+    GEMM_TF32X1 = 16,
+};
+
+struct GemmPlan {
+    int op = 0;
+    int64_t M = 0, N = 0, K = 0;
+    int BN = 0, m_tiles = 0, n_tiles = 0, k_chunks = 1;
+    int64_t k_chunk_len = 0;
+    CUtensorMap tmA, tmB;
+    float* C = nullptr;
+    int64_t ldc = 0;
+    float* partial = nullptr;   // op 2: [k_chunks][M][N]
+    const float* rowscale = nullptr;
+    int flags = 0;
+    int grid = 0;
+};
+
+// Builds tensor maps + tiling.  A/B pointers must be 16-B aligned, lda/ldb
+// multiples of 4 floats.  For op 2 returns the partial-buffer size needed.
+int gemm_plan(GemmPlan& p, int op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+              int64_t ldb, float* C, int64_t ldc, int flags, size_t* partial_floats);
+cudaError_t gemm_launch(const GemmPlan& p, cudaStream_t s);
+// op 2 second pass: C[m][n] (ldc) = sum_kc partial[kc][m][n], in kc order.
+cudaError_t launch_splitk_reduce(const float* partial, int k_chunks, int64_t M, int64_t N, float* C, int64_t ldc,
+                                 cudaStream_t s);
+
+// ------------------------------------------------------------------ misc
+// Softmax-CE forward + backward fused (Eq. 19 in place):
+// Z (n x C, ld) holds logits on entry and dLoss/dZ on exit (times
+// rowscale[row] if non-null; times [Z > 0] if relu_last).  Per-block fp64
+// partial loss sums into block_partial[grid].
+constexpr int kCeBlocks = 592;
+cudaError_t launch_softmax_ce(float* Z, int64_t n, int C, int64_t ld, const int32_t* y, const int64_t* ntrain,
+                              const float* rowscale, int relu_last, double* block_partial, cudaStream_t s);
+cudaError_t launch_sum_partials(const double* partial, int count, double* out, cudaStream_t s);
+cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* out, cudaStream_t s);
+cudaError_t launch_adam(float* W, const float* g, float* m, float* v, int64_t count, double lr, double b1,
+                        double b2, double eps, int64_t t, cudaStream_t s);
+// out[i] = sum_r in[r][i] in r order (loopback "all-reduce").
+cudaError_t launch_sum_buffers(const float* const* in, int nin, float* out, int64_t count, cudaStream_t s);
+cudaError_t launch_sum_i64(const int64_t* in, int nin, int64_t* out, cudaStream_t s);
+cudaError_t launch_sum_f64(const double* in, int nin, double* out, cudaStream_t s);
+cudaError_t launch_scale_rows(const float* in, int64_t ldi, float* out, int64_t ldo, int64_t n, int width,
+                              const float* rowscale, cudaStream_t s);
+
+}  // namespace mggcn

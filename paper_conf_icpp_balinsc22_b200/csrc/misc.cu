@@ -1,0 +1,244 @@
+// misc.cu — loss layer, Adam and small reductions (sm_100a).
+//
+// Softmax cross-entropy: P:1244-1246 ("softmax cross-entropy loss [9]"),
+// forward and backward fused into one warp-per-row pass whose gradient
+// overwrites the logits in place (Eq. 19: AHW_G -> AHWB).  Adam: P:1244 with
+// ref [23] (Kingma & Ba), reading C6.  All reductions run in a fixed order
+// (no floating-point atomics) so results are bitwise reproducible.
+#include <atomic>
+#include <cmath>
+
+#include "kernels.cuh"
+
+namespace mggcn {
+
+namespace {
+
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+__device__ __forceinline__ double warp_sum_d(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+constexpr int kCeWarps = 8;
+
+// Each warp owns a fixed, strided set of rows; per-warp fp64 loss sums are
+// combined in warp order, giving one partial per block (deterministic).
+__global__ void __launch_bounds__(kCeWarps * 32)
+softmax_ce_kernel(float* __restrict__ Z, int64_t n, int C, int64_t ld, const int32_t* __restrict__ y,
+                  const int64_t* __restrict__ ntrain, const float* __restrict__ rowscale, int relu_last,
+                  double* __restrict__ block_partial) {
+    __shared__ double wsum[kCeWarps];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t gw = (int64_t)blockIdx.x * kCeWarps + wid, nw = (int64_t)gridDim.x * kCeWarps;
+    const float inv_nt = 1.0f / (float)(*ntrain > 0 ? *ntrain : 1);
+    double lsum = 0.0;
+    for (int64_t r = gw; r < n; r += nw) {
+        float* z = Z + r * ld;
+        const int lab = y[r];
+        if (lab < 0) {
+            for (int c = lane; c < C; c += 32) z[c] = 0.f;
+            continue;
+        }
+        float mx = -INFINITY;
+        for (int c = lane; c < C; c += 32) mx = fmaxf(mx, z[c]);
+        mx = warp_max(mx);
+        float s = 0.f;
+        for (int c = lane; c < C; c += 32) s += expf(z[c] - mx);
+        s = warp_sum(s);
+        const float lse = mx + logf(s);
+        const float zy = z[lab];   // every lane reads the same address
+        if (lane == 0) lsum += (double)lse - (double)zy;
+        const float sc = inv_nt * (rowscale ? rowscale[r] : 1.f);
+        for (int c = lane; c < C; c += 32) {
+            const float zc = z[c];
+            float g = expf(zc - lse) - (c == lab ? 1.f : 0.f);
+            if (relu_last && !(zc > 0.f)) g = 0.f;
+            z[c] = g * sc;
+        }
+    }
+    if (lane == 0) wsum[wid] = lsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < kCeWarps; ++w) t += wsum[w];
+        block_partial[blockIdx.x] = t;
+    }
+}
+
+__global__ void sum_partials_kernel(const double* __restrict__ p, int count, double* __restrict__ out) {
+    // one warp, strided lane sums then fixed xor tree
+    double t = 0.0;
+    for (int i = threadIdx.x; i < count; i += 32) t += p[i];
+    t = warp_sum_d(t);
+    if (threadIdx.x == 0) *out = t;
+}
+
+__global__ void count_labelled_kernel(const int32_t* __restrict__ y, int64_t n, int64_t* __restrict__ out) {
+    __shared__ long long ws[32];
+    long long c = 0;
+    for (int64_t i = threadIdx.x; i < n; i += blockDim.x) c += y[i] >= 0 ? 1 : 0;
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long t = 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += ws[w];
+        *out = t;
+    }
+}
+
+// Adam (Kingma & Ba, Alg. 1): bias-corrected, eps outside the sqrt.
+__global__ void adam_kernel(float* __restrict__ W, const float* __restrict__ g, float* __restrict__ m,
+                            float* __restrict__ v, int64_t count, double lr, double b1, double b2, double eps,
+                            double c1, double c2) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+        const double gi = g[i];
+        const double mi = b1 * (double)m[i] + (1.0 - b1) * gi;
+        const double vi = b2 * (double)v[i] + (1.0 - b2) * gi * gi;
+        m[i] = (float)mi;
+        v[i] = (float)vi;
+        W[i] = (float)((double)W[i] - lr * (mi / c1) / (sqrt(vi / c2) + eps));
+    }
+}
+
+struct PtrArray {
+    const float* p[64];
+};
+
+__global__ void sum_buffers_kernel(PtrArray in, int nin, float* __restrict__ out, int64_t count) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+        float t = in.p[0][i];
+        for (int r = 1; r < nin; ++r) t += in.p[r][i];
+        out[i] = t;
+    }
+}
+
+__global__ void sum_i64_kernel(const int64_t* in, int nin, int64_t* out) {
+    int64_t t = 0;
+    for (int r = 0; r < nin; ++r) t += in[r];
+    *out = t;
+}
+
+__global__ void sum_f64_kernel(const double* in, int nin, double* out) {
+    double t = 0;
+    for (int r = 0; r < nin; ++r) t += in[r];
+    *out = t;
+}
+
+__global__ void scale_rows_kernel(const float* __restrict__ in, int64_t ldi, float* __restrict__ out, int64_t ldo,
+                                  int64_t n, int width, const float* __restrict__ rowscale) {
+    const int64_t total = n * width;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / width;
+        const int c = (int)(i % width);
+        out[r * ldo + c] = in[r * ldi + c] * (rowscale ? rowscale[r] : 1.f);
+    }
+}
+
+__global__ void splitk_reduce_kernel(const float* __restrict__ partial, int k_chunks, int64_t M, int64_t N,
+                                     float* __restrict__ C, int64_t ldc) {
+    const int64_t total = M * N;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        float t = 0.f;
+        for (int k = 0; k < k_chunks; ++k) t += partial[(int64_t)k * total + i];
+        C[(i / N) * ldc + (i % N)] = t;
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_softmax_ce(float* Z, int64_t n, int C, int64_t ld, const int32_t* y, const int64_t* ntrain,
+                              const float* rowscale, int relu_last, double* block_partial, cudaStream_t s) {
+    softmax_ce_kernel<<<kCeBlocks, kCeWarps * 32, 0, s>>>(Z, n, C, ld, y, ntrain, rowscale, relu_last, block_partial);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sum_partials(const double* partial, int count, double* out, cudaStream_t s) {
+    sum_partials_kernel<<<1, 32, 0, s>>>(partial, count, out);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* out, cudaStream_t s) {
+    count_labelled_kernel<<<1, 1024, 0, s>>>(y, n, out);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_adam(float* W, const float* g, float* m, float* v, int64_t count, double lr, double b1, double b2,
+                        double eps, int64_t t, cudaStream_t s) {
+    const double c1 = 1.0 - std::pow(b1, (double)t), c2 = 1.0 - std::pow(b2, (double)t);
+    int blocks = (int)((count + 255) / 256);
+    if (blocks > 1184) blocks = 1184;
+    if (blocks < 1) blocks = 1;
+    adam_kernel<<<blocks, 256, 0, s>>>(W, g, m, v, count, lr, b1, b2, eps, c1, c2);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sum_buffers(const float* const* in, int nin, float* out, int64_t count, cudaStream_t s) {
+    if (nin < 1 || nin > 64) return cudaErrorInvalidValue;
+    PtrArray a{};
+    for (int i = 0; i < nin; ++i) a.p[i] = in[i];
+    int blocks = (int)((count + 255) / 256);
+    if (blocks > 1184) blocks = 1184;
+    if (blocks < 1) blocks = 1;
+    sum_buffers_kernel<<<blocks, 256, 0, s>>>(a, nin, out, count);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sum_i64(const int64_t* in, int nin, int64_t* out, cudaStream_t s) {
+    sum_i64_kernel<<<1, 1, 0, s>>>(in, nin, out);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_sum_f64(const double* in, int nin, double* out, cudaStream_t s) {
+    sum_f64_kernel<<<1, 1, 0, s>>>(in, nin, out);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_scale_rows(const float* in, int64_t ldi, float* out, int64_t ldo, int64_t n, int width,
+                              const float* rowscale, cudaStream_t s) {
+    int64_t total = n * width;
+    int blocks = (int)((total + 255) / 256);
+    if (blocks > 4736) blocks = 4736;
+    if (blocks < 1) blocks = 1;
+    scale_rows_kernel<<<blocks, 256, 0, s>>>(in, ldi, out, ldo, n, width, rowscale);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_splitk_reduce(const float* partial, int k_chunks, int64_t M, int64_t N, float* C, int64_t ldc,
+                                 cudaStream_t s) {
+    int64_t total = M * N;
+    int blocks = (int)((total + 255) / 256);
+    if (blocks > 1184) blocks = 1184;
+    if (blocks < 1) blocks = 1;
+    splitk_reduce_kernel<<<blocks, 256, 0, s>>>(partial, k_chunks, M, N, C, ldc);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+}  // namespace mggcn
+
+namespace mggcn {
+static std::atomic<long long> g_launches{0};
+void count_launches(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+}  // namespace mggcn
+
+extern "C" int64_t mggcn_kernel_launch_count(void) { return (int64_t)mggcn::g_launches.load(); }

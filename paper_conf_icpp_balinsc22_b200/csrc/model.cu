@@ -1,0 +1,1186 @@
+// model.cu — executor of the MG-GCN hot path on B200: buffer plan (§4.2,
+// P:827-901), staged SpMM with double-buffered broadcast (§4.1 P:705-720,
+// §4.3), per-layer order choice (§4.4), loss, backward
+// (Eq. 8-11), W_G reduction and Adam.
+//
+// Streams: stream 0 = compute, stream 1 = communication.
+// Communication is NCCL (one process per GPU, nlocal = 1) or, for testing
+// the P-stage pipeline on one GPU, LOOPBACK (all P ranks in this model,
+// broadcasts = device copies on the comm stream with the same event graph).
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <tuple>
+#include <vector>
+
+#include "internal.h"
+#include "kernels.cuh"
+
+using namespace mggcn;
+
+namespace {
+
+enum Order { G_ORDER = 0, S_ORDER = 1 };   // GeMM-first / SpMM-first (§4.4)
+enum State { ST_READY = 0, ST_FWD = 1, ST_BWD = 2 };
+enum ProfClass { PC_SPMM = 0, PC_GEMM, PC_LOSS, PC_ADAM, PC_BCAST, PC_ALLRED, PC_OTHER, PC_N };
+
+struct Bump {
+    char* base = nullptr;
+    size_t off = 0;
+    template <typename T>
+    T* take(size_t count) {
+        off = (off + 255) & ~size_t(255);
+        T* p = base ? reinterpret_cast<T*>(base + off) : nullptr;
+        off += sizeof(T) * (count ? count : 1);
+        return p;
+    }
+};
+
+struct HostItems {
+    std::vector<int4> items, splits;
+    int64_t nslots = 0;
+};
+
+void build_items(const HostTile& t, HostItems& h) {
+    const auto& rp = t.rowptr;
+    for (int64_t r = 0; r < t.nrows; ++r) {
+        const int64_t len = rp[r + 1] - rp[r];
+        if (len > kSplit) {
+            const int64_t nseg = (len + kSplit - 1) / kSplit;
+            h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
+            for (int64_t s = 0; s < nseg; ++s) {
+                const int64_t b = rp[r] + s * kSplit, e = std::min<int64_t>(rp[r + 1], b + kSplit);
+                h.items.push_back(make_int4((int)r, (int)b, (int)e, (int)(h.nslots + s)));
+            }
+            h.nslots += nseg;
+        }
+    }
+    for (int64_t r = 0; r < t.nrows; ++r) {
+        const int64_t len = rp[r + 1] - rp[r];
+        if (len <= kSplit) h.items.push_back(make_int4((int)r, rp[r], rp[r + 1], -1));
+    }
+}
+
+struct Rank {
+    const mggcn_part_s* part = nullptr;
+    int rank = 0;
+    int64_t rows = 0, row_off = 0;   // row_off: offset inside the model's local rows
+    std::vector<SpmmTile> F, B;
+    std::vector<HostItems> hF, hB;
+    float* inv_deg = nullptr;
+    float* Xs = nullptr;
+    int32_t* y = nullptr;
+    float* T0 = nullptr;
+    float* HWB = nullptr;
+    float* BC[2] = {nullptr, nullptr};
+    std::vector<float*> AHWB;
+    float* spmm_partial = nullptr;
+    double* ce_partial = nullptr;
+    double* loss_local = nullptr;
+    int64_t* ntrain_local = nullptr;
+    float* WG_local = nullptr;
+    float* gemm_partial = nullptr;
+    cudaEvent_t ev_bc[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
+    // GEMM plans per layer: fwd (op 0), wgrad (op 2), igrad (op 1)
+    std::vector<GemmPlan> g_fwd, g_wgrad, g_igrad;
+    std::vector<int> has_fwd, has_wgrad, has_igrad;
+};
+
+}  // namespace
+
+struct mggcn_model_s {
+    int P = 1, nlocal = 1;
+    uint32_t flags = 0;
+    int L = 0;
+    std::vector<int64_t> d, ld;     // dims and padded leading dims (multiple of 4)
+    std::vector<int> order;
+    std::vector<int64_t> woff;      // per-layer offset into W/m/v/WG (floats)
+    int64_t wtotal = 0;
+    bool pattern = true;
+    int64_t n_local = 0;            // rows owned by this model (sum over local ranks)
+    int64_t max_rows_j = 0;
+    int64_t bc_ld = 0, hw_ld = 0;
+    std::vector<Rank> ranks;
+    float *W = nullptr, *Mom = nullptr, *Vel = nullptr, *WG = nullptr;
+    double* loss_sum = nullptr;
+    int64_t* ntrain = nullptr;
+    cudaStream_t cs = nullptr, ms = nullptr;
+    cudaEvent_t ev_begin = nullptr, ev_comm_end = nullptr, ev_tmp = nullptr, ev_wg = nullptr, ev_comm_done = nullptr;
+    ncclComm_t comm = nullptr;
+    int state = ST_READY;
+    int poisoned = 0;
+    int64_t t = 0;
+    bool need_wg_wait = false;
+    // profiling
+    std::vector<std::tuple<int, cudaEvent_t, cudaEvent_t>> prof_recs;
+    std::vector<cudaEvent_t> prof_pool;
+    double prof_ms[PC_N] = {0};
+    int64_t prof_n[PC_N] = {0};
+    // epoch work
+    double w_spmm_bytes = 0, w_gather_bytes = 0, w_gemm_flops = 0, w_bcast_bytes = 0;
+    // X staging plan bookkeeping
+    int layer_ids[64];
+};
+
+namespace {
+
+#define CK(expr)                                                                                \
+    do {                                                                                        \
+        cudaError_t _e = (expr);                                                                \
+        if (_e != cudaSuccess) {                                                                \
+            set_error(std::string("CUDA error: ") + cudaGetErrorString(_e) + " at " #expr);     \
+            return MGGCN_ECUDA;                                                                 \
+        }                                                                                       \
+    } while (0)
+
+#define NK(expr)                                                                                \
+    do {                                                                                        \
+        ncclResult_t _r = (expr);                                                               \
+        if (_r != ncclSuccess) {                                                                \
+            set_error(std::string("NCCL error: ") + ncclGetErrorString(_r) + " at " #expr);     \
+            return MGGCN_ENCCL;                                                                 \
+        }                                                                                       \
+    } while (0)
+
+#define RC(expr)                         \
+    do {                                 \
+        int _rc = (expr);                \
+        if (_rc != MGGCN_OK) return _rc; \
+    } while (0)
+
+// ---------------------------------------------------------------- profiling
+cudaEvent_t prof_event(mggcn_model_s* m) {
+    if (!m->prof_pool.empty()) {
+        cudaEvent_t e = m->prof_pool.back();
+        m->prof_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+
+struct ProfScope {
+    mggcn_model_s* m;
+    int cls;
+    cudaStream_t s;
+    cudaEvent_t a = nullptr;
+    ProfScope(mggcn_model_s* m_, int c, cudaStream_t s_) : m(m_), cls(c), s(s_) {
+        if (m->flags & MGGCN_F_PROFILE) {
+            a = prof_event(m);
+            cudaEventRecord(a, s);
+        }
+    }
+    ~ProfScope() {
+        if (a) {
+            cudaEvent_t b = prof_event(m);
+            cudaEventRecord(b, s);
+            m->prof_recs.emplace_back(cls, a, b);
+        }
+    }
+};
+
+// --------------------------------------------------------------- planning
+int64_t ld_of(int64_t d) { return round_up(d, 4); }
+
+int check_dims(int L, const int32_t* dims) {
+    if (L < 1 || L > 64 || !dims) {
+        set_error("model: L must be in [1, 64] and dims non-NULL");
+        return MGGCN_EINVAL;
+    }
+    for (int l = 0; l <= L; ++l)
+        if (dims[l] <= 0 || dims[l] > 65536) {
+            set_error("model: every d_l must be in [1, 65536]");
+            return MGGCN_EINVAL;
+        }
+    for (int l = 1; l < L; ++l)
+        if (dims[l] < dims[l + 1] && true) {
+            // SpMM-first at l > 0 (reading C22): needs a private T_l and a separate
+            // mask buffer for the backward SpMM; no BASELINE config uses it.
+            set_error("model: SpMM-first order (d_l < d_{l+1}) at layer l > 0 is not supported");
+            return MGGCN_EUNSUPPORTED;
+        }
+    return MGGCN_OK;
+}
+
+// Lays out (or sizes, when bump.base == nullptr) every device buffer.
+void plan_buffers(mggcn_model_s* m, Bump& b) {
+    const int L = m->L;
+    m->W = b.take<float>(m->wtotal);
+    m->Mom = b.take<float>(m->wtotal);
+    m->Vel = b.take<float>(m->wtotal);
+    m->WG = b.take<float>(m->wtotal);
+    m->loss_sum = b.take<double>(1);
+    m->ntrain = b.take<int64_t>(1);
+    for (auto& r : m->ranks) {
+        const mggcn_part_s* pt = r.part;
+        const int P = pt->P;
+        r.F.assign(P, SpmmTile());
+        r.B.assign(P, SpmmTile());
+        for (int j = 0; j < P; ++j) {
+            for (int dir = 0; dir < 2; ++dir) {
+                if (dir == 1 && pt->shared_fb) {
+                    r.B[j] = r.F[j];
+                    continue;
+                }
+                const HostTile& ht = dir == 0 ? pt->F[j] : pt->B[j];
+                const HostItems& hi = dir == 0 ? r.hF[j] : r.hB[j];
+                SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
+                t.nrows = ht.nrows;
+                t.ncols = ht.ncols;
+                t.nnz = ht.rowptr.back();
+                t.n_items = (int64_t)hi.items.size();
+                t.n_splits = (int64_t)hi.splits.size();
+                t.n_slots = hi.nslots;
+                t.items = b.take<int4>(hi.items.size());
+                t.splits = b.take<int4>(hi.splits.size());
+                t.col = b.take<int32_t>(ht.col.size());
+                t.val = pt->pattern ? nullptr : b.take<float>(ht.val.size());
+            }
+        }
+        r.inv_deg = b.take<float>(r.rows);
+        r.Xs = b.take<float>(r.rows * m->ld[0]);
+        r.y = b.take<int32_t>(r.rows);
+        r.T0 = m->order[0] == S_ORDER ? b.take<float>(r.rows * m->ld[0]) : nullptr;
+        r.HWB = b.take<float>(r.rows * std::max<int64_t>(m->hw_ld, 4));
+        if (P > 1) {
+            r.BC[0] = b.take<float>(m->max_rows_j * m->bc_ld);
+            r.BC[1] = b.take<float>(m->max_rows_j * m->bc_ld);
+        }
+        r.AHWB.assign(L, nullptr);
+        for (int l = 0; l < L; ++l) r.AHWB[l] = b.take<float>(r.rows * m->ld[l + 1]);
+        int64_t slots = 0;
+        for (int j = 0; j < P; ++j) {
+            slots = std::max(slots, r.hF[j].nslots);
+            if (!pt->shared_fb) slots = std::max(slots, r.hB[j].nslots);
+        }
+        r.spmm_partial = b.take<float>(slots * std::min<int64_t>(m->bc_ld, 512));
+        r.ce_partial = b.take<double>(kCeBlocks);
+        r.loss_local = b.take<double>(1);
+        r.ntrain_local = b.take<int64_t>(1);
+        r.WG_local = (m->nlocal > 1) ? b.take<float>(m->wtotal) : nullptr;
+        // split-K partial for W_G (op 2): k_chunks <= #SMs
+        size_t gp = 0;
+        for (int l = 0; l < L; ++l) gp = std::max(gp, (size_t)256 * (size_t)m->d[l] * (size_t)m->d[l + 1]);
+        r.gemm_partial = b.take<float>(gp);
+    }
+}
+
+int upload_static(mggcn_model_s* m) {
+    for (auto& r : m->ranks) {
+        const mggcn_part_s* pt = r.part;
+        for (int j = 0; j < pt->P; ++j)
+            for (int dir = 0; dir < 2; ++dir) {
+                if (dir == 1 && pt->shared_fb) continue;
+                const HostTile& ht = dir == 0 ? pt->F[j] : pt->B[j];
+                const HostItems& hi = dir == 0 ? r.hF[j] : r.hB[j];
+                SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
+                if (!hi.items.empty())
+                    CK(cudaMemcpyAsync(const_cast<int4*>(t.items), hi.items.data(), sizeof(int4) * hi.items.size(),
+                                       cudaMemcpyHostToDevice, m->cs));
+                if (!hi.splits.empty())
+                    CK(cudaMemcpyAsync(const_cast<int4*>(t.splits), hi.splits.data(),
+                                       sizeof(int4) * hi.splits.size(), cudaMemcpyHostToDevice, m->cs));
+                if (!ht.col.empty())
+                    CK(cudaMemcpyAsync(const_cast<int32_t*>(t.col), ht.col.data(), sizeof(int32_t) * ht.col.size(),
+                                       cudaMemcpyHostToDevice, m->cs));
+                if (t.val && !ht.val.empty())
+                    CK(cudaMemcpyAsync(const_cast<float*>(t.val), ht.val.data(), sizeof(float) * ht.val.size(),
+                                       cudaMemcpyHostToDevice, m->cs));
+            }
+        if (m->pattern && pt->shared_fb)
+            for (int j = 0; j < pt->P; ++j) r.B[j] = r.F[j];
+        CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
+        // zero every activation buffer once: padding columns stay 0 forever
+        CK(cudaMemsetAsync(r.Xs, 0, sizeof(float) * r.rows * m->ld[0], m->cs));
+        for (int l = 0; l < m->L; ++l)
+            CK(cudaMemsetAsync(r.AHWB[l], 0, sizeof(float) * r.rows * m->ld[l + 1], m->cs));
+        CK(cudaMemsetAsync(r.HWB, 0, sizeof(float) * r.rows * std::max<int64_t>(m->hw_ld, 4), m->cs));
+        if (r.T0) CK(cudaMemsetAsync(r.T0, 0, sizeof(float) * r.rows * m->ld[0], m->cs));
+        for (int s = 0; s < 2; ++s)
+            if (r.BC[s]) CK(cudaMemsetAsync(r.BC[s], 0, sizeof(float) * m->max_rows_j * m->bc_ld, m->cs));
+    }
+    CK(cudaMemsetAsync(m->W, 0, sizeof(float) * m->wtotal, m->cs));
+    CK(cudaMemsetAsync(m->Mom, 0, sizeof(float) * m->wtotal, m->cs));
+    CK(cudaMemsetAsync(m->Vel, 0, sizeof(float) * m->wtotal, m->cs));
+    CK(cudaMemsetAsync(m->WG, 0, sizeof(float) * m->wtotal, m->cs));
+    return MGGCN_OK;
+}
+
+// The input operand of layer l (H_l): staged X for l = 0, else H'_{l-1} in AHWB_{l-1}.
+float* layer_input(mggcn_model_s* m, Rank& r, int l) { return l == 0 ? r.Xs : r.AHWB[l - 1]; }
+
+int plan_gemms(mggcn_model_s* m) {
+    const int L = m->L;
+    const bool x1 = (m->flags & MGGCN_F_TF32X1) != 0;
+    for (auto& r : m->ranks) {
+        r.g_fwd.assign(L, GemmPlan());
+        r.g_wgrad.assign(L, GemmPlan());
+        r.g_igrad.assign(L, GemmPlan());
+        r.has_fwd.assign(L, 0);
+        r.has_wgrad.assign(L, 0);
+        r.has_igrad.assign(L, 0);
+        if (r.rows == 0) continue;
+        for (int l = 0; l < L; ++l) {
+            const bool relu_here = (l < L - 1) || (m->flags & MGGCN_F_RELU_LAST);
+            const float* Wl = m->W + m->woff[l];
+            int flags = x1 ? GEMM_TF32X1 : 0;
+            size_t pf = 0;
+            // forward: G-order HW = H W -> HWB ; S-order AHW = T W -> AHWB_l (+ReLU)
+            if (m->order[l] == G_ORDER) {
+                if (gemm_plan(r.g_fwd[l], 0, r.rows, m->d[l + 1], m->d[l], layer_input(m, r, l), m->ld[l], Wl,
+                              m->ld[l + 1], r.HWB, m->ld[l + 1], flags, &pf))
+                    goto fail;
+            } else {
+                if (gemm_plan(r.g_fwd[l], 0, r.rows, m->d[l + 1], m->d[l], r.T0, m->ld[0], Wl, m->ld[l + 1],
+                              r.AHWB[l], m->ld[l + 1], flags | (relu_here ? GEMM_RELU : 0), &pf))
+                    goto fail;
+            }
+            r.has_fwd[l] = 1;
+            // weight gradient (Eq. 10): W_G = H^T HW_G (G) or T^T Z_G (S)
+            {
+                const float* Aop = m->order[l] == G_ORDER ? layer_input(m, r, l) : r.T0;
+                const float* Bop = m->order[l] == G_ORDER ? r.HWB : r.AHWB[l];
+                const int64_t ldb = m->order[l] == G_ORDER ? m->ld[l + 1] : m->ld[l + 1];
+                if (gemm_plan(r.g_wgrad[l], 2, m->d[l], m->d[l + 1], r.rows, Aop, m->ld[l], Bop, ldb, nullptr, 0,
+                              flags, &pf))
+                    goto fail;
+                if (pf > (size_t)256 * (size_t)m->d[l] * (size_t)m->d[l + 1]) {
+                    set_error("model: split-K partial buffer too small");
+                    return MGGCN_EUNSUPPORTED;
+                }
+                r.g_wgrad[l].partial = r.gemm_partial;
+                r.has_wgrad[l] = 1;
+            }
+            // input gradient (Eq. 11) for l > 0 (G-order): AHWB_{l-1} = (HW_G W^T) * [H'_{l-1} > 0] (* inv_deg)
+            if (l > 0) {
+                int f = flags | GEMM_MASK;
+                if (m->order[l - 1] == G_ORDER && m->pattern) f |= GEMM_SCALE;
+                if (gemm_plan(r.g_igrad[l], 1, r.rows, m->d[l], m->d[l + 1], r.HWB, m->ld[l + 1], Wl, m->ld[l + 1],
+                              r.AHWB[l - 1], m->ld[l], f, &pf))
+                    goto fail;
+                r.g_igrad[l].rowscale = r.inv_deg;
+                r.has_igrad[l] = 1;
+            }
+        }
+    }
+    return MGGCN_OK;
+fail:
+    set_error("model: GEMM plan / tensor-map encoding failed (needs an sm_100 device)");
+    return MGGCN_ECUDA;
+}
+
+// --------------------------------------------------------- staged SpMM
+// C_r (+)= sum_j T_rj · S_j over stages; S_j = src(j) rows of rank j.
+// Local stage first, then ascending j (reading C13); broadcast q goes into
+// BC[k % 2] for the k-th remote stage; broadcast k waits for the SpMM of
+// remote stage k-2; SpMM k waits for broadcast k.
+struct SpmmJob {
+    int dir;                 // 0: F tiles (Â'^T), 1: B tiles (Â')
+    int64_t width;           // = ld of src/out (multiple of 4)
+    bool use_rowscale;       // inv_deg of the output row on the last stage
+    bool relu;
+    float* (*src)(mggcn_model_s*, Rank&, const void*);
+    float* (*dst)(mggcn_model_s*, Rank&, const void*);
+    const void* ctx;
+};
+
+int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags) {
+    const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
+    float* out = job.dst(m, r, job.ctx);
+    ProfScope ps(m, PC_SPMM, m->cs);
+    CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
+                   (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
+    return MGGCN_OK;
+}
+
+int remote_index(int q, int self) { return q < self ? q : q - 1; }
+
+int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
+    const int P = m->P;
+    const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
+    const bool overlap = (m->flags & MGGCN_F_OVERLAP) != 0;
+    if (P > 1) {
+        CK(cudaEventRecord(m->ev_begin, m->cs));
+        CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
+    }
+    // local stage
+    for (auto& r : m->ranks) {
+        if (r.rows == 0) continue;
+        const int last = (P == 1) ? SPMM_LAST : 0;
+        RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), last));
+    }
+    if (P == 1) return MGGCN_OK;
+    for (int q = 0; q < P; ++q) {
+        // ---- broadcast of block q (comm stream)
+        {
+            ProfScope ps(m, PC_BCAST, m->ms);
+            if (m->comm) {
+                Rank& r = m->ranks[0];
+                const size_t count = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width;
+                if (q == r.rank) {
+                    float* s = job.src(m, r, job.ctx);
+                    if (!nob && count) NK(ncclBroadcast(s, s, count, ncclFloat32, q, m->comm, m->ms));
+                } else {
+                    const int k = remote_index(q, r.rank), slot = k & 1;
+                    if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (!nob && count) NK(ncclBroadcast(r.BC[slot], r.BC[slot], count, ncclFloat32, q, m->comm, m->ms));
+                    CK(cudaEventRecord(r.ev_bc[slot], m->ms));
+                }
+            } else {
+                Rank& root = m->ranks[q];
+                const size_t bytes = (size_t)root.rows * (size_t)job.width * sizeof(float);
+                for (auto& r : m->ranks) {
+                    if (r.rank == q) continue;
+                    const int k = remote_index(q, r.rank), slot = k & 1;
+                    if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (!nob && bytes)
+                        CK(cudaMemcpyAsync(r.BC[slot], job.src(m, root, job.ctx), bytes, cudaMemcpyDeviceToDevice,
+                                           m->ms));
+                    CK(cudaEventRecord(r.ev_bc[slot], m->ms));
+                }
+            }
+        }
+        // ---- SpMM stage q on every local receiver (compute stream)
+        for (auto& r : m->ranks) {
+            if (r.rank == q) continue;
+            const int k = remote_index(q, r.rank), slot = k & 1;
+            CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
+            const int last_q = (r.rank == P - 1) ? P - 2 : P - 1;
+            const int flags = SPMM_ACCUM | (q == last_q ? SPMM_LAST : 0);
+            if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], flags));
+            CK(cudaEventRecord(r.ev_free[slot], m->cs));
+        }
+    }
+    CK(cudaEventRecord(m->ev_comm_end, m->ms));
+    CK(cudaStreamWaitEvent(m->cs, m->ev_comm_end, 0));
+    return MGGCN_OK;
+}
+
+float* src_HWB(mggcn_model_s*, Rank& r, const void*) { return r.HWB; }
+float* src_X(mggcn_model_s*, Rank& r, const void*) { return r.Xs; }
+float* src_T0(mggcn_model_s*, Rank& r, const void*) { return r.T0; }
+float* src_AHWB(mggcn_model_s*, Rank& r, const void* ctx) { return r.AHWB[*static_cast<const int*>(ctx)]; }
+
+// Tiny reductions across ranks (loss, |T|) for nlocal == 1: NCCL all-reduce
+// on the comm stream fenced by events, or a copy when P == 1.
+int reduce_scalars(mggcn_model_s* m, bool ntrain) {
+    Rank& r = m->ranks[0];
+    if (m->comm) {
+        CK(cudaEventRecord(m->ev_tmp, m->cs));
+        CK(cudaStreamWaitEvent(m->ms, m->ev_tmp, 0));
+        if (ntrain) NK(ncclAllReduce(r.ntrain_local, m->ntrain, 1, ncclInt64, ncclSum, m->comm, m->ms));
+        else NK(ncclAllReduce(r.loss_local, m->loss_sum, 1, ncclFloat64, ncclSum, m->comm, m->ms));
+        CK(cudaEventRecord(m->ev_tmp, m->ms));
+        CK(cudaStreamWaitEvent(m->cs, m->ev_tmp, 0));
+    } else if (ntrain) {
+        CK(cudaMemcpyAsync(m->ntrain, r.ntrain_local, 8, cudaMemcpyDeviceToDevice, m->cs));
+    } else {
+        CK(cudaMemcpyAsync(m->loss_sum, r.loss_local, 8, cudaMemcpyDeviceToDevice, m->cs));
+    }
+    return MGGCN_OK;
+}
+
+}  // namespace
+
+// Loopback scalar reduction with an explicit ordered kernel over gathered values.
+static int reduce_scalars_loopback(mggcn_model_s* m, bool ntrain) {
+    // gather into a contiguous scratch (the first rank's ce_partial has room: kCeBlocks doubles)
+    const int R = (int)m->ranks.size();
+    double* scratch = m->ranks[0].ce_partial;   // free between loss passes (consumed already)
+    for (int i = 0; i < R; ++i) {
+        if (ntrain)
+            CK(cudaMemcpyAsync(reinterpret_cast<int64_t*>(scratch) + i, m->ranks[i].ntrain_local, 8,
+                               cudaMemcpyDeviceToDevice, m->cs));
+        else
+            CK(cudaMemcpyAsync(scratch + i, m->ranks[i].loss_local, 8, cudaMemcpyDeviceToDevice, m->cs));
+    }
+    if (ntrain) CK(launch_sum_i64(reinterpret_cast<int64_t*>(scratch), R, m->ntrain, m->cs));
+    else CK(launch_sum_f64(scratch, R, m->loss_sum, m->cs));
+    return MGGCN_OK;
+}
+
+static int reduce_all(mggcn_model_s* m, bool ntrain) {
+    if (m->nlocal > 1) return reduce_scalars_loopback(m, ntrain);
+    return reduce_scalars(m, ntrain);
+}
+
+static int poison(mggcn_model_s* m, int rc) {
+    if (rc == MGGCN_ECUDA || rc == MGGCN_ENCCL) m->poisoned = rc;
+    return rc;
+}
+
+#define MODEL_GUARD(m)                                              \
+    do {                                                            \
+        if (!(m)) {                                                 \
+            set_error("NULL model");                                \
+            return MGGCN_EINVAL;                                    \
+        }                                                           \
+        if ((m)->poisoned) {                                        \
+            set_error("model is poisoned by an earlier CUDA/NCCL error"); \
+            return (m)->poisoned;                                   \
+        }                                                           \
+    } while (0)
+
+// ------------------------------------------------------------- creation
+static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t nlocal, int32_t L,
+                             const int32_t* dims, uint32_t flags) {
+    if (!parts || nlocal < 1) {
+        set_error("model: parts / nlocal invalid");
+        return MGGCN_EINVAL;
+    }
+    RC(check_dims(L, dims));
+    const mggcn_part_s* p0 = parts[0];
+    if (!p0) {
+        set_error("model: NULL part");
+        return MGGCN_EINVAL;
+    }
+    m->P = p0->P;
+    m->nlocal = nlocal;
+    m->flags = flags;
+    m->L = L;
+    if (nlocal != 1 && nlocal != m->P) {
+        set_error("model: nlocal must be 1 or P (loopback)");
+        return MGGCN_EINVAL;
+    }
+    for (int i = 0; i < nlocal; ++i) {
+        const mggcn_part_s* pi = parts[i];
+        if (!pi || pi->P != m->P || pi->n != p0->n || pi->pattern != p0->pattern ||
+            (nlocal > 1 && pi->rank != i) || pi->perm != p0->perm) {
+            set_error("model: parts must come from the same graph / P / seed (and be ranks 0..P-1 in loopback)");
+            return MGGCN_EINVAL;
+        }
+    }
+    m->pattern = p0->pattern;
+    m->d.assign(dims, dims + L + 1);
+    m->ld.resize(L + 1);
+    for (int l = 0; l <= L; ++l) m->ld[l] = ld_of(m->d[l]);
+    m->order.resize(L);
+    for (int l = 0; l < L; ++l) m->order[l] = m->d[l] < m->d[l + 1] ? S_ORDER : G_ORDER;   // §4.4, reading C10
+    m->woff.resize(L);
+    m->wtotal = 0;
+    for (int l = 0; l < L; ++l) {
+        m->woff[l] = m->wtotal;
+        m->wtotal += round_up(m->d[l] * m->ld[l + 1], 64);
+    }
+    m->hw_ld = 4;
+    m->bc_ld = 4;
+    for (int l = 0; l < L; ++l) {
+        if (m->order[l] == G_ORDER) {
+            m->hw_ld = std::max(m->hw_ld, m->ld[l + 1]);
+            m->bc_ld = std::max(m->bc_ld, m->ld[l + 1]);
+        } else {
+            m->bc_ld = std::max(m->bc_ld, m->ld[l]);
+        }
+    }
+    m->max_rows_j = 0;
+    for (int j = 0; j < m->P; ++j) m->max_rows_j = std::max(m->max_rows_j, p0->p[j + 1] - p0->p[j]);
+    m->ranks.assign(nlocal, Rank());
+    int64_t off = 0;
+    for (int i = 0; i < nlocal; ++i) {
+        Rank& r = m->ranks[i];
+        r.part = parts[i];
+        r.rank = parts[i]->rank;
+        r.rows = parts[i]->nrows();
+        r.row_off = off;
+        off += r.rows;
+        r.hF.assign(m->P, HostItems());
+        r.hB.assign(m->P, HostItems());
+        for (int j = 0; j < m->P; ++j) {
+            build_items(r.part->F[j], r.hF[j]);
+            if (!r.part->shared_fb) build_items(r.part->B[j], r.hB[j]);
+        }
+    }
+    m->n_local = off;
+    // epoch work model, per this model's rows
+    auto spmm_work = [&](int dir, int64_t width) {
+        for (auto& r : m->ranks)
+            for (int j = 0; j < m->P; ++j) {
+                const HostTile& t = dir == 0 ? r.part->F[j] : r.part->tileB(j);
+                const double nnz = (double)t.rowptr.back();
+                m->w_spmm_bytes += nnz * (m->pattern ? 4.0 : 8.0) + 4.0 * (double)(t.nrows + 1) +
+                                   4.0 * (double)width * (double)(t.ncols + t.nrows);
+                m->w_gather_bytes += nnz * 4.0 * (double)width;
+                if (j != r.rank) m->w_bcast_bytes += 4.0 * (double)width * (double)t.ncols;
+            }
+    };
+    for (int l = 0; l < L; ++l) {
+        const int64_t w = m->order[l] == G_ORDER ? m->d[l + 1] : m->d[l];
+        spmm_work(0, w);
+        const double gf = 2.0 * (double)m->n_local * (double)m->d[l] * (double)m->d[l + 1];
+        m->w_gemm_flops += gf;                       // forward
+        m->w_gemm_flops += gf;                       // W_G
+        if (l > 0) m->w_gemm_flops += gf;            // H_G
+        if (m->order[l] == G_ORDER) spmm_work(1, m->d[l + 1]);   // backward SpMM (Eq. 9)
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_workspace_bytes(const mggcn_part* parts, int32_t nlocal, int32_t L, const int32_t* dims,
+                                     uint32_t flags, size_t* bytes) {
+    if (!bytes) {
+        set_error("workspace_bytes: NULL out");
+        return MGGCN_EINVAL;
+    }
+    mggcn_model_s tmp;
+    try {
+        RC(model_init_common(&tmp, parts, nlocal, L, dims, flags));
+    } catch (const std::bad_alloc&) {
+        set_error("workspace_bytes: out of host memory");
+        return MGGCN_ENOMEM;
+    }
+    Bump b;
+    plan_buffers(&tmp, b);
+    *bytes = b.off + 256;
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_nccl_unique_id(void* out128) {
+    if (!out128) {
+        set_error("nccl_unique_id: NULL out");
+        return MGGCN_EINVAL;
+    }
+    ncclUniqueId id;
+    NK(ncclGetUniqueId(&id));
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    std::memcpy(out128, &id, 128);
+    return MGGCN_OK;
+}
+
+static void destroy(mggcn_model_s* m) {
+    if (!m) return;
+    if (m->cs) cudaStreamSynchronize(m->cs);
+    if (m->ms) cudaStreamSynchronize(m->ms);
+    for (auto& r : m->ranks)
+        for (int s = 0; s < 2; ++s) {
+            if (r.ev_bc[s]) cudaEventDestroy(r.ev_bc[s]);
+            if (r.ev_free[s]) cudaEventDestroy(r.ev_free[s]);
+        }
+    for (cudaEvent_t e : {m->ev_begin, m->ev_comm_end, m->ev_tmp, m->ev_wg, m->ev_comm_done})
+        if (e) cudaEventDestroy(e);
+    for (auto& rec : m->prof_recs) {
+        cudaEventDestroy(std::get<1>(rec));
+        cudaEventDestroy(std::get<2>(rec));
+    }
+    for (auto e : m->prof_pool) cudaEventDestroy(e);
+    if (m->comm) ncclCommDestroy(m->comm);
+    delete m;
+}
+
+extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32_t L, const int32_t* dims,
+                                  uint32_t flags, const void* nccl_id128, void* workspace, size_t ws_bytes,
+                                  uintptr_t compute_stream, uintptr_t comm_stream, mggcn_model* out) {
+    if (!out) {
+        set_error("model_create: NULL out");
+        return MGGCN_EINVAL;
+    }
+    *out = nullptr;
+    mggcn_model_s* m = new (std::nothrow) mggcn_model_s();
+    if (!m) {
+        set_error("model_create: out of host memory");
+        return MGGCN_ENOMEM;
+    }
+    int rc;
+    try {
+        rc = model_init_common(m, parts, nlocal, L, dims, flags);
+    } catch (const std::bad_alloc&) {
+        rc = MGGCN_ENOMEM;
+        set_error("model_create: out of host memory");
+    }
+    if (rc != MGGCN_OK) {
+        delete m;
+        return rc;
+    }
+    if (m->P > 1 && nlocal == 1 && !nccl_id128) {
+        set_error("model_create: P > 1 with nlocal = 1 needs an NCCL unique id");
+        delete m;
+        return MGGCN_EINVAL;
+    }
+    Bump sz;
+    plan_buffers(m, sz);
+    if (!workspace || (reinterpret_cast<uintptr_t>(workspace) & 255) || ws_bytes < sz.off + 256) {
+        set_error("model_create: workspace NULL, misaligned (256 B) or smaller than mggcn_workspace_bytes");
+        delete m;
+        return MGGCN_EINVAL;
+    }
+    Bump b;
+    b.base = static_cast<char*>(workspace);
+    plan_buffers(m, b);
+    m->cs = reinterpret_cast<cudaStream_t>(compute_stream);
+    m->ms = reinterpret_cast<cudaStream_t>(comm_stream);
+    auto fail = [&](int code) {
+        destroy(m);
+        return code;
+    };
+    for (cudaEvent_t* e : {&m->ev_begin, &m->ev_comm_end, &m->ev_tmp, &m->ev_wg, &m->ev_comm_done})
+        if (cudaEventCreateWithFlags(e, cudaEventDisableTiming) != cudaSuccess) {
+            set_error("model_create: cudaEventCreate failed");
+            return fail(MGGCN_ECUDA);
+        }
+    for (auto& r : m->ranks)
+        for (int s = 0; s < 2; ++s)
+            if (cudaEventCreateWithFlags(&r.ev_bc[s], cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&r.ev_free[s], cudaEventDisableTiming) != cudaSuccess) {
+                set_error("model_create: cudaEventCreate failed");
+                return fail(MGGCN_ECUDA);
+            }
+    rc = upload_static(m);
+    if (rc != MGGCN_OK) return fail(rc);
+    rc = plan_gemms(m);
+    if (rc != MGGCN_OK) return fail(rc);
+    if (m->P > 1 && nlocal == 1) {
+        ncclUniqueId id;
+        std::memcpy(&id, nccl_id128, 128);
+        ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
+        const char* mc = getenv("MGGCN_NCCL_MAX_CTAS");
+        cfg.maxCTAs = mc ? atoi(mc) : 16;
+        ncclResult_t nr = ncclCommInitRankConfig(&m->comm, m->P, id, m->ranks[0].rank, &cfg);
+        if (nr != ncclSuccess) {
+            set_error(std::string("model_create: ncclCommInitRankConfig: ") + ncclGetErrorString(nr));
+            m->comm = nullptr;
+            return fail(MGGCN_ENCCL);
+        }
+    }
+    if (cudaStreamSynchronize(m->cs) != cudaSuccess) {
+        set_error(std::string("model_create: ") + cudaGetErrorString(cudaGetLastError()));
+        return fail(MGGCN_ECUDA);
+    }
+    *out = m;
+    return MGGCN_OK;
+}
+
+extern "C" void mggcn_model_free(mggcn_model m) { destroy(m); }
+
+// ---------------------------------------------------------------- weights
+static int check_layer(mggcn_model_s* m, int32_t layer) {
+    if (layer < 0 || layer >= m->L) {
+        set_error("layer out of range");
+        return MGGCN_EINVAL;
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_set_weights(mggcn_model m, int32_t layer, const float* W) {
+    MODEL_GUARD(m);
+    RC(check_layer(m, layer));
+    if (!W) {
+        set_error("set_weights: NULL W");
+        return MGGCN_EINVAL;
+    }
+    const int64_t din = m->d[layer], dout = m->d[layer + 1], ld = m->ld[layer + 1];
+    int rc = MGGCN_OK;
+    auto body = [&]() -> int {
+        CK(cudaMemcpy2DAsync(m->W + m->woff[layer], ld * 4, W, dout * 4, dout * 4, din, cudaMemcpyHostToDevice, m->cs));
+        CK(cudaMemsetAsync(m->Mom, 0, sizeof(float) * m->wtotal, m->cs));
+        CK(cudaMemsetAsync(m->Vel, 0, sizeof(float) * m->wtotal, m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    rc = body();
+    m->t = 0;
+    return poison(m, rc);
+}
+
+extern "C" int mggcn_get_weights(mggcn_model m, int32_t layer, float* W) {
+    MODEL_GUARD(m);
+    RC(check_layer(m, layer));
+    const int64_t din = m->d[layer], dout = m->d[layer + 1], ld = m->ld[layer + 1];
+    auto body = [&]() -> int {
+        CK(cudaMemcpy2DAsync(W, dout * 4, m->W + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost, m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    return poison(m, body());
+}
+
+static int wait_wg(mggcn_model_s* m) {
+    if (m->need_wg_wait) {
+        CK(cudaStreamWaitEvent(m->cs, m->ev_wg, 0));
+        m->need_wg_wait = false;
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_get_grad(mggcn_model m, int32_t layer, float* WG) {
+    MODEL_GUARD(m);
+    RC(check_layer(m, layer));
+    const int64_t din = m->d[layer], dout = m->d[layer + 1], ld = m->ld[layer + 1];
+    auto body = [&]() -> int {
+        RC(wait_wg(m));
+        CK(cudaMemcpy2DAsync(WG, dout * 4, m->WG + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost, m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    return poison(m, body());
+}
+
+extern "C" int mggcn_get_adam(mggcn_model m, int32_t layer, float* mom, float* vel, int64_t* t) {
+    MODEL_GUARD(m);
+    RC(check_layer(m, layer));
+    const int64_t din = m->d[layer], dout = m->d[layer + 1], ld = m->ld[layer + 1];
+    auto body = [&]() -> int {
+        if (mom)
+            CK(cudaMemcpy2DAsync(mom, dout * 4, m->Mom + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost,
+                                 m->cs));
+        if (vel)
+            CK(cudaMemcpy2DAsync(vel, dout * 4, m->Vel + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost,
+                                 m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    if (t) *t = m->t;
+    return poison(m, body());
+}
+
+extern "C" int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, const float* vel, int64_t t) {
+    MODEL_GUARD(m);
+    RC(check_layer(m, layer));
+    if (!mom || !vel || t < 0) {
+        set_error("set_adam: NULL moments or t < 0");
+        return MGGCN_EINVAL;
+    }
+    const int64_t din = m->d[layer], dout = m->d[layer + 1], ld = m->ld[layer + 1];
+    auto body = [&]() -> int {
+        CK(cudaMemcpy2DAsync(m->Mom + m->woff[layer], ld * 4, mom, dout * 4, dout * 4, din, cudaMemcpyHostToDevice,
+                             m->cs));
+        CK(cudaMemcpy2DAsync(m->Vel + m->woff[layer], ld * 4, vel, dout * 4, dout * 4, din, cudaMemcpyHostToDevice,
+                             m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    m->t = t;
+    return poison(m, body());
+}
+
+// ---------------------------------------------------------------- forward
+static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int32_t* y, float* loss,
+                        float* logits) {
+    const int L = m->L;
+    // inputs -> internal buffers (host or device source; this is the e2e H2D when host)
+    for (auto& r : m->ranks) {
+        if (r.rows == 0) continue;
+        ProfScope ps(m, PC_OTHER, m->cs);
+        CK(cudaMemcpy2DAsync(r.Xs, m->ld[0] * 4, X + r.row_off * ldx, ldx * 4, m->d[0] * 4, r.rows,
+                             cudaMemcpyDefault, m->cs));
+        CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
+    }
+    for (int l = 0; l < L; ++l) {
+        const bool relu_here = (l < L - 1) || (m->flags & MGGCN_F_RELU_LAST);
+        int* layer_ids = m->layer_ids;
+        layer_ids[l] = l;
+        if (m->order[l] == G_ORDER) {
+            for (auto& r : m->ranks)
+                if (r.has_fwd[l]) {
+                    ProfScope ps(m, PC_GEMM, m->cs);
+                    CK(gemm_launch(r.g_fwd[l], m->cs));                                  // Eq. 5 -> HWB (Eq. 16)
+                }
+            SpmmJob job{0, m->ld[l + 1], m->pattern, relu_here, src_HWB,
+                        [](mggcn_model_s*, Rank& r, const void* c) { return r.AHWB[*static_cast<const int*>(c)]; },
+                        &layer_ids[l]};
+            RC(staged_spmm(m, job));                                                     // Eq. 6-7 -> AHWB (Eq. 17-18)
+        } else {
+            SpmmJob job{0, m->ld[0], m->pattern, false, src_X,
+                        [](mggcn_model_s*, Rank& r, const void*) { return r.T0; }, nullptr};
+            RC(staged_spmm(m, job));                                                     // T = Â'^T X (§4.4)
+            for (auto& r : m->ranks)
+                if (r.has_fwd[l]) {
+                    ProfScope ps(m, PC_GEMM, m->cs);
+                    CK(gemm_launch(r.g_fwd[l], m->cs));                                  // T W (+ReLU) -> AHWB_0
+                }
+        }
+    }
+    // ---- loss: |T|, logits out, fused CE fwd+bwd in place (Eq. 19)
+    for (auto& r : m->ranks) CK(launch_count_labelled(r.y, r.rows, r.ntrain_local, m->cs));
+    RC(reduce_all(m, true));
+    if (logits) {
+        for (auto& r : m->ranks)
+            if (r.rows)
+                CK(cudaMemcpy2DAsync(logits + r.row_off * m->d[L], m->d[L] * 4, r.AHWB[L - 1], m->ld[L] * 4,
+                                     m->d[L] * 4, r.rows, cudaMemcpyDeviceToDevice, m->cs));
+    }
+    const bool prescale = m->order[L - 1] == G_ORDER && m->pattern;
+    for (auto& r : m->ranks) {
+        ProfScope ps(m, PC_LOSS, m->cs);
+        CK(launch_softmax_ce(r.AHWB[L - 1], r.rows, (int)m->d[L], m->ld[L], r.y, m->ntrain,
+                             prescale ? r.inv_deg : nullptr, (m->flags & MGGCN_F_RELU_LAST) ? 1 : 0, r.ce_partial,
+                             m->cs));
+        CK(launch_sum_partials(r.ce_partial, kCeBlocks, r.loss_local, m->cs));
+    }
+    RC(reduce_all(m, false));
+    if (loss) {
+        double s = 0;
+        int64_t nt = 0;
+        CK(cudaMemcpyAsync(&s, m->loss_sum, 8, cudaMemcpyDeviceToHost, m->cs));
+        CK(cudaMemcpyAsync(&nt, m->ntrain, 8, cudaMemcpyDeviceToHost, m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        *loss = (float)(s / (double)(nt > 0 ? nt : 1));
+        if (m->comm) {
+            ncclResult_t ae;
+            if (ncclCommGetAsyncError(m->comm, &ae) == ncclSuccess && ae != ncclSuccess) {
+                set_error(std::string("NCCL async error: ") + ncclGetErrorString(ae));
+                return MGGCN_ENCCL;
+            }
+        }
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float* loss,
+                             float* logits_local) {
+    MODEL_GUARD(m);
+    if (!X_local || !y_local || ldx < m->d[0]) {
+        set_error("forward: NULL X/y or ldx < d_0");
+        return MGGCN_EINVAL;
+    }
+    RC(poison(m, wait_wg(m)));
+    int rc = forward_impl(m, X_local, ldx, y_local, loss, logits_local);
+    if (rc == MGGCN_OK) m->state = ST_FWD;
+    return poison(m, rc);
+}
+
+extern "C" int mggcn_get_loss(mggcn_model m, float* loss) {
+    MODEL_GUARD(m);
+    if (!loss) {
+        set_error("get_loss: NULL out");
+        return MGGCN_EINVAL;
+    }
+    double s = 0;
+    int64_t nt = 0;
+    auto body = [&]() -> int {
+        CK(cudaMemcpyAsync(&s, m->loss_sum, 8, cudaMemcpyDeviceToHost, m->cs));
+        CK(cudaMemcpyAsync(&nt, m->ntrain, 8, cudaMemcpyDeviceToHost, m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    int rc = body();
+    *loss = (float)(s / (double)(nt > 0 ? nt : 1));
+    return poison(m, rc);
+}
+
+// --------------------------------------------------------------- backward
+static int wgrad_reduce(mggcn_model_s* m, int l) {
+    // per-rank partial W_G (Eq. 10) -> sum over ranks (reading C23)
+    const int64_t din = m->d[l], dout = m->d[l + 1], ld = m->ld[l + 1];
+    for (auto& r : m->ranks) {
+        float* dst = (m->nlocal > 1 ? r.WG_local : m->WG) + m->woff[l];
+        if (r.has_wgrad[l]) {
+            {
+                ProfScope ps(m, PC_GEMM, m->cs);
+                CK(gemm_launch(r.g_wgrad[l], m->cs));
+            }
+            CK(launch_splitk_reduce(r.gemm_partial, r.g_wgrad[l].k_chunks, din, dout, dst, ld, m->cs));
+        } else {
+            CK(cudaMemsetAsync(dst, 0, sizeof(float) * din * ld, m->cs));
+        }
+    }
+    if (m->nlocal > 1) {
+        std::vector<const float*> in;
+        for (auto& r : m->ranks) in.push_back(r.WG_local + m->woff[l]);
+        ProfScope ps(m, PC_ALLRED, m->cs);
+        CK(launch_sum_buffers(in.data(), (int)in.size(), m->WG + m->woff[l], din * ld, m->cs));
+    } else if (m->comm) {
+        CK(cudaEventRecord(m->ev_tmp, m->cs));
+        CK(cudaStreamWaitEvent(m->ms, m->ev_tmp, 0));
+        {
+            ProfScope ps(m, PC_ALLRED, m->ms);
+            NK(ncclAllReduce(m->WG + m->woff[l], m->WG + m->woff[l], (size_t)(din * ld), ncclFloat32, ncclSum, m->comm,
+                             m->ms));
+        }
+        CK(cudaEventRecord(m->ev_wg, m->ms));
+        m->need_wg_wait = true;
+    }
+    return MGGCN_OK;
+}
+
+static int backward_impl(mggcn_model_s* m) {
+    const int L = m->L;
+    int* layer_ids = m->layer_ids;
+    for (int l = L - 1; l >= 0; --l) {
+        layer_ids[l] = l;
+        if (m->order[l] == G_ORDER) {
+            // Eq. 9: HW_G = Â' · AHW_G (AHWB_l, pre-scaled by inv_deg when pattern-only) -> HWB (Eq. 20)
+            SpmmJob job{1, m->ld[l + 1], false, false, src_AHWB,
+                        [](mggcn_model_s*, Rank& r, const void*) { return r.HWB; }, &layer_ids[l]};
+            RC(staged_spmm(m, job));
+            RC(wgrad_reduce(m, l));                                           // Eq. 10
+            if (l > 0)
+                for (auto& r : m->ranks)
+                    if (r.has_igrad[l]) {
+                        ProfScope ps(m, PC_GEMM, m->cs);
+                        CK(gemm_launch(r.g_igrad[l], m->cs));                 // Eq. 11 + Eq. 8 mask -> AHWB_{l-1}
+                    }
+        } else {
+            // S-order (l == 0 only): W_G = T^T Z_G; no input-feature gradient (§4.4 skip, reading C11)
+            RC(wgrad_reduce(m, l));
+        }
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_backward(mggcn_model m) {
+    MODEL_GUARD(m);
+    if (m->state != ST_FWD) {
+        set_error("backward: needs a preceding forward");
+        return MGGCN_ESTATE;
+    }
+    int rc = backward_impl(m);
+    if (rc == MGGCN_OK) m->state = ST_BWD;
+    return poison(m, rc);
+}
+
+extern "C" int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps) {
+    MODEL_GUARD(m);
+    if (m->state != ST_BWD) {
+        set_error("step: needs a preceding backward");
+        return MGGCN_ESTATE;
+    }
+    if (!(lr > 0) || !(beta1 >= 0 && beta1 < 1) || !(beta2 >= 0 && beta2 < 1) || !(eps > 0)) {
+        set_error("step: bad hyper-parameters");
+        return MGGCN_EINVAL;
+    }
+    auto body = [&]() -> int {
+        RC(wait_wg(m));
+        m->t += 1;
+        ProfScope ps(m, PC_ADAM, m->cs);
+        CK(launch_adam(m->W, m->WG, m->Mom, m->Vel, m->wtotal, lr, beta1, beta2, eps, m->t, m->cs));
+        return MGGCN_OK;
+    };
+    int rc = body();
+    if (rc == MGGCN_OK) m->state = ST_READY;
+    return poison(m, rc);
+}
+
+// -------------------------------------------------------------- profiling
+extern "C" int mggcn_get_profile(mggcn_model m, double* ms, int64_t* launches, int32_t reset) {
+    MODEL_GUARD(m);
+    if (cudaStreamSynchronize(m->cs) != cudaSuccess || cudaStreamSynchronize(m->ms) != cudaSuccess) {
+        set_error("get_profile: stream sync failed");
+        return poison(m, MGGCN_ECUDA);
+    }
+    for (auto& rec : m->prof_recs) {
+        float t = 0;
+        cudaEventElapsedTime(&t, std::get<1>(rec), std::get<2>(rec));
+        m->prof_ms[std::get<0>(rec)] += t;
+        m->prof_n[std::get<0>(rec)] += 1;
+        m->prof_pool.push_back(std::get<1>(rec));
+        m->prof_pool.push_back(std::get<2>(rec));
+    }
+    m->prof_recs.clear();
+    for (int c = 0; c < PC_N; ++c) {
+        if (ms) ms[c] = m->prof_ms[c];
+        if (launches) launches[c] = m->prof_n[c];
+        if (reset) {
+            m->prof_ms[c] = 0;
+            m->prof_n[c] = 0;
+        }
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* gather, double* flops, double* bcast) {
+    if (!m) {
+        set_error("NULL model");
+        return MGGCN_EINVAL;
+    }
+    if (spmm_bytes) *spmm_bytes = m->w_spmm_bytes;
+    if (gather) *gather = m->w_gather_bytes;
+    if (flops) *flops = m->w_gemm_flops;
+    if (bcast) *bcast = m->w_bcast_bytes;
+    return MGGCN_OK;
+}
+
+// ------------------------------------------------------------- test hooks
+extern "C" int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int64_t ldb, int32_t width, float* out,
+                                int64_t ldo) {
+    MODEL_GUARD(m);
+    if ((dir != 0 && dir != 1) || !B || !out || width <= 0 || (ldb & 3) || (ldo & 3) || ldb < width || ldo < width) {
+        set_error("debug_spmm: bad arguments");
+        return MGGCN_EINVAL;
+    }
+    if (m->P > 1 && m->nlocal == 1) {
+        set_error("debug_spmm: needs P == 1 or loopback mode");
+        return MGGCN_EUNSUPPORTED;
+    }
+    const int64_t w = round_up(width, 4);
+    if (w > m->bc_ld && m->P > 1) {
+        set_error("debug_spmm: width exceeds the model's broadcast buffers");
+        return MGGCN_EINVAL;
+    }
+    // staging: per rank a contiguous (rows x w) input (pre-scaled by inv_deg for the
+    // pattern-only backward) and output, carved from one cudaMalloc
+    size_t tot = 0;
+    for (auto& r : m->ranks) tot += 2 * (size_t)r.rows * w;
+    float* scratch = nullptr;
+    auto body = [&]() -> int {
+        CK(cudaMalloc(&scratch, sizeof(float) * (tot + 64)));
+        CK(cudaMemsetAsync(scratch, 0, sizeof(float) * (tot + 64), m->cs));
+        struct Ctx {
+            std::vector<float*> in, out;
+        } ctx;
+        size_t off = 0;
+        for (auto& r : m->ranks) {
+            ctx.in.push_back(scratch + off);
+            off += (size_t)r.rows * w;
+            ctx.out.push_back(scratch + off);
+            off += (size_t)r.rows * w;
+            const bool pre = dir == 1 && m->pattern;
+            if (r.rows)
+                CK(launch_scale_rows(B + r.row_off * ldb, ldb, ctx.in.back(), w, r.rows, width,
+                                     pre ? r.inv_deg : nullptr, m->cs));
+        }
+        SpmmJob job{dir, w, dir == 0 && m->pattern, false,
+                    [](mggcn_model_s* mm, Rank& r, const void* c) {
+                        return static_cast<const Ctx*>(c)->in[&r - mm->ranks.data()];
+                    },
+                    [](mggcn_model_s* mm, Rank& r, const void* c) {
+                        return static_cast<const Ctx*>(c)->out[&r - mm->ranks.data()];
+                    },
+                    &ctx};
+        RC(staged_spmm(m, job));
+        for (size_t i = 0; i < m->ranks.size(); ++i) {
+            Rank& r = m->ranks[i];
+            if (r.rows)
+                CK(cudaMemcpy2DAsync(out + r.row_off * ldo, ldo * 4, ctx.out[i], w * 4, width * 4, r.rows,
+                                     cudaMemcpyDeviceToDevice, m->cs));
+        }
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    int rc = body();
+    if (scratch) cudaFree(scratch);
+    return poison(m, rc);
+}
+
+extern "C" int mggcn_debug_gemm(int32_t op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda,
+                                const float* B, int64_t ldb, float* C, int64_t ldc, uint32_t flags, uintptr_t stream) {
+    if (op < 0 || op > 2 || !A || !B || !C || ldc < N) {
+        set_error("debug_gemm: bad arguments");
+        return MGGCN_EINVAL;
+    }
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    GemmPlan g;
+    size_t pf = 0;
+    const int gf = (flags & MGGCN_F_TF32X1) ? GEMM_TF32X1 : 0;
+    if (gemm_plan(g, op, M, N, K, A, lda, B, ldb, C, ldc, gf, &pf)) {
+        set_error("debug_gemm: plan failed (alignment: pointers 16 B, lda/ldb multiple of 4; needs sm_100)");
+        return MGGCN_EINVAL;
+    }
+    float* part = nullptr;
+    auto body = [&]() -> int {
+        if (op == 2) {
+            CK(cudaMalloc(&part, sizeof(float) * (pf + 4)));
+            g.partial = part;
+        }
+        CK(gemm_launch(g, s));
+        if (op == 2) CK(launch_splitk_reduce(part, g.k_chunks, M, N, C, ldc, s));
+        CK(cudaStreamSynchronize(s));
+        return MGGCN_OK;
+    };
+    int rc = body();
+    if (part) cudaFree(part);
+    return rc;
+}

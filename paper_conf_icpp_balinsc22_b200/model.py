@@ -1,0 +1,119 @@
+"""GCN: convenience wrapper over the C ABI (marshalling only).
+
+Owns one graph -> partition(s) -> model chain, the torch workspace tensor and
+the two CUDA streams (compute = stream 0, comm = stream 1 of P:929-933).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import (MGGCN_F_OVERLAP, mggcn_backward, mggcn_epoch_work, mggcn_forward, mggcn_get_adam, mggcn_get_grad,
+               mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free, mggcn_load_csr,
+               mggcn_model_create, mggcn_model_free, mggcn_part_free, mggcn_part_info, mggcn_partition,
+               mggcn_set_adam, mggcn_set_weights, mggcn_step, mggcn_workspace_bytes)
+
+
+class GCN:
+    """Full-batch GCN (Eq. 1-11) on one GPU rank, or all P ranks in loopback mode.
+
+    rowptr/col/vals: CSR of A in ORIGINAL vertex ids.  dims = (d_0, ..., d_L).
+    """
+
+    def __init__(self, n, rowptr, col, vals, dims, P=1, rank=0, perm_seed=0, flags=MGGCN_F_OVERLAP,
+                 loopback=False, nccl_id=None, device=None, graph=None):
+        import torch
+        self.torch = torch
+        self.dims = tuple(int(d) for d in dims)
+        self.L = len(self.dims) - 1
+        self.P, self.rank, self.loopback = P, rank, loopback
+        own_graph = graph is None
+        g = mggcn_load_csr(n, rowptr, col, vals) if own_graph else graph
+        try:
+            ranks = list(range(P)) if loopback else [rank]
+            self.parts = [mggcn_partition(g, P, r, perm_seed) for r in ranks]
+        finally:
+            if own_graph:
+                mggcn_graph_free(g)
+        info = mggcn_part_info(self.parts[0])
+        self.n, self.p, self.perm = info["n"], info["p"], info["perm"]
+        self.row0 = 0 if loopback else int(self.p[rank])
+        self.rows = n if loopback else int(self.p[rank + 1] - self.p[rank])
+        self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        self.ws_bytes = mggcn_workspace_bytes(self.parts, self.dims, flags)
+        self.workspace = torch.empty(self.ws_bytes, dtype=torch.uint8, device=self.device)
+        self.cs = torch.cuda.Stream(device=self.device)
+        self.ms = torch.cuda.Stream(device=self.device)
+        self.m = mggcn_model_create(self.parts, self.dims, flags, nccl_id, self.workspace.data_ptr(), self.ws_bytes,
+                                    self.cs.cuda_stream, self.ms.cuda_stream)
+
+    # ---------------------------------------------------------------- data
+    def permute_rows(self, X):
+        """Rows owned by this model of the permuted matrix X' (X'[perm[v]] = X[v])."""
+        X = np.asarray(X)
+        Xp = np.empty_like(X)
+        Xp[self.perm] = X
+        return np.ascontiguousarray(Xp[self.row0:self.row0 + self.rows])
+
+    def set_weights(self, Ws):
+        for l, W in enumerate(Ws):
+            mggcn_set_weights(self.m, l, W)
+
+    def get_weights(self):
+        return [mggcn_get_weights(self.m, l, (self.dims[l], self.dims[l + 1])) for l in range(self.L)]
+
+    # ---------------------------------------------------------- hot path
+    def forward(self, X_local, y_local, want_loss=True, logits=None):
+        """X_local / y_local: numpy (host) or torch (device or pinned host) rows of X', y'."""
+        torch = self.torch
+        if isinstance(X_local, torch.Tensor) and X_local.is_cuda:
+            self.cs.wait_stream(torch.cuda.current_stream(self.device))
+        ldx = X_local.shape[1] if X_local.ndim == 2 else self.dims[0]
+        if isinstance(X_local, np.ndarray):
+            X_local = np.ascontiguousarray(X_local, dtype=np.float32)
+            y_local = np.ascontiguousarray(y_local, dtype=np.int32)
+        loss = mggcn_forward(self.m, X_local, ldx, y_local, want_loss, logits)
+        if logits is not None:
+            torch.cuda.current_stream(self.device).wait_stream(self.cs)
+        return loss
+
+    def backward(self):
+        mggcn_backward(self.m)
+
+    def step(self, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8):
+        mggcn_step(self.m, lr, beta1, beta2, eps)
+
+    def loss(self):
+        return mggcn_get_loss(self.m)
+
+    def grads(self):
+        return [mggcn_get_grad(self.m, l, (self.dims[l], self.dims[l + 1])) for l in range(self.L)]
+
+    def adam_state(self, layer):
+        return mggcn_get_adam(self.m, layer, (self.dims[layer], self.dims[layer + 1]))
+
+    def set_adam_state(self, layer, mom, vel, t):
+        mggcn_set_adam(self.m, layer, mom, vel, t)
+
+    def profile(self, reset=False):
+        return mggcn_get_profile(self.m, reset)
+
+    def epoch_work(self):
+        return mggcn_epoch_work(self.m)
+
+    def synchronize(self):
+        self.cs.synchronize()
+        self.ms.synchronize()
+
+    def close(self):
+        if getattr(self, "m", None) is not None:
+            mggcn_model_free(self.m)
+            self.m = None
+        for p in getattr(self, "parts", []):
+            mggcn_part_free(p)
+        self.parts = []
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,204 @@
+"""Whole-epoch GPU parity through the C ABI against the CPU oracle:
+logits, loss, every W_G, Adam m / v and W after one step (SURVEY.md §8(c)
+"GPU-vs-oracle acceptance"; tolerance from BASELINE.json north_star).
+Loopback mode runs the P-stage broadcast pipeline with P ranks on one GPU."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from helpers import random_directed
+
+pytestmark = pytest.mark.gpu
+
+REL_TOL = 1e-3
+
+
+def rel(x, r):
+    return float(np.abs(np.asarray(x, np.float64) - r).max() / max(np.abs(r).max(), 1e-30))
+
+
+@pytest.fixture(scope="module")
+def mg():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_icpp_balinsc22_b200 as mg
+    return mg
+
+
+def run_library(mg, n, rp, col, vals, X, y, Ws, dims, P, seed, flags, host_inputs=False, steps=1, lr=0.01):
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    gm = GCN(n, rp, col, vals, dims, P=P, perm_seed=seed, flags=flags, loopback=P > 1)
+    gm.set_weights(Ws)
+    Xl = gm.permute_rows(X)
+    yl = gm.permute_rows(y)
+    if host_inputs:
+        Xin, yin = Xl, yl
+    else:
+        Xin, yin = torch.from_numpy(Xl).cuda(), torch.from_numpy(yl).cuda()
+    logits = torch.empty((n, dims[-1]), dtype=torch.float32, device="cuda")
+    out = {}
+    for s in range(steps):
+        out["loss"] = gm.forward(Xin, yin, want_loss=True, logits=logits if s == 0 else None)
+        if s == 0:
+            out["logits"] = logits.cpu().numpy()
+        gm.backward()
+        if s == 0:
+            out["WG"] = gm.grads()
+        gm.step(lr=lr)
+    out["W"] = gm.get_weights()
+    out["adam"] = [gm.adam_state(l) for l in range(len(Ws))]
+    out["perm"] = gm.perm
+    gm.close()
+    return out
+
+
+def compare(lib, ref, dims, tol=REL_TOL):
+    assert np.array_equal(lib["perm"], ref.perm)
+    assert rel(lib["logits"], ref.logits) < tol, rel(lib["logits"], ref.logits)
+    assert abs(lib["loss"] - ref.loss) / abs(ref.loss) < tol, (lib["loss"], ref.loss)
+    for l, (a, b) in enumerate(zip(lib["WG"], ref.WG)):
+        assert rel(a, b) < tol, (l, rel(a, b))
+    for l in range(len(dims) - 1):
+        mo, ve, t = lib["adam"][l]
+        assert t == 1
+        assert rel(mo, ref.m[l]) < tol and rel(ve, ref.v[l]) < 2 * tol
+        # W only where |g| is not tiny (first Adam step ~ lr * sign(g))
+        g = ref.WG[l]
+        mask = np.abs(g) > 1e-3 * np.abs(g).max()
+        np.testing.assert_allclose(lib["W"][l][mask], ref.W[l][mask], rtol=0, atol=1e-5)
+
+
+def workload_inputs(w, unlabelled=0):
+    rp, col = gen.rmat_csr(w.n, w.m, w.seed_G)
+    X = gen.features(w.n, w.dims[0], w.seed_X)
+    y = gen.labels(w.n, w.dims[-1], w.seed_y, unlabelled)
+    Ws = [gen.glorot(w.dims[l], w.dims[l + 1], w.seed_W + l) for l in range(len(w.dims) - 1)]
+    return rp, col, X, y, Ws
+
+
+@pytest.mark.parametrize("P", [1, 2, 4])
+def test_cora_shaped_epoch(mg, P):
+    """BASELINE configs[0]: Cora-shaped, 2 layers 1433 -> 16 -> 7."""
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    pg = oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed)
+    ref = oracle.epoch(pg, X, y, Ws)
+    lib = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, P, w.perm_seed, mg.MGGCN_F_OVERLAP)
+    compare(lib, ref, w.dims)
+
+
+def test_cora_shaped_unlabelled_host_inputs(mg):
+    """10 % unlabelled vertices, inputs given as HOST pointers (the e2e path)."""
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w, unlabelled=100)
+    assert (y < 0).sum() > 100
+    pg = oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed)
+    ref = oracle.epoch(pg, X, y, Ws)
+    lib = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 1, w.perm_seed, mg.MGGCN_F_OVERLAP,
+                      host_inputs=True)
+    compare(lib, ref, w.dims)
+
+
+@pytest.mark.parametrize("P", [1, 3])
+@pytest.mark.parametrize("dims", [(8, 32, 32, 5), (100, 256, 256, 47), (24, 16, 12)])
+def test_small_rmat_epoch(mg, P, dims):
+    """SpMM-first layer 0 (d0 < d1, §4.4) and GeMM-first layers; ragged widths."""
+    n, m = 3001, 60000
+    rp, col = gen.rmat_csr(n, m, 71)
+    X = gen.features(n, dims[0], 72)
+    y = gen.labels(n, dims[-1], 73)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 74 + l) for l in range(len(dims) - 1)]
+    pg = oracle.permute_graph(n, rp, col, None, seed=75)
+    ref = oracle.epoch(pg, X, y, Ws)
+    lib = run_library(mg, n, rp, col, None, X, y, Ws, dims, P, 75, mg.MGGCN_F_OVERLAP)
+    compare(lib, ref, dims)
+
+
+@pytest.mark.parametrize("P", [1, 2])
+def test_weighted_directed_epoch(mg, P):
+    n = 1500
+    rp, col, vals = random_directed(n, 20000, 8, weighted=True)
+    dims = (20, 16, 6)
+    X = gen.features(n, dims[0], 81)
+    y = gen.labels(n, dims[-1], 82)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 83 + l) for l in range(2)]
+    pg = oracle.permute_graph(n, rp, col, vals, seed=84)
+    ref = oracle.epoch(pg, X, y, Ws)
+    lib = run_library(mg, n, rp, col, vals, X, y, Ws, dims, P, 84, mg.MGGCN_F_OVERLAP)
+    compare(lib, ref, dims)
+
+
+def test_relu_last_and_no_overlap(mg):
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    pg = oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed)
+    ref = oracle.epoch(pg, X, y, Ws, relu_last=True)
+    lib = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 2, w.perm_seed, mg.MGGCN_F_RELU_LAST)
+    compare(lib, ref, w.dims)
+
+
+def test_bitwise_determinism_and_pipeline_invariance(mg):
+    """Same inputs twice -> bitwise identical; P-way loopback with and without
+    overlap -> bitwise identical (same stage order, only the schedule differs)."""
+    n, m = 2000, 40000
+    rp, col = gen.rmat_csr(n, m, 91)
+    dims = (32, 64, 10)
+    X = gen.features(n, dims[0], 92)
+    y = gen.labels(n, dims[-1], 93)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 94 + l) for l in range(2)]
+    a = run_library(mg, n, rp, col, None, X, y, Ws, dims, 3, 95, mg.MGGCN_F_OVERLAP)
+    b = run_library(mg, n, rp, col, None, X, y, Ws, dims, 3, 95, mg.MGGCN_F_OVERLAP)
+    c = run_library(mg, n, rp, col, None, X, y, Ws, dims, 3, 95, 0)
+    for other in (b, c):
+        assert np.array_equal(a["logits"], other["logits"])
+        assert a["loss"] == other["loss"]
+        for x, z in zip(a["WG"], other["WG"]):
+            assert np.array_equal(x, z)
+
+
+def test_multi_step_training_decreases_loss(mg):
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    gm = GCN(w.n, rp, col, None, w.dims, perm_seed=w.perm_seed)
+    gm.set_weights(Ws)
+    Xd = torch.from_numpy(gm.permute_rows(X)).cuda()
+    yd = torch.from_numpy(gm.permute_rows(y)).cuda()
+    losses = []
+    for _ in range(20):
+        losses.append(gm.forward(Xd, yd))
+        gm.backward()
+        gm.step(lr=0.01)
+    assert losses[-1] < losses[0]
+    # oracle 3 steps agree
+    pg = oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed)
+    Wc = [W.copy() for W in Ws]
+    st = None
+    gm2 = GCN(w.n, rp, col, None, w.dims, perm_seed=w.perm_seed)
+    gm2.set_weights(Ws)
+    for t in range(1, 4):
+        r = oracle.epoch(pg, X, y, Wc, adam_state=st, t=t)
+        lo = gm2.forward(Xd, yd)
+        assert abs(lo - r.loss) / r.loss < REL_TOL
+        gm2.backward()
+        gm2.step()
+        Wc, st = r.W, (r.m, r.v)
+    gm.close()
+    gm2.close()
+
+
+def test_state_errors(mg):
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    rp, col = gen.rmat_csr(200, 2000, 1)
+    gm = GCN(200, rp, col, None, (8, 4))
+    with pytest.raises(mg.MggcnError) as e:
+        gm.backward()
+    assert e.value.code == mg.MGGCN_ESTATE
+    with pytest.raises(mg.MggcnError) as e:
+        gm.step()
+    assert e.value.code == mg.MGGCN_ESTATE
+    gm.close()
+    with pytest.raises(mg.MggcnError) as e:
+        GCN(200, rp, col, None, (8, 4, 16, 2))      # SpMM-first at l = 1
+    assert e.value.code == mg.MGGCN_EUNSUPPORTED

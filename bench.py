@@ -1,0 +1,370 @@
+"""Benchmark: full-batch GCN epoch time on B200 (BASELINE.json metric
+"full-batch GCN epoch ms at 1/2/4/8 B200; SpMM HBM GB/s vs peak").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload reddit] [--impl mggcn|reference]
+
+A step is one full epoch of the hot path (forward over all layers with the
+P-stage SpMM, softmax-CE, backward, W_G all-reduce, Adam) on synthetic
+R-MAT inputs shaped like BASELINE.json's config (default configs[1],
+Reddit-shaped, which fits one GPU).  Rank 0 prints ONE JSON line.
+
+For N > 1 launch with torchrun (one rank per GPU, NCCL over NVLink); the
+library creates its own NCCL communicator from a unique id shared through
+torch.distributed.  --impl reference times the CPU oracle (the tier's
+reference arm) on a bounded row sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402
+
+METRIC = "full-batch GCN epoch ms"
+UNIT = "ms"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=int(os.environ.get("WORLD_SIZE", "1")))
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--workload", default="reddit", choices=sorted(gen.WORKLOADS))
+    ap.add_argument("--impl", default="mggcn", choices=["mggcn", "reference"])
+    ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--tf32x1", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--oracle-rows", type=int, default=0, help="row sample of the oracle leg (0 = auto)")
+    return ap.parse_args()
+
+
+def workload_desc(w, P):
+    return {"workload": f"{w.name}-shaped R-MAT (Graph500 a,b,c,d = .57,.19,.19,.05; symmetric, duplicates kept)",
+            "n": w.n, "nnz": w.m, "dims": list(w.dims), "layers": len(w.dims) - 1, "P": P,
+            "perm_seed": w.perm_seed, "graph_seed": w.seed_G, "partition": "1D row, P-stage broadcast (BC1/BC2)",
+            "l2": "no flush: every epoch streams inputs larger than L2 (features, CSR, activations)"}
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.f = tempfile.NamedTemporaryFile(mode="w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f,
+                                      stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as fh:
+            for line in fh:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) >= 9:
+                    rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"], "samples": 0}
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows),
+                "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit())
+                if any(r[3].replace(".", "").isdigit() for r in rows) else None}
+
+
+# ------------------------------------------------------- oracle (CPU) leg
+_ORACLE_CACHE = {}
+
+
+def oracle_epoch_sample(w, rp, col, rows_per_step, seed=0):
+    """Time the CPU oracle's ops for ONE epoch of workload `w` restricted to a
+    random sample of `rows_per_step` output rows (every SpMM, GEMM and the CE
+    of the epoch, in the paper's order, Eq. 5-11); returns (estimated
+    full-epoch ms, wall seconds, R).  Row-proportional work is scaled by n/R;
+    Adam runs on the full weights."""
+    import oracle
+    n, L, dims = w.n, len(w.dims) - 1, w.dims
+    R = min(rows_per_step, n)
+    rows = np.sort(np.random.default_rng(seed).choice(n, R, replace=False))
+    key = (w.name, id(rp))
+    if key not in _ORACLE_CACHE:
+        # a symmetric graph: rows of Â^T have the pattern of A's rows (values 1/deg)
+        _, ahat = oracle.normalise(n, rp, col)
+        csr = oracle.CSR(np.asarray(rp, np.int64), np.asarray(col, np.int64), ahat)
+        B = gen.features(n, max(dims), 12345)      # dense operand rows (values irrelevant for timing)
+        _ORACLE_CACHE.clear()
+        _ORACLE_CACHE[key] = (csr, B)
+    csr, B = _ORACLE_CACHE[key]
+    Ws = [gen.glorot(dims[l], dims[l + 1], w.seed_W + l) for l in range(L)]
+    y = gen.labels(R, dims[-1], 3)
+    cols = lambda d: np.ascontiguousarray(B[:, :d])
+    rws = lambda d: np.ascontiguousarray(B[rows, :d])
+    wall0 = time.perf_counter()
+    Z = None
+    for l in range(L):                               # forward (Eq. 5-7, §4.4 order)
+        if oracle.spmm_first(dims[l], dims[l + 1]):
+            Z = oracle.gemm(oracle.spmm(csr, cols(dims[l]), rows=rows), Ws[l])
+        else:
+            oracle.gemm(rws(dims[l]), Ws[l])
+            Z = oracle.spmm(csr, cols(dims[l + 1]), rows=rows)
+        Z = oracle.relu(Z) if l < L - 1 else Z
+    oracle.softmax_ce(np.ascontiguousarray(Z), y, R)
+    for l in range(L - 1, -1, -1):                   # backward (Eq. 8-11)
+        if oracle.spmm_first(dims[l], dims[l + 1]):
+            oracle.gemm(rws(dims[l]), rws(dims[l + 1]), transA=True)
+        else:
+            HWG = oracle.spmm(csr, cols(dims[l + 1]), rows=rows)
+            oracle.gemm(rws(dims[l]), HWG, transA=True)
+            if l > 0:
+                oracle.gemm(HWG, Ws[l], transB=True)
+    t_row = time.perf_counter() - wall0
+    t = time.perf_counter()
+    for l in range(L):                               # Adam, full size
+        W = Ws[l].copy()
+        oracle.adam(W, np.ascontiguousarray(W * 0.01), np.zeros_like(W), np.zeros_like(W), 1)
+    t_fixed = time.perf_counter() - t
+    return (t_row * (n / R) + t_fixed) * 1e3, time.perf_counter() - wall0, R
+
+
+def auto_rows(w):
+    # about 3 s of single-core oracle work per sampled epoch
+    per_row = (w.m / w.n) * sum(w.dims) * 2 + 3 * sum(w.dims[l] * w.dims[l + 1] for l in range(len(w.dims) - 1))
+    return int(max(200, min(w.n, 1.5e9 / per_row)))
+
+
+def run_reference(args):
+    """Reference arm of this tier: the CPU oracle, as it stands, on host cores."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    w = gen.WORKLOADS[args.workload]
+    rp, col = gen.rmat_csr(w.n, w.m, w.seed_G)
+    R = args.oracle_rows or auto_rows(w)
+    vals, walls = [], []
+    for s in range(args.warmup + args.steps):
+        est, wall, _ = oracle_epoch_sample(w, rp, col, R, seed=s)
+        if s >= args.warmup:
+            vals.append(est)
+            walls.append(wall)
+    value = statistics.median(vals)
+    sample = f"{R} random output rows of every SpMM/GEMM/CE op of one epoch (n = {w.n}), scaled by n/R; Adam full"
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": statistics.median(walls) * 1e3,
+            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f32 storage, f64 accumulate",
+            "data": "synthetic", "config": workload_desc(w, 1),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------ GPU arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_balinsc22_b200 as mg
+    from paper_conf_icpp_balinsc22_b200 import GCN
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    P = world
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    w = gen.WORKLOADS[args.workload]
+
+    t0 = time.perf_counter()
+    rp, col = gen.rmat_csr(w.n, w.m, w.seed_G)
+    X = gen.features(w.n, w.dims[0], w.seed_X)
+    y = gen.labels(w.n, w.dims[-1], w.seed_y)
+    Ws = [gen.glorot(w.dims[l], w.dims[l + 1], w.seed_W + l) for l in range(len(w.dims) - 1)]
+    t_gen = time.perf_counter() - t0
+
+    nccl_id = None
+    if world > 1:
+        obj = [mg.mggcn_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nccl_id = obj[0]
+    flags = mg.MGGCN_F_PROFILE | (0 if args.no_overlap else mg.MGGCN_F_OVERLAP)
+    if args.tf32x1:
+        flags |= mg.MGGCN_F_TF32X1
+    t0 = time.perf_counter()
+    gm = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed, flags=flags, nccl_id=nccl_id)
+    t_setup = time.perf_counter() - t0
+    gm.set_weights(Ws)
+    Xl = gm.permute_rows(X)
+    yl = gm.permute_rows(y)
+    del X
+    Xd = torch.from_numpy(Xl).cuda()
+    yd = torch.from_numpy(yl).cuda()
+    torch.cuda.synchronize()
+
+    def epoch(Xin, yin, want_loss=False):
+        loss = gm.forward(Xin, yin, want_loss=want_loss)
+        gm.backward()
+        gm.step(lr=0.01)
+        return loss
+
+    for _ in range(args.warmup):
+        epoch(Xd, yd)
+    gm.synchronize()
+    gm.profile(reset=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)       # let the sampler start
+    launches0 = mg.mggcn_kernel_launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(gm.cs)
+    for _ in range(args.steps):
+        epoch(Xd, yd)
+    ev1.record(gm.cs)
+    ev1.synchronize()
+    gm.synchronize()
+    launches = mg.mggcn_kernel_launch_count() - launches0
+    clk = clocks.stop()
+    if world > 1:
+        dist.barrier()
+    ms = ev0.elapsed_time(ev1) / args.steps
+    prof = gm.profile(reset=True)
+    work = gm.epoch_work()
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+
+    # ---- end to end: host (pinned) inputs through the C ABI, loss read back every step
+    e2e = None
+    if not args.no_e2e:
+        Xh = torch.from_numpy(Xl).pin_memory()
+        yh = torch.from_numpy(yl).pin_memory()
+        for _ in range(2):
+            epoch(Xh, yh, want_loss=True)
+        gm.synchronize()
+        if world > 1:
+            dist.barrier()
+        tw = time.perf_counter()
+        for _ in range(args.steps):
+            epoch(Xh, yh, want_loss=True)
+        gm.synchronize()
+        e2e_ms = (time.perf_counter() - tw) * 1e3 / args.steps
+        te = torch.tensor([e2e_ms], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e = {"value": float(te.item()), "unit": UNIT,
+               "h2d_bytes_per_step": int(Xl.nbytes + yl.nbytes), "d2h_bytes_per_step": 16,
+               "how": "wall clock over K epochs; X, y copied from pinned host memory inside mggcn_forward; "
+                      "loss read back (synchronising) every epoch"}
+    loss_now = gm.loss()
+
+    if rank != 0:
+        gm.close()
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peaks = {}
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            peaks = json.load(f)
+    except Exception:
+        pass
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    peak_src = "MEASURED_PEAKS.json hbm_gbs (measured)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"
+    spmm_ms, spmm_n = prof["spmm"]
+    spmm_launch_ms = spmm_ms / max(spmm_n, 1)
+    launches_per_epoch = spmm_n / args.steps
+    bytes_per_launch = work["spmm_bytes"] / max(launches_per_epoch, 1)
+    achieved = bytes_per_launch / (spmm_launch_ms * 1e-3) / 1e9 if spmm_ms > 0 else 0.0
+    gather_gbs = (work["spmm_gather_bytes"] / max(launches_per_epoch, 1)) / (spmm_launch_ms * 1e-3) / 1e9 \
+        if spmm_ms > 0 else 0.0
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", f"spmm_traffic_{args.workload}_P{P}.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    gemm_ms, gemm_n = prof["gemm"]
+    tf32_peak = float(peaks.get("bf16_tflops_sustained", 1352.7)) / 2.0
+
+    line = {
+        "metric": METRIC, "value": ms_max, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": False, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": workload_desc(w, P) | {"overlap": not args.no_overlap,
+                                         "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)"},
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "clocks": clk,
+        "roofline": {"bound": "hbm", "kernel": "spmm_stage (staged CSR SpMM, F2/B1)",
+                     "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
+                     "traffic": traffic, "peak_source": peak_src,
+                     "algorithmic_bytes_per_launch": bytes_per_launch,
+                     "launch_ms": spmm_launch_ms, "launches_per_epoch": launches_per_epoch,
+                     "gather_model_GBps": gather_gbs,
+                     "note": "achieved = compulsory bytes (indices + rowptr + each input and output row once, "
+                             "SURVEY §8d) / measured launch time; gather_model_GBps = nnz*width*4 B / time"},
+        "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
+        "gemm": {"tflops": work["gemm_flops"] / (gemm_ms / args.steps * 1e-3) / 1e12 if gemm_ms else None,
+                 "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps},
+        "loss_after": loss_now,
+        "setup_s": {"generate": t_gen, "load_csr+partition+upload": t_setup},
+    }
+    # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1 only)
+    if world == 1 and not args.no_cpu_baseline:
+        R = args.oracle_rows or auto_rows(w)
+        ests = []
+        for s in range(3):
+            est, _, _ = oracle_epoch_sample(w, rp, col, R, seed=s)
+            ests.append(est)
+        line["cpu_baseline"] = {"value": statistics.median(ests), "unit": UNIT, "cores": 1, "kind": "oracle",
+                                "sample": f"3 x {R} random output rows of every SpMM/GEMM/CE op of one epoch "
+                                          f"(n = {w.n}), scaled by n/R; Adam full; single thread"}
+    print(json.dumps(line), flush=True)
+    gm.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

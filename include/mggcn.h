@@ -58,7 +58,9 @@ enum {
     MGGCN_F_TF32X1 = 4u,      /* 1xTF32 GEMMs (faster, ~1e-3 rel. error); default is
                                  3xTF32 (hi/lo split, ~fp32 accuracy)                  */
     MGGCN_F_NO_BCAST = 16u,   /* TIMING ONLY: skip broadcasts; results invalid         */
-    MGGCN_F_PROFILE = 32u     /* record per-op CUDA events (see mggcn_get_profile)     */
+    MGGCN_F_PROFILE = 32u,    /* record per-op CUDA events (see mggcn_get_profile)     */
+    MGGCN_F_NO_COALESCE = 64u /* keep duplicate entries as separate gathers (default:
+                                 merged on the device copy, value = multiplicity)       */
 };
 
 typedef struct mggcn_graph_s* mggcn_graph; /* host CSR of A + in-degrees                     */

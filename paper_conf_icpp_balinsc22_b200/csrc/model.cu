@@ -65,12 +65,50 @@ void build_items(const HostTile& t, HostItems& h) {
     }
 }
 
+// Duplicate entries (multi-edges, reading C19) are adjacent within a row
+// (tiles are sorted by column); merge them: value = multiplicity for a
+// pattern-only graph (Â_uv = mult / deg(v)), else the fp32 sum of the Â values.
+void coalesce(const HostTile& t, HostTile& o) {
+    o.nrows = t.nrows;
+    o.ncols = t.ncols;
+    o.col0 = t.col0;
+    o.rowptr.assign(t.nrows + 1, 0);
+    o.col.clear();
+    o.val.clear();
+    o.col.reserve(t.col.size());
+    o.val.reserve(t.col.size());
+    const bool pat = t.val.empty();
+    for (int64_t r = 0; r < t.nrows; ++r) {
+        const int64_t b = t.rowptr[r], e = t.rowptr[r + 1];
+        const size_t start = o.col.size();
+        for (int64_t q = b; q < e; ++q) {
+            const float v = pat ? 1.0f : t.val[q];
+            if (o.col.size() > start && o.col.back() == t.col[q]) o.val.back() += v;
+            else {
+                o.col.push_back(t.col[q]);
+                o.val.push_back(v);
+            }
+        }
+        o.rowptr[r + 1] = (int32_t)o.col.size();
+    }
+}
+
 struct Rank {
     const mggcn_part_s* part = nullptr;
     int rank = 0;
     int64_t rows = 0, row_off = 0;   // row_off: offset inside the model's local rows
     std::vector<SpmmTile> F, B;
     std::vector<HostItems> hF, hB;
+    // the tiles as uploaded: the partition's tiles, or (default) a copy with
+    // duplicate entries coalesced into one entry whose value is the
+    // multiplicity (pattern-only) or the sum of the values (weighted)
+    std::vector<HostTile> cF, cB;
+    bool coalesced = false;
+    const HostTile& tF(int j) const { return coalesced ? cF[j] : part->F[j]; }
+    const HostTile& tB(int j) const {
+        if (coalesced) return part->shared_fb ? cF[j] : cB[j];
+        return part->tileB(j);
+    }
     float* inv_deg = nullptr;
     float* Xs = nullptr;
     int32_t* y = nullptr;
@@ -227,7 +265,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                     r.B[j] = r.F[j];
                     continue;
                 }
-                const HostTile& ht = dir == 0 ? pt->F[j] : pt->B[j];
+                const HostTile& ht = dir == 0 ? r.tF(j) : r.tB(j);
                 const HostItems& hi = dir == 0 ? r.hF[j] : r.hB[j];
                 SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
                 t.nrows = ht.nrows;
@@ -239,7 +277,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                 t.items = b.take<int4>(hi.items.size());
                 t.splits = b.take<int4>(hi.splits.size());
                 t.col = b.take<int32_t>(ht.col.size());
-                t.val = pt->pattern ? nullptr : b.take<float>(ht.val.size());
+                t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
             }
         }
         r.inv_deg = b.take<float>(r.rows);
@@ -276,7 +314,7 @@ int upload_static(mggcn_model_s* m) {
         for (int j = 0; j < pt->P; ++j)
             for (int dir = 0; dir < 2; ++dir) {
                 if (dir == 1 && pt->shared_fb) continue;
-                const HostTile& ht = dir == 0 ? pt->F[j] : pt->B[j];
+                const HostTile& ht = dir == 0 ? r.tF(j) : r.tB(j);
                 const HostItems& hi = dir == 0 ? r.hF[j] : r.hB[j];
                 SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
                 if (!hi.items.empty())
@@ -292,7 +330,7 @@ int upload_static(mggcn_model_s* m) {
                     CK(cudaMemcpyAsync(const_cast<float*>(t.val), ht.val.data(), sizeof(float) * ht.val.size(),
                                        cudaMemcpyHostToDevice, m->cs));
             }
-        if (m->pattern && pt->shared_fb)
+        if (pt->shared_fb)
             for (int j = 0; j < pt->P; ++j) r.B[j] = r.F[j];
         CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
         // zero every activation buffer once: padding columns stay 0 forever
@@ -590,9 +628,18 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         off += r.rows;
         r.hF.assign(m->P, HostItems());
         r.hB.assign(m->P, HostItems());
+        r.coalesced = !(flags & MGGCN_F_NO_COALESCE);
+        if (r.coalesced) {
+            r.cF.resize(m->P);
+            for (int j = 0; j < m->P; ++j) coalesce(r.part->F[j], r.cF[j]);
+            if (!r.part->shared_fb) {
+                r.cB.resize(m->P);
+                for (int j = 0; j < m->P; ++j) coalesce(r.part->B[j], r.cB[j]);
+            }
+        }
         for (int j = 0; j < m->P; ++j) {
-            build_items(r.part->F[j], r.hF[j]);
-            if (!r.part->shared_fb) build_items(r.part->B[j], r.hB[j]);
+            build_items(r.tF(j), r.hF[j]);
+            if (!r.part->shared_fb) build_items(r.tB(j), r.hB[j]);
         }
     }
     m->n_local = off;
@@ -600,9 +647,9 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
     auto spmm_work = [&](int dir, int64_t width) {
         for (auto& r : m->ranks)
             for (int j = 0; j < m->P; ++j) {
-                const HostTile& t = dir == 0 ? r.part->F[j] : r.part->tileB(j);
+                const HostTile& t = dir == 0 ? r.tF(j) : r.tB(j);
                 const double nnz = (double)t.rowptr.back();
-                m->w_spmm_bytes += nnz * (m->pattern ? 4.0 : 8.0) + 4.0 * (double)(t.nrows + 1) +
+                m->w_spmm_bytes += nnz * (t.val.empty() ? 4.0 : 8.0) + 4.0 * (double)(t.nrows + 1) +
                                    4.0 * (double)width * (double)(t.ncols + t.nrows);
                 m->w_gather_bytes += nnz * 4.0 * (double)width;
                 if (j != r.rank) m->w_bcast_bytes += 4.0 * (double)width * (double)t.ncols;

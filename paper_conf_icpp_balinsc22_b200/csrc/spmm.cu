@@ -14,6 +14,8 @@
 //   - epilogue fused: accumulate into the previous stage's output (RMW), and
 //     on the last stage the 1/deg row scale (Eq. 2 for pattern-only graphs)
 //     and ReLU (Eq. 7 / Eq. 18 in place).
+#include <cstdlib>
+
 #include "kernels.cuh"
 
 namespace mggcn {
@@ -21,7 +23,6 @@ namespace mggcn {
 namespace {
 
 constexpr int kWarpsPerBlock = 8;
-constexpr int kUnroll = 8;
 
 __device__ __forceinline__ float4 f4_fma(float a, float4 x, float4 acc) {
     acc.x = fmaf(a, x.x, acc.x);
@@ -68,6 +69,14 @@ __device__ __forceinline__ float4 epilogue(float4 acc, const float4* out_row, in
 }
 
 // G lanes per gathered row (1..32), CH float4 chunks per lane, S = 32/G slots.
+// Full groups of U entries per slot are issued with no predicates or selects,
+// so all U*CH 128-bit gathers of a lane are in flight before the first FMA
+// (a select such as `ok ? load : 0` would force a move right after each load
+// and serialise them); only the last < U*S entries of a 32-entry chunk take
+// the guarded tail path.
+template <int CH>
+__host__ __device__ constexpr int unroll_for() { return CH == 1 ? 16 : CH == 2 ? 8 : CH == 3 ? 5 : 4; }
+
 template <int G, int CH, bool VALS>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
@@ -75,66 +84,88 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,
                   const float* __restrict__ rowscale, int w4, int flags) {
     constexpr int S = 32 / G;
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    // U entries per slot per group; U * S <= 32 so a group fits a 32-entry chunk
+    constexpr int U = unroll_for<CH>() < G ? unroll_for<CH>() : G;
     const int lane = threadIdx.x & 31;
-    if (warp >= n_items) return;
-    const int4 it = __ldg(items + warp);
     const int slot = lane / G, cl = lane % G;
-
-    float4 acc[CH];
-#pragma unroll
-    for (int c = 0; c < CH; ++c) acc[c] = make_float4(0.f, 0.f, 0.f, 0.f);
-
-    for (int base = it.y; base < it.z; base += 32) {
-        const int cnt = min(32, it.z - base);
-        const int my_c = lane < cnt ? ld_stream_i32(col + base + lane) : 0;
-        float my_v = 0.f;
-        if (VALS) my_v = lane < cnt ? ld_stream_f32(val + base + lane) : 0.f;
-        // entries k = step*S + slot, steps of U issued together
-        for (int k0 = 0; k0 < cnt; k0 += kUnroll * S) {
-            float4 x[kUnroll][CH];
-            float a[kUnroll];
-#pragma unroll
-            for (int u = 0; u < kUnroll; ++u) {
-                const int k = k0 + u * S + slot;
-                const int c = __shfl_sync(0xffffffffu, my_c, k & 31);
-                float v = VALS ? __shfl_sync(0xffffffffu, my_v, k & 31) : 1.f;
-                const bool ok = k < cnt;
-                a[u] = ok ? v : 0.f;
-                const float4* brow = B + (int64_t)c * ldb4;
-#pragma unroll
-                for (int ch = 0; ch < CH; ++ch) {
-                    const int q = cl + ch * G;
-                    x[u][ch] = (ok && q < w4) ? __ldg(brow + q) : make_float4(0.f, 0.f, 0.f, 0.f);
-                }
-            }
-#pragma unroll
-            for (int u = 0; u < kUnroll; ++u)
-#pragma unroll
-                for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(a[u], x[u][ch], acc[ch]);
-        }
-    }
-    // combine the S slots (fixed xor tree => deterministic)
-#pragma unroll
-    for (int off = G; off < 32; off <<= 1)
-#pragma unroll
-        for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_add(acc[ch], shfl_xor4(acc[ch], off));
-    if (slot != 0) return;
-    if (it.w >= 0) {
-        float4* prow = partial + (int64_t)it.w * ldp4;
-#pragma unroll
-        for (int ch = 0; ch < CH; ++ch) {
-            const int q = cl + ch * G;
-            if (q < w4) prow[q] = acc[ch];
-        }
-        return;
-    }
-    float4* orow = out + (int64_t)it.x * ldo4;
-    const float scale = rowscale ? __ldg(rowscale + it.x) : 1.f;
+    const uint32_t ldb = (uint32_t)ldb4;
+    int qc[CH];
 #pragma unroll
     for (int ch = 0; ch < CH; ++ch) {
         const int q = cl + ch * G;
-        if (q < w4) orow[q] = epilogue(acc[ch], orow, q, flags, scale);
+        qc[ch] = q < w4 ? q : 0;      // clamped: always a valid address, result unused
+    }
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    // persistent warps: static stride over the work items (hub segments first)
+    for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; wi < n_items; wi += nwarps) {
+        const int4 it = __ldg(items + wi);
+        float4 acc[CH];
+#pragma unroll
+        for (int c = 0; c < CH; ++c) acc[c] = make_float4(0.f, 0.f, 0.f, 0.f);
+        int nxt_c = (it.y + lane < it.z) ? ld_stream_i32(col + it.y + lane) : 0;
+        float nxt_v = 0.f;
+        if (VALS) nxt_v = (it.y + lane < it.z) ? ld_stream_f32(val + it.y + lane) : 0.f;
+        for (int base = it.y; base < it.z; base += 32) {
+            const int cnt = min(32, it.z - base);
+            const int my_c = nxt_c;
+            const float my_v = nxt_v;
+            if (base + 32 < it.z) {       // prefetch the next chunk's indices
+                const int e = base + 32 + lane;
+                nxt_c = e < it.z ? ld_stream_i32(col + e) : 0;
+                if (VALS) nxt_v = e < it.z ? ld_stream_f32(val + e) : 0.f;
+            }
+            int k0 = 0;
+            for (; k0 + U * S <= cnt; k0 += U * S) {
+                float4 x[U][CH];
+                float a[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int k = k0 + u * S + slot;
+                    const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, my_c, k);
+                    a[u] = VALS ? __shfl_sync(0xffffffffu, my_v, k) : 1.f;
+                    const float4* brow = B + c * ldb;
+#pragma unroll
+                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = __ldg(brow + qc[ch]);
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(a[u], x[u][ch], acc[ch]);
+            }
+            for (; k0 < cnt; k0 += S) {   // tail: < U*S entries
+                const int k = k0 + slot;
+                const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, my_c, k & 31);
+                const float v = VALS ? __shfl_sync(0xffffffffu, my_v, k & 31) : 1.f;
+                if (k < cnt) {
+                    const float4* brow = B + c * ldb;
+#pragma unroll
+                    for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(v, __ldg(brow + qc[ch]), acc[ch]);
+                }
+            }
+        }
+        // combine the S slots (fixed xor tree => deterministic)
+#pragma unroll
+        for (int off = G; off < 32; off <<= 1)
+#pragma unroll
+            for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_add(acc[ch], shfl_xor4(acc[ch], off));
+        if (slot == 0) {
+            if (it.w >= 0) {
+                float4* prow = partial + (int64_t)it.w * ldp4;
+#pragma unroll
+                for (int ch = 0; ch < CH; ++ch) {
+                    const int q = cl + ch * G;
+                    if (q < w4) prow[q] = acc[ch];
+                }
+            } else {
+                float4* orow = out + (int64_t)it.x * ldo4;
+                const float scale = rowscale ? __ldg(rowscale + it.x) : 1.f;
+#pragma unroll
+                for (int ch = 0; ch < CH; ++ch) {
+                    const int q = cl + ch * G;
+                    if (q < w4) orow[q] = epilogue(acc[ch], orow, q, flags, scale);
+                }
+            }
+        }
     }
 }
 
@@ -156,10 +187,33 @@ spmm_fixup_kernel(const int4* __restrict__ splits, int64_t n_splits, const float
     }
 }
 
+int sm_count() {
+    static int n = 0;
+    if (n == 0) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+template <int G, int CH, bool V>
+int64_t persistent_blocks(int64_t n_items) {
+    static int per_sm = 0;
+    if (per_sm == 0) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmm_stage_kernel<G, CH, V>, kWarpsPerBlock * 32, 0);
+        if (per_sm <= 0) per_sm = 1;
+    }
+    const int64_t need = (n_items + kWarpsPerBlock - 1) / kWarpsPerBlock;
+    const int64_t cap = (int64_t)per_sm * sm_count();
+    return need < cap ? need : cap;
+}
+
 template <int G, int CH>
 cudaError_t launch_gc(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, int64_t ldo4, float4* partial,
                       int64_t ldp4, const float* rowscale, int w4, int flags, cudaStream_t s) {
-    const int64_t blocks = (t.n_items + kWarpsPerBlock - 1) / kWarpsPerBlock;
+    const int64_t blocks = t.val ? persistent_blocks<G, CH, true>(t.n_items) : persistent_blocks<G, CH, false>(t.n_items);
     if (t.val)
         spmm_stage_kernel<G, CH, true><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
             t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags);
@@ -170,14 +224,46 @@ cudaError_t launch_gc(const SpmmTile& t, const float4* B, int64_t ldb4, float4* 
     return cudaGetLastError();
 }
 
+// (G lanes per row, CH float4 per lane): the instantiated shapes; the
+// dispatcher picks the one that covers w4 with the fewest idle lanes.
+#define MGGCN_SPMM_SHAPES(X) \
+    X(1, 1) X(2, 1) X(4, 1) X(8, 1) X(16, 1) X(32, 1) X(2, 2) X(4, 2) X(8, 2) X(16, 2) X(32, 2) \
+    X(4, 3) X(8, 3) X(16, 3) X(32, 3) X(8, 4) X(16, 4) X(32, 4)
+
+cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, int64_t ldo4,
+                        float4* partial, int64_t ldp4, const float* rowscale, int flags, cudaStream_t s) {
+    int bg = 0, bc = 0;
+    double best = 1e9;
+#define MGGCN_PICK(g, c)                                                         \
+    if (g * c >= w4) {                                                            \
+        const double waste = (double)(g * c - w4) / (g * c) + 1e-3 * (c == 1);    \
+        if (waste < best - 1e-9) { best = waste; bg = g; bc = c; }               \
+    }
+    MGGCN_SPMM_SHAPES(MGGCN_PICK)
+#undef MGGCN_PICK
+#define MGGCN_CALL(g, c) \
+    if (bg == g && bc == c) return launch_gc<g, c>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, s);
+    MGGCN_SPMM_SHAPES(MGGCN_CALL)
+#undef MGGCN_CALL
+    return cudaErrorInvalidValue;
+}
+
 }  // namespace
 
 cudaError_t launch_spmm(const SpmmTile& t, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
                         const float* rowscale, int width, int flags, cudaStream_t s) {
     if (t.nrows == 0) return cudaSuccess;
-    // column windows of at most 128 float4 (512 floats)
-    for (int c0 = 0; c0 < width; c0 += 512) {
-        const int w = width - c0 < 512 ? width - c0 : 512;
+    // column windows of at most `win` floats (default 512): narrower windows
+    // keep the gathered operand slice L2-resident and raise occupancy
+    static int win_env = -1;
+    if (win_env < 0) {
+        const char* e = getenv("MGGCN_SPMM_WIN");
+        win_env = e ? atoi(e) : 512;
+        if (win_env < 4 || win_env > 512 || (win_env & 3)) win_env = 512;
+    }
+    const int win = win_env;
+    for (int c0 = 0; c0 < width; c0 += win) {
+        const int w = width - c0 < win ? width - c0 : win;
         const int w4 = (w + 3) / 4;
         const float4* Bw = reinterpret_cast<const float4*>(B + c0);
         float4* Ow = reinterpret_cast<float4*>(out + c0);
@@ -185,15 +271,7 @@ cudaError_t launch_spmm(const SpmmTile& t, const float* B, int64_t ldb, float* o
         const int64_t ldb4 = ldb / 4, ldo4 = ldo / 4, ldp4 = w4;
         cudaError_t e;
         if (t.n_items > 0) {
-            if (w4 <= 1) e = launch_gc<1, 1>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 2) e = launch_gc<2, 1>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 4) e = launch_gc<4, 1>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 8) e = launch_gc<8, 1>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 16) e = launch_gc<16, 1>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 32) e = launch_gc<32, 1>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 64) e = launch_gc<32, 2>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else if (w4 <= 96) e = launch_gc<32, 3>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
-            else e = launch_gc<32, 4>(t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, w4, flags, s);
+            e = dispatch_gc(w4, t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, flags, s);
             if (e != cudaSuccess) return e;
         }
         if (t.n_splits > 0) {

@@ -129,6 +129,16 @@ def test_weighted_directed_epoch(mg, P):
     compare(lib, ref, dims)
 
 
+def test_cora_shaped_no_coalesce(mg):
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    pg = oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed)
+    ref = oracle.epoch(pg, X, y, Ws)
+    lib = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 2, w.perm_seed,
+                      mg.MGGCN_F_OVERLAP | mg.MGGCN_F_NO_COALESCE)
+    compare(lib, ref, w.dims)
+
+
 def test_relu_last_and_no_overlap(mg):
     w = gen.WORKLOADS["cora"]
     rp, col, X, y, Ws = workload_inputs(w)

@@ -100,9 +100,9 @@ def _model(mg, n, rp, col, vals, dims, P, seed, flags=None):
     return GCN(n, rp, col, vals, dims, P=P, perm_seed=seed, flags=flags, loopback=P > 1)
 
 
-def _spmm_check(mg, n, rp, col, vals, P, width, seed, exact):
+def _spmm_check(mg, n, rp, col, vals, P, width, seed, exact, flags=None):
     dims = (max(width, 1), max(width, 1))       # one G-order layer; bc width covers `width`
-    gm = _model(mg, n, rp, col, vals, dims, P, seed)
+    gm = _model(mg, n, rp, col, vals, dims, P, seed, flags)
     pg = oracle.permute_graph(n, rp, col, vals, seed=seed)
     ld = (width + 3) // 4 * 4
     rng = np.random.default_rng(width + P)
@@ -140,13 +140,16 @@ def test_spmm_exactness_graph(mg, P, width):
 
 
 @pytest.mark.parametrize("P", [1, 2, 4])
-@pytest.mark.parametrize("width", [8, 48, 128, 256])
-def test_spmm_rmat_hubs(mg, P, width):
-    """R-MAT with hub rows longer than the 2048-entry split (segments + fix-up)."""
+@pytest.mark.parametrize("width", [8, 44, 48, 100, 128, 172, 256, 512, 600])
+@pytest.mark.parametrize("coalesce", [True, False])
+def test_spmm_rmat_hubs(mg, P, width, coalesce):
+    """R-MAT with hub rows longer than the 2048-entry split (segments + fix-up),
+    duplicate entries merged (default) or kept as separate gathers."""
     n, m = 4096, 400000
     rp, col = gen.rmat_csr(n, m, 17)
     assert np.diff(rp).max() > 4 * 2048
-    _spmm_check(mg, n, rp, col, None, P, width, seed=9, exact=False)
+    flags = mg.MGGCN_F_OVERLAP | (0 if coalesce else mg.MGGCN_F_NO_COALESCE)
+    _spmm_check(mg, n, rp, col, None, P, width, seed=9, exact=False, flags=flags)
 
 
 @pytest.mark.parametrize("P", [1, 3])

@@ -189,6 +189,41 @@ __device__ __forceinline__ void decode_tile(const KParams& p, int tile, int& mt,
     kc = rest / p.m_tiles;
 }
 
+
+// Fused epilogue store of 16 accumulator columns [nb, nb+16) of `row`:
+// ReLU' mask from the old value (Eq. 8 / Eq. 21 in place), inv_deg row scale,
+// ReLU (Eq. 7); 128-bit stores when the 16 columns are all valid.
+__device__ __forceinline__ void store_epilogue(const KParams& p, int row, int nb, const float* v, float sc) {
+    float* dst = p.C + (int64_t)row * p.ldc + nb;
+    if (nb + 16 <= p.N) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+            if (p.flags & GEMM_MASK) {
+                const float4 old = reinterpret_cast<const float4*>(dst)[q];
+                o.x = old.x > 0.f ? o.x : 0.f;
+                o.y = old.y > 0.f ? o.y : 0.f;
+                o.z = old.z > 0.f ? o.z : 0.f;
+                o.w = old.w > 0.f ? o.w : 0.f;
+            }
+            o.x *= sc; o.y *= sc; o.z *= sc; o.w *= sc;
+            if (p.flags & GEMM_RELU) {
+                o.x = fmaxf(o.x, 0.f); o.y = fmaxf(o.y, 0.f);
+                o.z = fmaxf(o.z, 0.f); o.w = fmaxf(o.w, 0.f);
+            }
+            reinterpret_cast<float4*>(dst)[q] = o;
+        }
+    } else {
+        for (int i = 0; i < 16 && nb + i < p.N; ++i) {
+            float o = v[i];
+            if ((p.flags & GEMM_MASK) && !(dst[i] > 0.f)) o = 0.f;
+            o *= sc;
+            if (p.flags & GEMM_RELU) o = fmaxf(o, 0.f);
+            dst[i] = o;
+        }
+    }
+}
+
 template <bool AT, bool BT>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tf32_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const KParams p) {
@@ -339,35 +374,7 @@ gemm_tf32_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                         if (nb + i < p.N) dst[i] = v[i];
                     continue;
                 }
-                float* dst = p.C + (int64_t)row * p.ldc + nb;
-                const float sc = (p.flags & GEMM_SCALE) ? __ldg(p.rowscale + row) : 1.f;
-                if (nb + 16 <= p.N) {
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-                        if (p.flags & GEMM_MASK) {
-                            const float4 old = reinterpret_cast<const float4*>(dst)[q];
-                            o.x = old.x > 0.f ? o.x : 0.f;
-                            o.y = old.y > 0.f ? o.y : 0.f;
-                            o.z = old.z > 0.f ? o.z : 0.f;
-                            o.w = old.w > 0.f ? o.w : 0.f;
-                        }
-                        o.x *= sc; o.y *= sc; o.z *= sc; o.w *= sc;
-                        if (p.flags & GEMM_RELU) {
-                            o.x = fmaxf(o.x, 0.f); o.y = fmaxf(o.y, 0.f);
-                            o.z = fmaxf(o.z, 0.f); o.w = fmaxf(o.w, 0.f);
-                        }
-                        reinterpret_cast<float4*>(dst)[q] = o;
-                    }
-                } else {
-                    for (int i = 0; i < 16 && nb + i < p.N; ++i) {
-                        float o = v[i];
-                        if ((p.flags & GEMM_MASK) && !(dst[i] > 0.f)) o = 0.f;
-                        o *= sc;
-                        if (p.flags & GEMM_RELU) o = fmaxf(o, 0.f);
-                        dst[i] = o;
-                    }
-                }
+                store_epilogue(p, row, nb, v, (p.flags & GEMM_SCALE) ? __ldg(p.rowscale + row) : 1.f);
             }
             tc_fence_before();
             mbar_arrive(tmem_empty + acc);
@@ -377,6 +384,181 @@ gemm_tf32_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     if (warp == kMmaWarp) {
         tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(kTmemCols));
+    }
+}
+
+
+// ===================================================================== rows
+// Row GEMM (op 0 / op 1): C[M x N] = A[M x K] · B^T with B given PRE-SPLIT as
+// tf32 hi / lo copies in K-major [N x K] layout (the weights; split once per
+// step by launch_split_weights).  Per stage: TMA writes raw A (SW128) and
+// B_hi / B_lo straight into the MMA operand buffers; the 4 transform warps
+// split A IN PLACE (A -> A_hi, A_lo); BN = N up to 256 so A is staged once.
+constexpr int kRowStage = 96 * 1024;        // A 16K | A_lo 16K | B_hi 32K | B_lo 32K
+constexpr int kRowBars = 2 * kRowStage;     // 6 mbarriers + TMEM slot
+constexpr int kRowSmem = kRowBars + 256 + 1024;
+
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBh,
+                 const __grid_constant__ CUtensorMap tmBl, const KParams p) {
+    extern __shared__ uint8_t smem_dyn[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_dyn) + 1023) & ~uintptr_t(1023));
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kRowBars);
+    uint64_t* full = bars + 0;
+    uint64_t* xf = bars + 2;
+    uint64_t* empty = bars + 4;
+    uint64_t* tmem_full = bars + 6;
+    uint64_t* tmem_empty = bars + 8;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 10);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const bool x1 = (p.flags & GEMM_TF32X1) != 0;
+    const int BN = p.BN;
+    const uint32_t tcols = BN > 128 ? 512u : 256u;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(full + s, 1);
+            mbar_init(xf + s, 128);
+            mbar_init(empty + s, 1);
+            mbar_init(tmem_full + s, 1);
+            mbar_init(tmem_empty + s, 128);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == kMmaWarp) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(tcols));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int total_tiles = p.m_tiles * p.n_tiles;
+    const int nkb = (p.K + BK - 1) / BK;
+
+    if (warp == kTmaWarp) {
+        if (lane == 0) {
+            const uint32_t bytes = (uint32_t)(BM * BK * 4 + BN * BK * 4 * (x1 ? 1 : 2));
+            uint32_t it = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
+                for (int kb = 0; kb < nkb; ++kb, ++it) {
+                    const int s = it & 1;
+                    const uint32_t ph = (it >> 1) & 1;
+                    uint8_t* st = smem + s * kRowStage;
+                    mbar_wait(empty + s, ph ^ 1);
+                    mbar_expect_tx(full + s, bytes);
+                    tma_load_2d(st, &tmA, kb * BK, mt * BM, full + s);
+                    tma_load_2d(st + 32768, &tmBh, kb * BK, nt * BN, full + s);
+                    if (!x1) tma_load_2d(st + 65536, &tmBl, kb * BK, nt * BN, full + s);
+                }
+            }
+        }
+    } else if (warp >= kXfWarp0 && warp < kXfWarp0 + 4) {
+        const int t = threadIdx.x - kXfWarp0 * 32;
+        uint32_t it = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+            for (int kb = 0; kb < nkb; ++kb, ++it) {
+                const int s = it & 1;
+                const uint32_t ph = (it >> 1) & 1;
+                float4* a = reinterpret_cast<float4*>(smem + s * kRowStage);
+                float4* al = reinterpret_cast<float4*>(smem + s * kRowStage + 16384);
+                mbar_wait(full + s, ph);
+#pragma unroll
+                for (int c = t; c < BM * 8; c += 128) {
+                    float4 v = a[c], h, l;
+                    split4(v, h, l, x1);
+                    a[c] = h;
+                    if (!x1) al[c] = l;
+                }
+                fence_proxy_async();
+                mbar_arrive(xf + s);
+            }
+        }
+    } else if (warp == kMmaWarp) {
+        if (lane == 0) {
+            const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
+                                   ((uint32_t)(BM >> 4) << 24);
+            uint32_t it = 0, tc = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
+                const int acc = tc & 1;
+                const uint32_t aph = (tc >> 1) & 1;
+                mbar_wait(tmem_empty + acc, aph ^ 1);
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
+                for (int kb = 0; kb < nkb; ++kb, ++it) {
+                    const int s = it & 1;
+                    const uint32_t ph = (it >> 1) & 1;
+                    mbar_wait(xf + s, ph);
+                    tc_fence_after();
+                    const uint32_t base = smem_u32(smem + s * kRowStage);
+                    const uint64_t ah = sw128_desc(base), al = sw128_desc(base + 16384);
+                    const uint64_t bh = sw128_desc(base + 32768), bl = sw128_desc(base + 65536);
+#pragma unroll
+                    for (int kk = 0; kk < BK / 8; ++kk) {
+                        const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);
+                        if (!x1) {   // small products first
+                            mma_tf32(d_tmem, al + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
+                            mma_tf32(d_tmem, ah + adv, bl + adv, idesc, 1u);
+                            mma_tf32(d_tmem, ah + adv, bh + adv, idesc, 1u);
+                        } else {
+                            mma_tf32(d_tmem, ah + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
+                        }
+                    }
+                    mma_commit(empty + s);
+                }
+                mma_commit(tmem_full + acc);
+            }
+        }
+    } else {
+        uint32_t tc = 0;
+        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
+            const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
+            const int acc = tc & 1;
+            const uint32_t aph = (tc >> 1) & 1;
+            mbar_wait(tmem_full + acc, aph);
+            tc_fence_after();
+            const int row = mt * BM + warp * 32 + lane;
+            const int n0 = nt * BN;
+            const float sc = ((p.flags & GEMM_SCALE) && row < p.M) ? __ldg(p.rowscale + row) : 1.f;
+            for (int c0 = 0; c0 < BN; c0 += 16) {
+                float v[16];
+                tmem_ld16(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)(acc * BN + c0), v);
+                const int nb = n0 + c0;
+                if (row >= p.M || nb >= p.N) continue;
+                store_epilogue(p, row, nb, v, sc);
+            }
+            tc_fence_before();
+            mbar_arrive(tmem_empty + acc);
+        }
+    }
+    __syncthreads();
+    if (warp == kMmaWarp) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
+    }
+}
+
+// tf32 hi/lo split of a small matrix W (din x dout, row stride ldw) into the
+// two K-major B layouts: T = W^T ([dout x din], stride ldt; op 0 uses it for
+// H·W) and S = W ([din x dout], stride ldw; op 1 uses it for G·W^T).
+__global__ void split_weights_kernel(const float* __restrict__ W, int din, int dout, int64_t ldw,
+                                     float* __restrict__ t_hi, float* __restrict__ t_lo, int64_t ldt,
+                                     float* __restrict__ s_hi, float* __restrict__ s_lo, int x1) {
+    const int64_t total = (int64_t)din * dout;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int c = (int)(i / dout), k = (int)(i % dout);
+        float hi, lo;
+        split_tf32(W[c * ldw + k], hi, lo, x1 != 0);
+        if (t_hi) {
+            t_hi[(int64_t)k * ldt + c] = hi;
+            t_lo[(int64_t)k * ldt + c] = lo;
+        }
+        if (s_hi) {
+            s_hi[(int64_t)c * ldw + k] = hi;
+            s_lo[(int64_t)c * ldw + k] = lo;
+        }
     }
 }
 
@@ -439,17 +621,30 @@ cudaError_t launch_kernel(const GemmPlan& g, const KParams& kp, cudaStream_t s) 
     return cudaGetLastError();
 }
 
+cudaError_t launch_rows(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaError_t e = cudaFuncSetAttribute(gemm_rows_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kRowSmem);
+        if (e != cudaSuccess) return e;
+        attr_set = true;
+    }
+    gemm_rows_kernel<<<g.grid, kThreads, kRowSmem, s>>>(g.tmA, g.tmB, g.tmB2, kp);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
 }  // namespace
 
-int gemm_plan(GemmPlan& g, int op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
-              int64_t ldb, float* C, int64_t ldc, int flags, size_t* partial_floats) {
+int gemm_plan_rows(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* Bhi,
+                   const float* Blo, int64_t ldb, float* C, int64_t ldc, int flags) {
     if (M <= 0 || N <= 0 || K <= 0 || M >= (1 << 30) || K >= (1 << 30) || N > 65536) return -1;
-    if ((lda & 3) || (ldb & 3) || (reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
+    if ((lda & 3) || (ldb & 3) || (reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(Bhi) & 15) ||
+        (reinterpret_cast<uintptr_t>(Blo) & 15))
         return -1;
     g = GemmPlan();
-    g.op = op;
+    g.op = 0;
     g.M = M; g.N = N; g.K = K;
-    g.n_tiles = (int)((N + kMaxBN - 1) / kMaxBN);
+    g.n_tiles = (int)((N + 255) / 256);
     g.BN = (int)(((N + g.n_tiles - 1) / g.n_tiles + 15) / 16 * 16);
     g.m_tiles = (int)((M + BM - 1) / BM);
     g.C = C;
@@ -457,30 +652,54 @@ int gemm_plan(GemmPlan& g, int op, int64_t M, int64_t N, int64_t K, const float*
     g.flags = flags;
     g.k_chunks = 1;
     g.k_chunk_len = (K + BK - 1) / BK * BK;
-    if (op == 2) {
-        const int mn = g.m_tiles * g.n_tiles;
-        int want = (num_sms() + mn - 1) / mn;
-        const int64_t kblocks = (K + BK - 1) / BK;
-        if (want > kblocks) want = (int)kblocks;
-        if (want < 1) want = 1;
-        g.k_chunk_len = (kblocks + want - 1) / want * BK;
-        g.k_chunks = (int)((K + g.k_chunk_len - 1) / g.k_chunk_len);
-        if (partial_floats) *partial_floats = (size_t)g.k_chunks * (size_t)M * (size_t)N;
-    } else if (partial_floats) {
-        *partial_floats = 0;
-    }
-    int rc;
-    // A operand: op 0/1 A is M x K (K contiguous); op 2 A is K x M (M contiguous)
-    if (op == 2) rc = encode2d(&g.tmA, A, M, K, lda, BM, BK, false);
-    else rc = encode2d(&g.tmA, A, K, M, lda, BK, BM, true);
+    int rc = encode2d(&g.tmA, A, K, M, lda, BK, BM, true);
+    if (!rc) rc = encode2d(&g.tmB, Bhi, K, N, ldb, BK, g.BN, true);
+    if (!rc) rc = encode2d(&g.tmB2, Blo, K, N, ldb, BK, g.BN, true);
     if (rc) return rc;
-    // B operand: op 0 and 2: B is K x N (N contiguous); op 1: B is N x K (K contiguous)
-    if (op == 1) rc = encode2d(&g.tmB, B, K, N, ldb, BK, g.BN, true);
-    else rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, BK, false);
+    const int total = g.m_tiles * g.n_tiles;
+    g.grid = total < num_sms() ? total : num_sms();
+    return 0;
+}
+
+int gemm_plan_wgrad(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+                    int64_t ldb, int flags, size_t* partial_floats) {
+    if (M <= 0 || N <= 0 || K <= 0 || M >= (1 << 30) || K >= (1 << 30) || N > 65536) return -1;
+    if ((lda & 3) || (ldb & 3) || (reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
+        return -1;
+    g = GemmPlan();
+    g.op = 2;
+    g.M = M; g.N = N; g.K = K;
+    g.n_tiles = (int)((N + kMaxBN - 1) / kMaxBN);
+    g.BN = (int)(((N + g.n_tiles - 1) / g.n_tiles + 15) / 16 * 16);
+    g.m_tiles = (int)((M + BM - 1) / BM);
+    g.flags = flags;
+    const int mn = g.m_tiles * g.n_tiles;
+    int want = (num_sms() + mn - 1) / mn;
+    const int64_t kblocks = (K + BK - 1) / BK;
+    if (want > kblocks) want = (int)kblocks;
+    if (want < 1) want = 1;
+    g.k_chunk_len = (kblocks + want - 1) / want * BK;
+    g.k_chunks = (int)((K + g.k_chunk_len - 1) / g.k_chunk_len);
+    if (partial_floats) *partial_floats = (size_t)g.k_chunks * (size_t)M * (size_t)N;
+    // A is K x M (M contiguous), B is K x N (N contiguous): raw tiles, transposed in smem
+    int rc = encode2d(&g.tmA, A, M, K, lda, BM, BK, false);
+    if (!rc) rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, BK, false);
     if (rc) return rc;
     const int total = g.m_tiles * g.n_tiles * g.k_chunks;
     g.grid = total < num_sms() ? total : num_sms();
     return 0;
+}
+
+size_t gemm_wgrad_partial_floats(int64_t M, int64_t N, int64_t K) {
+    const int n_tiles = (int)((N + kMaxBN - 1) / kMaxBN);
+    const int m_tiles = (int)((M + BM - 1) / BM);
+    const int mn = m_tiles * n_tiles;
+    int want = (num_sms() + mn - 1) / mn;
+    const int64_t kblocks = (K + BK - 1) / BK;
+    if (want > kblocks) want = (int)kblocks;
+    if (want < 1) want = 1;
+    const int64_t len = (kblocks + want - 1) / want * BK;
+    return (size_t)((K + len - 1) / len) * (size_t)M * (size_t)N;
 }
 
 cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
@@ -490,12 +709,19 @@ cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
     kp.k_chunks = g.k_chunks; kp.k_chunk_len = (int)g.k_chunk_len;
     kp.C = g.C; kp.ldc = g.ldc; kp.partial = g.partial; kp.rowscale = g.rowscale;
     kp.flags = g.flags; kp.op2 = g.op == 2;
-    switch (g.op) {
-        case 0: return launch_kernel<false, true>(g, kp, s);
-        case 1: return launch_kernel<false, false>(g, kp, s);
-        case 2: return launch_kernel<true, true>(g, kp, s);
-        default: return cudaErrorInvalidValue;
-    }
+    if (g.op == 2) return launch_kernel<true, true>(g, kp, s);
+    return launch_rows(g, kp, s);
+}
+
+cudaError_t launch_split_weights(const float* W, int64_t din, int64_t dout, int64_t ldw, float* t_hi, float* t_lo,
+                                 int64_t ldt, float* s_hi, float* s_lo, int x1, cudaStream_t s) {
+    const int64_t total = din * dout;
+    int blocks = (int)((total + 255) / 256);
+    if (blocks > 1184) blocks = 1184;
+    if (blocks < 1) blocks = 1;
+    split_weights_kernel<<<blocks, 256, 0, s>>>(W, (int)din, (int)dout, ldw, t_hi, t_lo, ldt, s_hi, s_lo, x1);
+    count_launches(1);
+    return cudaGetLastError();
 }
 
 }  // namespace mggcn

@@ -56,7 +56,7 @@ struct GemmPlan {
     int64_t M = 0, N = 0, K = 0;
     int BN = 0, m_tiles = 0, n_tiles = 0, k_chunks = 1;
     int64_t k_chunk_len = 0;
-    CUtensorMap tmA, tmB;
+    CUtensorMap tmA, tmB, tmB2;
     float* C = nullptr;
     int64_t ldc = 0;
     float* partial = nullptr;   // op 2: [k_chunks][M][N]
@@ -65,10 +65,20 @@ struct GemmPlan {
     int grid = 0;
 };
 
-// Builds tensor maps + tiling.  A/B pointers must be 16-B aligned, lda/ldb
-// multiples of 4 floats.  For op 2 returns the partial-buffer size needed.
-int gemm_plan(GemmPlan& p, int op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
-              int64_t ldb, float* C, int64_t ldc, int flags, size_t* partial_floats);
+// Row GEMM (op 0 and op 1 of the comment above): C = A · B^T with B given
+// pre-split (launch_split_weights) as tf32 hi / lo copies in K-major [N x K]
+// layout, row stride ldb.  Pointers 16-B aligned, lda / ldb multiples of 4.
+int gemm_plan_rows(GemmPlan& p, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* Bhi,
+                   const float* Blo, int64_t ldb, float* C, int64_t ldc, int flags);
+// Weight-gradient GEMM (op 2): partial[kc] = A^T B over K chunks; caller sets
+// p.partial and reduces with launch_splitk_reduce.
+int gemm_plan_wgrad(GemmPlan& p, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
+                    int64_t ldb, int flags, size_t* partial_floats);
+size_t gemm_wgrad_partial_floats(int64_t M, int64_t N, int64_t K);
+// W (din x dout, stride ldw) -> T = W^T hi/lo ([dout x din], stride ldt) and
+// S = W hi/lo ([din x dout], stride ldw); either pair may be null.
+cudaError_t launch_split_weights(const float* W, int64_t din, int64_t dout, int64_t ldw, float* t_hi, float* t_lo,
+                                 int64_t ldt, float* s_hi, float* s_lo, int x1, cudaStream_t s);
 cudaError_t gemm_launch(const GemmPlan& p, cudaStream_t s);
 // op 2 second pass: C[m][n] (ldc) = sum_kc partial[kc][m][n], in kc order.
 cudaError_t launch_splitk_reduce(const float* partial, int k_chunks, int64_t M, int64_t N, float* C, int64_t ldc,

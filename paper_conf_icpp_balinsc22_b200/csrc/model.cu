@@ -144,6 +144,9 @@ struct mggcn_model_s {
     int64_t bc_ld = 0, hw_ld = 0;
     std::vector<Rank> ranks;
     float *W = nullptr, *Mom = nullptr, *Vel = nullptr, *WG = nullptr;
+    // tf32 hi/lo copies of W for the tcgen05 row GEMMs (refreshed after every update):
+    // Wt_* = W^T [d_{l+1} x ld(d_l)] (B of Eq. 5), Ws_* = W [d_l x ld(d_{l+1})] (B of Eq. 11)
+    std::vector<float*> Wt_hi, Wt_lo, Ws_hi, Ws_lo;
     double* loss_sum = nullptr;
     int64_t* ntrain = nullptr;
     cudaStream_t cs = nullptr, ms = nullptr;
@@ -254,6 +257,14 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
     m->WG = b.take<float>(m->wtotal);
     m->loss_sum = b.take<double>(1);
     m->ntrain = b.take<int64_t>(1);
+    m->Wt_hi.assign(L, nullptr); m->Wt_lo.assign(L, nullptr);
+    m->Ws_hi.assign(L, nullptr); m->Ws_lo.assign(L, nullptr);
+    for (int l = 0; l < L; ++l) {
+        m->Wt_hi[l] = b.take<float>(m->d[l + 1] * m->ld[l]);
+        m->Wt_lo[l] = b.take<float>(m->d[l + 1] * m->ld[l]);
+        m->Ws_hi[l] = b.take<float>(m->d[l] * m->ld[l + 1]);
+        m->Ws_lo[l] = b.take<float>(m->d[l] * m->ld[l + 1]);
+    }
     for (auto& r : m->ranks) {
         const mggcn_part_s* pt = r.part;
         const int P = pt->P;
@@ -301,9 +312,10 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
         r.loss_local = b.take<double>(1);
         r.ntrain_local = b.take<int64_t>(1);
         r.WG_local = (m->nlocal > 1) ? b.take<float>(m->wtotal) : nullptr;
-        // split-K partial for W_G (op 2): k_chunks <= #SMs
+        // split-K partials for W_G (Eq. 10)
         size_t gp = 0;
-        for (int l = 0; l < L; ++l) gp = std::max(gp, (size_t)256 * (size_t)m->d[l] * (size_t)m->d[l + 1]);
+        for (int l = 0; l < L; ++l)
+            gp = std::max(gp, gemm_wgrad_partial_floats(m->d[l], m->d[l + 1], std::max<int64_t>(r.rows, 1)));
         r.gemm_partial = b.take<float>(gp);
     }
 }
@@ -343,6 +355,12 @@ int upload_static(mggcn_model_s* m) {
             if (r.BC[s]) CK(cudaMemsetAsync(r.BC[s], 0, sizeof(float) * m->max_rows_j * m->bc_ld, m->cs));
     }
     CK(cudaMemsetAsync(m->W, 0, sizeof(float) * m->wtotal, m->cs));
+    for (int l = 0; l < m->L; ++l) {
+        CK(cudaMemsetAsync(m->Wt_hi[l], 0, sizeof(float) * m->d[l + 1] * m->ld[l], m->cs));
+        CK(cudaMemsetAsync(m->Wt_lo[l], 0, sizeof(float) * m->d[l + 1] * m->ld[l], m->cs));
+        CK(cudaMemsetAsync(m->Ws_hi[l], 0, sizeof(float) * m->d[l] * m->ld[l + 1], m->cs));
+        CK(cudaMemsetAsync(m->Ws_lo[l], 0, sizeof(float) * m->d[l] * m->ld[l + 1], m->cs));
+    }
     CK(cudaMemsetAsync(m->Mom, 0, sizeof(float) * m->wtotal, m->cs));
     CK(cudaMemsetAsync(m->Vel, 0, sizeof(float) * m->wtotal, m->cs));
     CK(cudaMemsetAsync(m->WG, 0, sizeof(float) * m->wtotal, m->cs));
@@ -354,7 +372,7 @@ float* layer_input(mggcn_model_s* m, Rank& r, int l) { return l == 0 ? r.Xs : r.
 
 int plan_gemms(mggcn_model_s* m) {
     const int L = m->L;
-    const bool x1 = (m->flags & MGGCN_F_TF32X1) != 0;
+    const int flags = (m->flags & MGGCN_F_TF32X1) ? GEMM_TF32X1 : 0;
     for (auto& r : m->ranks) {
         r.g_fwd.assign(L, GemmPlan());
         r.g_wgrad.assign(L, GemmPlan());
@@ -365,41 +383,35 @@ int plan_gemms(mggcn_model_s* m) {
         if (r.rows == 0) continue;
         for (int l = 0; l < L; ++l) {
             const bool relu_here = (l < L - 1) || (m->flags & MGGCN_F_RELU_LAST);
-            const float* Wl = m->W + m->woff[l];
-            int flags = x1 ? GEMM_TF32X1 : 0;
-            size_t pf = 0;
-            // forward: G-order HW = H W -> HWB ; S-order AHW = T W -> AHWB_l (+ReLU)
+            // forward (Eq. 5): G-order HW = H W -> HWB ; S-order AHW = T W (+ReLU) -> AHWB_l
             if (m->order[l] == G_ORDER) {
-                if (gemm_plan(r.g_fwd[l], 0, r.rows, m->d[l + 1], m->d[l], layer_input(m, r, l), m->ld[l], Wl,
-                              m->ld[l + 1], r.HWB, m->ld[l + 1], flags, &pf))
+                if (gemm_plan_rows(r.g_fwd[l], r.rows, m->d[l + 1], m->d[l], layer_input(m, r, l), m->ld[l],
+                                   m->Wt_hi[l], m->Wt_lo[l], m->ld[l], r.HWB, m->ld[l + 1], flags))
                     goto fail;
             } else {
-                if (gemm_plan(r.g_fwd[l], 0, r.rows, m->d[l + 1], m->d[l], r.T0, m->ld[0], Wl, m->ld[l + 1],
-                              r.AHWB[l], m->ld[l + 1], flags | (relu_here ? GEMM_RELU : 0), &pf))
+                if (gemm_plan_rows(r.g_fwd[l], r.rows, m->d[l + 1], m->d[l], r.T0, m->ld[0], m->Wt_hi[l],
+                                   m->Wt_lo[l], m->ld[l], r.AHWB[l], m->ld[l + 1],
+                                   flags | (relu_here ? GEMM_RELU : 0)))
                     goto fail;
             }
             r.has_fwd[l] = 1;
-            // weight gradient (Eq. 10): W_G = H^T HW_G (G) or T^T Z_G (S)
+            // weight gradient (Eq. 10, reading C2): W_G = H^T HW_G (G) or T^T Z_G (S)
             {
                 const float* Aop = m->order[l] == G_ORDER ? layer_input(m, r, l) : r.T0;
                 const float* Bop = m->order[l] == G_ORDER ? r.HWB : r.AHWB[l];
-                const int64_t ldb = m->order[l] == G_ORDER ? m->ld[l + 1] : m->ld[l + 1];
-                if (gemm_plan(r.g_wgrad[l], 2, m->d[l], m->d[l + 1], r.rows, Aop, m->ld[l], Bop, ldb, nullptr, 0,
-                              flags, &pf))
+                size_t pf = 0;
+                if (gemm_plan_wgrad(r.g_wgrad[l], m->d[l], m->d[l + 1], r.rows, Aop, m->ld[l], Bop, m->ld[l + 1], flags,
+                                    &pf))
                     goto fail;
-                if (pf > (size_t)256 * (size_t)m->d[l] * (size_t)m->d[l + 1]) {
-                    set_error("model: split-K partial buffer too small");
-                    return MGGCN_EUNSUPPORTED;
-                }
                 r.g_wgrad[l].partial = r.gemm_partial;
                 r.has_wgrad[l] = 1;
             }
-            // input gradient (Eq. 11) for l > 0 (G-order): AHWB_{l-1} = (HW_G W^T) * [H'_{l-1} > 0] (* inv_deg)
+            // input gradient (Eq. 11) for l > 0: AHWB_{l-1} = (HW_G W^T) * [H'_{l-1} > 0] (* inv_deg)
             if (l > 0) {
                 int f = flags | GEMM_MASK;
                 if (m->order[l - 1] == G_ORDER && m->pattern) f |= GEMM_SCALE;
-                if (gemm_plan(r.g_igrad[l], 1, r.rows, m->d[l], m->d[l + 1], r.HWB, m->ld[l + 1], Wl, m->ld[l + 1],
-                              r.AHWB[l - 1], m->ld[l], f, &pf))
+                if (gemm_plan_rows(r.g_igrad[l], r.rows, m->d[l], m->d[l + 1], r.HWB, m->ld[l + 1], m->Ws_hi[l],
+                                   m->Ws_lo[l], m->ld[l + 1], r.AHWB[l - 1], m->ld[l], f))
                     goto fail;
                 r.g_igrad[l].rowscale = r.inv_deg;
                 r.has_igrad[l] = 1;
@@ -410,6 +422,15 @@ int plan_gemms(mggcn_model_s* m) {
 fail:
     set_error("model: GEMM plan / tensor-map encoding failed (needs an sm_100 device)");
     return MGGCN_ECUDA;
+}
+
+// tf32 hi / lo weight copies for the row GEMMs (after set_weights and Adam).
+int refresh_weight_splits(mggcn_model_s* m) {
+    const int x1 = (m->flags & MGGCN_F_TF32X1) ? 1 : 0;
+    for (int l = 0; l < m->L; ++l)
+        CK(launch_split_weights(m->W + m->woff[l], m->d[l], m->d[l + 1], m->ld[l + 1], m->Wt_hi[l], m->Wt_lo[l],
+                                m->ld[l], m->Ws_hi[l], m->Ws_lo[l], x1, m->cs));
+    return MGGCN_OK;
 }
 
 // --------------------------------------------------------- staged SpMM
@@ -822,6 +843,7 @@ extern "C" int mggcn_set_weights(mggcn_model m, int32_t layer, const float* W) {
     int rc = MGGCN_OK;
     auto body = [&]() -> int {
         CK(cudaMemcpy2DAsync(m->W + m->woff[layer], ld * 4, W, dout * 4, dout * 4, din, cudaMemcpyHostToDevice, m->cs));
+        RC(refresh_weight_splits(m));
         CK(cudaMemsetAsync(m->Mom, 0, sizeof(float) * m->wtotal, m->cs));
         CK(cudaMemsetAsync(m->Vel, 0, sizeof(float) * m->wtotal, m->cs));
         CK(cudaStreamSynchronize(m->cs));
@@ -1094,6 +1116,7 @@ extern "C" int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, flo
         m->t += 1;
         ProfScope ps(m, PC_ADAM, m->cs);
         CK(launch_adam(m->W, m->WG, m->Mom, m->Vel, m->wtotal, lr, beta1, beta2, eps, m->t, m->cs));
+        RC(refresh_weight_splits(m));
         return MGGCN_OK;
     };
     int rc = body();
@@ -1204,30 +1227,44 @@ extern "C" int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int6
 
 extern "C" int mggcn_debug_gemm(int32_t op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda,
                                 const float* B, int64_t ldb, float* C, int64_t ldc, uint32_t flags, uintptr_t stream) {
-    if (op < 0 || op > 2 || !A || !B || !C || ldc < N) {
+    if (op < 0 || op > 2 || !A || !B || !C || ldc < N || M <= 0 || N <= 0 || K <= 0) {
         set_error("debug_gemm: bad arguments");
         return MGGCN_EINVAL;
     }
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-    GemmPlan g;
-    size_t pf = 0;
     const int gf = (flags & MGGCN_F_TF32X1) ? GEMM_TF32X1 : 0;
-    if (gemm_plan(g, op, M, N, K, A, lda, B, ldb, C, ldc, gf, &pf)) {
-        set_error("debug_gemm: plan failed (alignment: pointers 16 B, lda/ldb multiple of 4; needs sm_100)");
-        return MGGCN_EINVAL;
-    }
-    float* part = nullptr;
+    float* scratch = nullptr;
     auto body = [&]() -> int {
+        GemmPlan g;
         if (op == 2) {
-            CK(cudaMalloc(&part, sizeof(float) * (pf + 4)));
-            g.partial = part;
+            size_t pf = 0;
+            if (gemm_plan_wgrad(g, M, N, K, A, lda, B, ldb, gf, &pf)) {
+                set_error("debug_gemm: plan failed (alignment: pointers 16 B, lda/ldb multiple of 4; needs sm_100)");
+                return MGGCN_EINVAL;
+            }
+            CK(cudaMalloc(&scratch, sizeof(float) * (pf + 4)));
+            g.partial = scratch;
+            CK(gemm_launch(g, s));
+            CK(launch_splitk_reduce(scratch, g.k_chunks, M, N, C, ldc, s));
+        } else {
+            // B^T operand as K-major [N x K] hi / lo (op 0: transpose of B [K x N]; op 1: B [N x K] itself)
+            const int64_t ldk = op == 0 ? round_up(K, 4) : ldb;
+            CK(cudaMalloc(&scratch, sizeof(float) * (2 * N * ldk + 8)));
+            float* bh = scratch;
+            float* bl = scratch + N * ldk;
+            CK(cudaMemsetAsync(scratch, 0, sizeof(float) * 2 * N * ldk, s));
+            if (op == 0) CK(launch_split_weights(B, K, N, ldb, bh, bl, ldk, nullptr, nullptr, gf ? 1 : 0, s));
+            else CK(launch_split_weights(B, N, K, ldb, nullptr, nullptr, 0, bh, bl, gf ? 1 : 0, s));
+            if (gemm_plan_rows(g, M, N, K, A, lda, bh, bl, ldk, C, ldc, gf)) {
+                set_error("debug_gemm: plan failed (alignment: pointers 16 B, lda/ldb multiple of 4; needs sm_100)");
+                return MGGCN_EINVAL;
+            }
+            CK(gemm_launch(g, s));
         }
-        CK(gemm_launch(g, s));
-        if (op == 2) CK(launch_splitk_reduce(part, g.k_chunks, M, N, C, ldc, s));
         CK(cudaStreamSynchronize(s));
         return MGGCN_OK;
     };
     int rc = body();
-    if (part) cudaFree(part);
+    if (scratch) cudaFree(scratch);
     return rc;
 }

@@ -202,6 +202,9 @@ template <int G, int CH, bool V>
 int64_t persistent_blocks(int64_t n_items) {
     static int per_sm = 0;
     if (per_sm == 0) {
+        const char* co = getenv("MGGCN_SPMM_CARVEOUT");
+        if (co) cudaFuncSetAttribute(spmm_stage_kernel<G, CH, V>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                     atoi(co));
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmm_stage_kernel<G, CH, V>, kWarpsPerBlock * 32, 0);
         if (per_sm <= 0) per_sm = 1;
     }

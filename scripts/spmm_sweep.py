@@ -16,7 +16,7 @@ wl = sys.argv[1] if len(sys.argv) > 1 else "reddit"
 widths = [int(x) for x in sys.argv[2:]] or [256, 44]
 w = gen.WORKLOADS[wl]
 rp, col = gen.rmat_csr(w.n, w.m, w.seed_G)
-gm = GCN(w.n, rp, col, None, (max(widths), max(widths)), perm_seed=w.perm_seed,
+gm = GCN(w.n, rp, col, None, (max(widths), max(widths)), perm_seed=int(os.environ.get('PERM_SEED', w.perm_seed)),
          flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE)
 for width in widths:
     B = torch.randn((w.n, width), device="cuda")
@@ -35,4 +35,5 @@ for width in widths:
         ms = sp_ms / max(sp_n, 1)
         gb = w.m * width * 4 / 1e9
         print(f"{wl} width {width} dir {d}: {ms:.3f} ms/launch (wall {wall:.3f})  gather {gb / ms:.1f} TB/s  "
-              f"WIN={os.environ.get('MGGCN_SPMM_WIN', '512')}", flush=True)
+              f"WIN={os.environ.get('MGGCN_SPMM_WIN', '512')} CARVE={os.environ.get('MGGCN_SPMM_CARVEOUT')} "
+              f"PERM={os.environ.get('PERM_SEED')}", flush=True)

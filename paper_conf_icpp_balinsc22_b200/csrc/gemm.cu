@@ -146,50 +146,6 @@ __device__ __forceinline__ void split4(float4 x, float4& hi, float4& lo, bool x1
     split_tf32(x.w, hi.w, lo.w, x1);
 }
 
-// Operand tile of `rows` x 32 k.  NOT transposed: raw is already the K-major
-// SW128 image written by TMA -> elementwise split at identical offsets.
-// Transposed: raw[kk][r] (pitch `rows` floats) -> K-major SW128:
-// element (r, k) lives at r*128 + (((k>>2) ^ (r&7)) << 4) + (k&3)*4.
-template <bool TRANS>
-__device__ __forceinline__ void transform_tile(const uint8_t* raw, uint8_t* hi, uint8_t* lo, int rows, int t,
-                                               bool x1) {
-    const int nchunks = rows * 8;   // 16-B chunks
-    if (!TRANS) {
-        const float4* src = reinterpret_cast<const float4*>(raw);
-        float4* h = reinterpret_cast<float4*>(hi);
-        float4* l = reinterpret_cast<float4*>(lo);
-        for (int c = t; c < nchunks; c += 128) {
-            float4 a = src[c], ah, al;
-            split4(a, ah, al, x1);
-            h[c] = ah;
-            if (!x1) l[c] = al;
-        }
-    } else {
-        const float* src = reinterpret_cast<const float*>(raw);
-        for (int idx = t; idx < nchunks; idx += 128) {
-            const int r = idx % rows, kq = idx / rows;
-            float4 a;
-            a.x = src[(4 * kq + 0) * rows + r];
-            a.y = src[(4 * kq + 1) * rows + r];
-            a.z = src[(4 * kq + 2) * rows + r];
-            a.w = src[(4 * kq + 3) * rows + r];
-            float4 ah, al;
-            split4(a, ah, al, x1);
-            const int off = r * 128 + ((kq ^ (r & 7)) << 4);
-            *reinterpret_cast<float4*>(hi + off) = ah;
-            if (!x1) *reinterpret_cast<float4*>(lo + off) = al;
-        }
-    }
-}
-
-__device__ __forceinline__ void decode_tile(const KParams& p, int tile, int& mt, int& nt, int& kc) {
-    nt = tile % p.n_tiles;
-    const int rest = tile / p.n_tiles;
-    mt = rest % p.m_tiles;
-    kc = rest / p.m_tiles;
-}
-
-
 // Fused epilogue store of 16 accumulator columns [nb, nb+16) of `row`:
 // ReLU' mask from the old value (Eq. 8 / Eq. 21 in place), inv_deg row scale,
 // ReLU (Eq. 7); 128-bit stores when the 16 columns are all valid.
@@ -224,38 +180,81 @@ __device__ __forceinline__ void store_epilogue(const KParams& p, int row, int nb
     }
 }
 
-template <bool AT, bool BT>
+// ==================================================================== wgrad
+// Weight-gradient GEMM (op 2, Eq. 10): partial[kc] = A^T B over one K chunk,
+// A [K x M] and B [K x N] both stored K-outer (the feature matrices).  One
+// CTA per (M tile, K chunk), full N <= 256 per tile so A is staged once.
+// Raw tiles come in by TMA (2 stages); warps 0-7 transpose + split them into
+// the K-major SW128 hi / lo operand buffers (1 stage); warp 9 issues the MMAs
+// into one TMEM accumulator; warps 0-3 then drain it into the partial buffer.
+constexpr int kWgRawA = 0;                  // 2 x 16 KB  raw A [32 k][128 m]
+constexpr int kWgRawB = 2 * 16384;          // 2 x 32 KB  raw B [32 k][<=256 n]
+constexpr int kWgAhi = 6 * 16384;           // 16 KB
+constexpr int kWgAlo = 7 * 16384;           // 16 KB
+constexpr int kWgBhi = 8 * 16384;           // 32 KB
+constexpr int kWgBlo = 10 * 16384;          // 32 KB
+constexpr int kWgBars = 12 * 16384;
+constexpr int kWgSmem = kWgBars + 256 + 1024;
+constexpr int kWgXfThreads = 256;
+
+template <int NT>
+__device__ __forceinline__ void transpose_split(const float* __restrict__ raw, uint8_t* hi, uint8_t* lo, int rows,
+                                                int t, bool x1) {
+    // raw[kk][r] (pitch `rows`) -> element (r, k) at r*128 + (((k>>2) ^ (r&7)) << 4) + (k&3)*4
+    const int nchunks = rows * 8;
+    for (int idx = t; idx < nchunks; idx += NT) {
+        const int r = idx % rows, kq = idx / rows;
+        float4 a;
+        a.x = raw[(4 * kq + 0) * rows + r];
+        a.y = raw[(4 * kq + 1) * rows + r];
+        a.z = raw[(4 * kq + 2) * rows + r];
+        a.w = raw[(4 * kq + 3) * rows + r];
+        float4 ah, al;
+        split4(a, ah, al, x1);
+        const int off = r * 128 + ((kq ^ (r & 7)) << 4);
+        *reinterpret_cast<float4*>(hi + off) = ah;
+        if (!x1) *reinterpret_cast<float4*>(lo + off) = al;
+    }
+}
+
 __global__ void __launch_bounds__(kThreads, 1)
-gemm_tf32_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const KParams p) {
+gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const KParams p) {
     extern __shared__ uint8_t smem_dyn[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_dyn) + 1023) & ~uintptr_t(1023));
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kBars);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kWgBars);
     uint64_t* raw_full = bars + 0;
     uint64_t* raw_empty = bars + 2;
     uint64_t* split_full = bars + 4;
-    uint64_t* split_empty = bars + 6;
-    uint64_t* tmem_full = bars + 8;
-    uint64_t* tmem_empty = bars + 10;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 12);
-
+    uint64_t* split_empty = bars + 5;
+    uint64_t* tmem_full = bars + 6;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 7);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
     const int BN = p.BN;
+    const uint32_t tcols = BN > 128 ? 256u : 128u;
+
+    // tile = (m tile, k chunk); n_tiles == 1 (BN = N <= 256) or N tiles of BN
+    const int tile = blockIdx.x;
+    const int nt = tile % p.n_tiles;
+    const int mt = (tile / p.n_tiles) % p.m_tiles;
+    const int kc = tile / (p.n_tiles * p.m_tiles);
+    const int k0 = kc * p.k_chunk_len;
+    const int k1 = min(p.K, k0 + p.k_chunk_len);
+    const int nkb = (k1 - k0 + BK - 1) / BK;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < 2; ++s) {
             mbar_init(raw_full + s, 1);
-            mbar_init(raw_empty + s, 128);
-            mbar_init(split_full + s, 128);
-            mbar_init(split_empty + s, 1);
-            mbar_init(tmem_full + s, 1);
-            mbar_init(tmem_empty + s, 128);
+            mbar_init(raw_empty + s, kWgXfThreads);
         }
+        mbar_init(split_full, kWgXfThreads);
+        mbar_init(split_empty, 1);
+        mbar_init(tmem_full, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == kMmaWarp) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "r"(kTmemCols));
+                     "r"(tcols));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     tc_fence_before();
@@ -263,130 +262,82 @@ gemm_tf32_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
-    const int total_tiles = p.m_tiles * p.n_tiles * p.k_chunks;
-
     if (warp == kTmaWarp) {
         if (lane == 0) {
             const uint32_t bytes = (uint32_t)(BM * BK * 4 + BN * BK * 4);
-            uint32_t it = 0;
-            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
-                int mt, nt, kc;
-                decode_tile(p, tile, mt, nt, kc);
-                const int k0 = kc * p.k_chunk_len;
-                const int k1 = min(p.K, k0 + p.k_chunk_len);
-                for (int k = k0; k < k1; k += BK, ++it) {
-                    const int s = it & 1;
-                    const uint32_t ph = (it >> 1) & 1;
-                    mbar_wait(raw_empty + s, ph ^ 1);
-                    mbar_expect_tx(raw_full + s, bytes);
-                    if (AT) tma_load_2d(smem + kRawA + s * 16384, &tmA, mt * BM, k, raw_full + s);
-                    else tma_load_2d(smem + kRawA + s * 16384, &tmA, k, mt * BM, raw_full + s);
-                    if (BT) tma_load_2d(smem + kRawB + s * 16384, &tmB, nt * BN, k, raw_full + s);
-                    else tma_load_2d(smem + kRawB + s * 16384, &tmB, k, nt * BN, raw_full + s);
-                }
-            }
-        }
-    } else if (warp >= kXfWarp0 && warp < kXfWarp0 + 4) {
-        const int t = threadIdx.x - kXfWarp0 * 32;
-        uint32_t it = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
-            int mt, nt, kc;
-            decode_tile(p, tile, mt, nt, kc);
-            const int k0 = kc * p.k_chunk_len;
-            const int k1 = min(p.K, k0 + p.k_chunk_len);
-            for (int k = k0; k < k1; k += BK, ++it) {
-                const int s = it & 1;
-                const uint32_t ph = (it >> 1) & 1;
-                mbar_wait(raw_full + s, ph);
-                mbar_wait(split_empty + s, ph ^ 1);
-                transform_tile<AT>(smem + kRawA + s * 16384, smem + kAhi + s * 16384, smem + kAlo + s * 16384, BM, t,
-                                   x1);
-                transform_tile<BT>(smem + kRawB + s * 16384, smem + kBhi + s * 16384, smem + kBlo + s * 16384, BN, t,
-                                   x1);
-                fence_proxy_async();
-                mbar_arrive(raw_empty + s);
-                mbar_arrive(split_full + s);
+            for (int kb = 0; kb < nkb; ++kb) {
+                const int s = kb & 1;
+                const uint32_t ph = (kb >> 1) & 1;
+                mbar_wait(raw_empty + s, ph ^ 1);
+                mbar_expect_tx(raw_full + s, bytes);
+                tma_load_2d(smem + kWgRawA + s * 16384, &tmA, mt * BM, k0 + kb * BK, raw_full + s);
+                tma_load_2d(smem + kWgRawB + s * 32768, &tmB, nt * BN, k0 + kb * BK, raw_full + s);
             }
         }
     } else if (warp == kMmaWarp) {
         if (lane == 0) {
-            // instruction descriptor: D f32, A/B tf32, both K-major, N>>3 at 17, M>>4 at 24
             const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
                                    ((uint32_t)(BM >> 4) << 24);
-            uint32_t it = 0, tc = 0;
-            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
-                int mt, nt, kc;
-                decode_tile(p, tile, mt, nt, kc);
-                const int k0 = kc * p.k_chunk_len;
-                const int k1 = min(p.K, k0 + p.k_chunk_len);
-                const int acc = tc & 1;
-                const uint32_t aph = (tc >> 1) & 1;
-                mbar_wait(tmem_empty + acc, aph ^ 1);
+            const uint64_t ah = sw128_desc(smem_u32(smem + kWgAhi)), al = sw128_desc(smem_u32(smem + kWgAlo));
+            const uint64_t bh = sw128_desc(smem_u32(smem + kWgBhi)), bl = sw128_desc(smem_u32(smem + kWgBlo));
+            for (int kb = 0; kb < nkb; ++kb) {
+                mbar_wait(split_full, kb & 1);
                 tc_fence_after();
-                const uint32_t d_tmem = tmem_base + (uint32_t)(acc * kMaxBN);
-                bool first = true;
-                for (int k = k0; k < k1; k += BK, ++it) {
-                    const int s = it & 1;
-                    const uint32_t ph = (it >> 1) & 1;
-                    mbar_wait(split_full + s, ph);
-                    tc_fence_after();
-                    const uint64_t ah = sw128_desc(smem_u32(smem + kAhi + s * 16384));
-                    const uint64_t al = sw128_desc(smem_u32(smem + kAlo + s * 16384));
-                    const uint64_t bh = sw128_desc(smem_u32(smem + kBhi + s * 16384));
-                    const uint64_t bl = sw128_desc(smem_u32(smem + kBlo + s * 16384));
 #pragma unroll
-                    for (int kk = 0; kk < BK / 8; ++kk) {
-                        const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);   // 32 B per UMMA_K=8 step
-                        mma_tf32(d_tmem, ah + adv, bh + adv, idesc, first ? 0u : 1u);
-                        first = false;
-                        if (!x1) {
-                            mma_tf32(d_tmem, ah + adv, bl + adv, idesc, 1u);
-                            mma_tf32(d_tmem, al + adv, bh + adv, idesc, 1u);
-                        }
+                for (int kk = 0; kk < BK / 8; ++kk) {
+                    const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);
+                    if (!x1) {
+                        mma_tf32(tmem_base, al + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
+                        mma_tf32(tmem_base, ah + adv, bl + adv, idesc, 1u);
+                        mma_tf32(tmem_base, ah + adv, bh + adv, idesc, 1u);
+                    } else {
+                        mma_tf32(tmem_base, ah + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
                     }
-                    mma_commit(split_empty + s);
                 }
-                mma_commit(tmem_full + acc);
+                mma_commit(split_empty);
             }
+            mma_commit(tmem_full);
         }
     } else {
-        // epilogue warps 0-3: TMEM lane quadrant = warp
-        uint32_t tc = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
-            int mt, nt, kc;
-            decode_tile(p, tile, mt, nt, kc);
-            const int acc = tc & 1;
-            const uint32_t aph = (tc >> 1) & 1;
-            mbar_wait(tmem_full + acc, aph);
+        // warps 0-7: transform every k block; then warps 0-3 run the epilogue
+        const int t = threadIdx.x;
+        for (int kb = 0; kb < nkb; ++kb) {
+            const int s = kb & 1;
+            const uint32_t ph = (kb >> 1) & 1;
+            mbar_wait(raw_full + s, ph);
+            mbar_wait(split_empty, (kb & 1) ^ 1);
+            transpose_split<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawA + s * 16384), smem + kWgAhi,
+                                          smem + kWgAlo, BM, t, x1);
+            transpose_split<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawB + s * 32768), smem + kWgBhi,
+                                          smem + kWgBlo, BN, t, x1);
+            fence_proxy_async();
+            mbar_arrive(raw_empty + s);
+            mbar_arrive(split_full);
+        }
+        if (warp < 4) {
+            mbar_wait(tmem_full, 0);
             tc_fence_after();
             const int row = mt * BM + warp * 32 + lane;
             const int n0 = nt * BN;
             for (int c0 = 0; c0 < BN; c0 += 16) {
                 float v[16];
-                tmem_ld16(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)(acc * kMaxBN + c0), v);
-                if (row >= p.M) continue;
+                tmem_ld16(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
                 const int nb = n0 + c0;
-                if (nb >= p.N) continue;
-                if (p.op2) {
-                    float* dst = p.partial + ((int64_t)kc * p.M + row) * (int64_t)p.N + nb;
+                if (row >= p.M || nb >= p.N) continue;
+                float* dst = p.partial + ((int64_t)kc * p.M + row) * (int64_t)p.N + nb;
 #pragma unroll
-                    for (int i = 0; i < 16; ++i)
-                        if (nb + i < p.N) dst[i] = v[i];
-                    continue;
-                }
-                store_epilogue(p, row, nb, v, (p.flags & GEMM_SCALE) ? __ldg(p.rowscale + row) : 1.f);
+                for (int i = 0; i < 16; ++i)
+                    if (nb + i < p.N) dst[i] = v[i];
             }
             tc_fence_before();
-            mbar_arrive(tmem_empty + acc);
         }
     }
     __syncthreads();
     if (warp == kMmaWarp) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(kTmemCols));
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
     }
 }
-
 
 // ===================================================================== rows
 // Row GEMM (op 0 / op 1): C[M x N] = A[M x K] · B^T with B given PRE-SPLIT as
@@ -607,16 +558,14 @@ int num_sms() {
     return n;
 }
 
-template <bool AT, bool BT>
-cudaError_t launch_kernel(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
+cudaError_t launch_wgrad(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
     static bool attr_set = false;
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(gemm_tf32_kernel<AT, BT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             kSmemBytes);
+        cudaError_t e = cudaFuncSetAttribute(gemm_wgrad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kWgSmem);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    gemm_tf32_kernel<AT, BT><<<g.grid, kThreads, kSmemBytes, s>>>(g.tmA, g.tmB, kp);
+    gemm_wgrad_kernel<<<g.grid, kThreads, kWgSmem, s>>>(g.tmA, g.tmB, kp);
     count_launches(1);
     return cudaGetLastError();
 }
@@ -669,7 +618,7 @@ int gemm_plan_wgrad(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A
     g = GemmPlan();
     g.op = 2;
     g.M = M; g.N = N; g.K = K;
-    g.n_tiles = (int)((N + kMaxBN - 1) / kMaxBN);
+    g.n_tiles = (int)((N + 255) / 256);
     g.BN = (int)(((N + g.n_tiles - 1) / g.n_tiles + 15) / 16 * 16);
     g.m_tiles = (int)((M + BM - 1) / BM);
     g.flags = flags;
@@ -685,13 +634,12 @@ int gemm_plan_wgrad(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A
     int rc = encode2d(&g.tmA, A, M, K, lda, BM, BK, false);
     if (!rc) rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, BK, false);
     if (rc) return rc;
-    const int total = g.m_tiles * g.n_tiles * g.k_chunks;
-    g.grid = total < num_sms() ? total : num_sms();
+    g.grid = g.m_tiles * g.n_tiles * g.k_chunks;   // one CTA per tile
     return 0;
 }
 
 size_t gemm_wgrad_partial_floats(int64_t M, int64_t N, int64_t K) {
-    const int n_tiles = (int)((N + kMaxBN - 1) / kMaxBN);
+    const int n_tiles = (int)((N + 255) / 256);
     const int m_tiles = (int)((M + BM - 1) / BM);
     const int mn = m_tiles * n_tiles;
     int want = (num_sms() + mn - 1) / mn;
@@ -709,7 +657,7 @@ cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
     kp.k_chunks = g.k_chunks; kp.k_chunk_len = (int)g.k_chunk_len;
     kp.C = g.C; kp.ldc = g.ldc; kp.partial = g.partial; kp.rowscale = g.rowscale;
     kp.flags = g.flags; kp.op2 = g.op == 2;
-    if (g.op == 2) return launch_kernel<true, true>(g, kp, s);
+    if (g.op == 2) return launch_wgrad(g, kp, s);
     return launch_rows(g, kp, s);
 }
 

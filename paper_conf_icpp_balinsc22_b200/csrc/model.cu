@@ -929,12 +929,31 @@ extern "C" int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, co
 static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int32_t* y, float* loss,
                         float* logits) {
     const int L = m->L;
-    // inputs -> internal buffers (host or device source; this is the e2e H2D when host)
+    // inputs -> internal buffers (host or device source; this is the e2e H2D when host).
+    // A host X with a row pitch != the padded ld is staged through HWB (free at
+    // this point) in contiguous chunks: one 1-D H2D copy per chunk, then a
+    // device 2-D copy into the padded layout (pitched H2D copies are slow).
+    cudaPointerAttributes pa;
+    const bool host_x = cudaPointerGetAttributes(&pa, X) != cudaSuccess || pa.type == cudaMemoryTypeHost ||
+                        pa.type == cudaMemoryTypeUnregistered;
+    cudaGetLastError();   // clear a possible error from the attribute query
     for (auto& r : m->ranks) {
         if (r.rows == 0) continue;
         ProfScope ps(m, PC_OTHER, m->cs);
-        CK(cudaMemcpy2DAsync(r.Xs, m->ld[0] * 4, X + r.row_off * ldx, ldx * 4, m->d[0] * 4, r.rows,
-                             cudaMemcpyDefault, m->cs));
+        if (host_x && ldx != m->ld[0]) {
+            const int64_t stage_floats = r.rows * std::max<int64_t>(m->hw_ld, 4);
+            const int64_t chunk = std::max<int64_t>(1, stage_floats / ldx);
+            for (int64_t r0 = 0; r0 < r.rows; r0 += chunk) {
+                const int64_t nr = std::min(chunk, r.rows - r0);
+                CK(cudaMemcpyAsync(r.HWB, X + (r.row_off + r0) * ldx, sizeof(float) * nr * ldx,
+                                   cudaMemcpyHostToDevice, m->cs));
+                CK(cudaMemcpy2DAsync(r.Xs + r0 * m->ld[0], m->ld[0] * 4, r.HWB, ldx * 4, m->d[0] * 4, nr,
+                                     cudaMemcpyDeviceToDevice, m->cs));
+            }
+        } else {
+            CK(cudaMemcpy2DAsync(r.Xs, m->ld[0] * 4, X + r.row_off * ldx, ldx * 4, m->d[0] * 4, r.rows,
+                                 cudaMemcpyDefault, m->cs));
+        }
         CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
     }
     for (int l = 0; l < L; ++l) {

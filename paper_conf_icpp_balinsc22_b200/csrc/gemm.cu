@@ -19,6 +19,7 @@
 // accumulator[2] MMA -> epilogue (double-buffered TMEM, 2 x 128 columns).
 #include <cuda.h>
 
+#include <cstdlib>
 #include <mutex>
 
 #include "kernels.cuh"
@@ -182,73 +183,94 @@ __device__ __forceinline__ void store_epilogue(const KParams& p, int row, int nb
 
 // ==================================================================== wgrad
 // Weight-gradient GEMM (op 2, Eq. 10): partial[kc] = A^T B over one K chunk,
-// A [K x M] and B [K x N] both stored K-outer (the feature matrices).  One
-// CTA per (M tile, K chunk), full N <= 256 per tile so A is staged once.
-// Raw tiles come in by TMA (2 stages); warps 0-7 transpose + split them into
-// the K-major SW128 hi / lo operand buffers (1 stage); warp 9 issues the MMAs
-// into one TMEM accumulator; warps 0-3 then drain it into the partial buffer.
-constexpr int kWgRawA = 0;                  // 2 x 16 KB  raw A [32 k][128 m]
-constexpr int kWgRawB = 2 * 16384;          // 2 x 32 KB  raw B [32 k][<=256 n]
-constexpr int kWgAhi = 6 * 16384;           // 16 KB
-constexpr int kWgAlo = 7 * 16384;           // 16 KB
-constexpr int kWgBhi = 8 * 16384;           // 32 KB
-constexpr int kWgBlo = 10 * 16384;          // 32 KB
-constexpr int kWgBars = 12 * 16384;
+// A [K x M] and B [K x N] both stored K-outer (the feature matrices).
+// (MN-major operand descriptors with kind::tf32 produced all-zero
+// accumulators on B200 in our tests, so the operands are transposed.)
+// K blocks of 16: raw tiles [16 k][M or N] come in by TMA (3 stages, no
+// swizzle); 8 warps transpose + split them into K-major SWIZZLE_64B hi / lo
+// operand buffers (3 stages) so the transform of block kb+1 overlaps the MMAs
+// of block kb; warp 9 issues hi.hi + hi.lo + lo.hi per 8-deep k step; warps
+// 0-3 drain the TMEM accumulator into the split-K partial buffer.
+constexpr int kWgBK = 16;
+constexpr int kWgNS = 3;                         // pipeline stages
+constexpr int kWgRawA = 0;                       // 3 x  8 KB  raw A [16 k][128 m]
+constexpr int kWgRawB = kWgNS * 8192;            // 3 x 16 KB  raw B [16 k][<=256 n]
+constexpr int kWgSplit = kWgRawB + kWgNS * 16384;  // 3 x 48 KB: A_hi 8K | A_lo 8K | B_hi 16K | B_lo 16K
+constexpr int kWgSplitStage = 49152;
+constexpr int kWgBars = kWgSplit + kWgNS * kWgSplitStage;
 constexpr int kWgSmem = kWgBars + 256 + 1024;
 constexpr int kWgXfThreads = 256;
 
+// K-major SWIZZLE_64B descriptor: rows of 64 B (16 tf32), 8-row atoms 512 B apart.
+__device__ __forceinline__ uint64_t sw64_desc(uint32_t saddr) {
+    return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(512 >> 4) << 32) |
+           ((uint64_t)1 << 46) | ((uint64_t)4 << 61);
+}
+
+// raw[kk][r] (pitch `rows`, kk < 16) -> K-major SW64: element (r, k) at
+// r*64 + (((k>>2) ^ ((r>>1)&3)) << 4) + (k&3)*4.  Thread t owns row
+// r = t % rows and the k-quads kq = g, g+G, ... (g = t / rows, G = NT / rows):
+// all its shared loads are issued before the first split (ILP).
 template <int NT>
-__device__ __forceinline__ void transpose_split(const float* __restrict__ raw, uint8_t* hi, uint8_t* lo, int rows,
-                                                int t, bool x1) {
-    // raw[kk][r] (pitch `rows`) -> element (r, k) at r*128 + (((k>>2) ^ (r&7)) << 4) + (k&3)*4
-    const int nchunks = rows * 8;
-    for (int idx = t; idx < nchunks; idx += NT) {
-        const int r = idx % rows, kq = idx / rows;
-        float4 a;
-        a.x = raw[(4 * kq + 0) * rows + r];
-        a.y = raw[(4 * kq + 1) * rows + r];
-        a.z = raw[(4 * kq + 2) * rows + r];
-        a.w = raw[(4 * kq + 3) * rows + r];
-        float4 ah, al;
-        split4(a, ah, al, x1);
-        const int off = r * 128 + ((kq ^ (r & 7)) << 4);
-        *reinterpret_cast<float4*>(hi + off) = ah;
-        if (!x1) *reinterpret_cast<float4*>(lo + off) = al;
+__device__ __forceinline__ void transpose_split16(const float* __restrict__ raw, uint8_t* hi, uint8_t* lo, int rows,
+                                                  int t, bool x1) {
+    const int G = NT / rows;
+    const int g = t / rows, r = t - g * rows;
+    if (g >= G) return;
+    float4 a[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const int kq = g + j * G;
+        if (kq < 4) {
+            a[j].x = raw[(4 * kq + 0) * rows + r];
+            a[j].y = raw[(4 * kq + 1) * rows + r];
+            a[j].z = raw[(4 * kq + 2) * rows + r];
+            a[j].w = raw[(4 * kq + 3) * rows + r];
+        }
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const int kq = g + j * G;
+        if (kq < 4) {
+            float4 ah, al;
+            split4(a[j], ah, al, x1);
+            const int off = r * 64 + ((kq ^ ((r >> 1) & 3)) << 4);
+            *reinterpret_cast<float4*>(hi + off) = ah;
+            if (!x1) *reinterpret_cast<float4*>(lo + off) = al;
+        }
     }
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const KParams p) {
     extern __shared__ uint8_t smem_dyn[];
-    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_dyn) + 1023) & ~uintptr_t(1023));
+    uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);   // keeps the shared state space
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kWgBars);
-    uint64_t* raw_full = bars + 0;
-    uint64_t* raw_empty = bars + 2;
-    uint64_t* split_full = bars + 4;
-    uint64_t* split_empty = bars + 5;
-    uint64_t* tmem_full = bars + 6;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 7);
+    uint64_t* raw_full = bars + 0;               // [3]
+    uint64_t* raw_empty = bars + 3;              // [3]
+    uint64_t* split_full = bars + 6;             // [3]
+    uint64_t* split_empty = bars + 9;            // [3]
+    uint64_t* tmem_full = bars + 12;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
     const int BN = p.BN;
     const uint32_t tcols = BN > 128 ? 256u : 128u;
-
-    // tile = (m tile, k chunk); n_tiles == 1 (BN = N <= 256) or N tiles of BN
     const int tile = blockIdx.x;
     const int nt = tile % p.n_tiles;
     const int mt = (tile / p.n_tiles) % p.m_tiles;
     const int kc = tile / (p.n_tiles * p.m_tiles);
     const int k0 = kc * p.k_chunk_len;
     const int k1 = min(p.K, k0 + p.k_chunk_len);
-    const int nkb = (k1 - k0 + BK - 1) / BK;
+    const int nkb = (k1 - k0 + kWgBK - 1) / kWgBK;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < 2; ++s) {
+        for (int s = 0; s < kWgNS; ++s) {
             mbar_init(raw_full + s, 1);
             mbar_init(raw_empty + s, kWgXfThreads);
+            mbar_init(split_full + s, kWgXfThreads);
+            mbar_init(split_empty + s, 1);
         }
-        mbar_init(split_full, kWgXfThreads);
-        mbar_init(split_empty, 1);
         mbar_init(tmem_full, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -264,28 +286,32 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 
     if (warp == kTmaWarp) {
         if (lane == 0) {
-            const uint32_t bytes = (uint32_t)(BM * BK * 4 + BN * BK * 4);
+            const uint32_t bytes = (uint32_t)(BM * kWgBK * 4 + BN * kWgBK * 4);
+            int s = 0;
+            uint32_t ph = 0;
             for (int kb = 0; kb < nkb; ++kb) {
-                const int s = kb & 1;
-                const uint32_t ph = (kb >> 1) & 1;
                 mbar_wait(raw_empty + s, ph ^ 1);
                 mbar_expect_tx(raw_full + s, bytes);
-                tma_load_2d(smem + kWgRawA + s * 16384, &tmA, mt * BM, k0 + kb * BK, raw_full + s);
-                tma_load_2d(smem + kWgRawB + s * 32768, &tmB, nt * BN, k0 + kb * BK, raw_full + s);
+                tma_load_2d(smem + kWgRawA + s * 8192, &tmA, mt * BM, k0 + kb * kWgBK, raw_full + s);
+                tma_load_2d(smem + kWgRawB + s * 16384, &tmB, nt * BN, k0 + kb * kWgBK, raw_full + s);
+                if (++s == kWgNS) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == kMmaWarp) {
         if (lane == 0) {
             const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
                                    ((uint32_t)(BM >> 4) << 24);
-            const uint64_t ah = sw128_desc(smem_u32(smem + kWgAhi)), al = sw128_desc(smem_u32(smem + kWgAlo));
-            const uint64_t bh = sw128_desc(smem_u32(smem + kWgBhi)), bl = sw128_desc(smem_u32(smem + kWgBlo));
+            int s = 0;
+            uint32_t ph = 0;
             for (int kb = 0; kb < nkb; ++kb) {
-                mbar_wait(split_full, kb & 1);
+                mbar_wait(split_full + s, ph);
                 tc_fence_after();
+                const uint32_t base = smem_u32(smem + kWgSplit + s * kWgSplitStage);
+                const uint64_t ah = sw64_desc(base), al = sw64_desc(base + 8192);
+                const uint64_t bh = sw64_desc(base + 16384), bl = sw64_desc(base + 32768);
 #pragma unroll
-                for (int kk = 0; kk < BK / 8; ++kk) {
-                    const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);
+                for (int kk = 0; kk < kWgBK / 8; ++kk) {
+                    const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);   // 32 B per 8-deep k step
                     if (!x1) {
                         mma_tf32(tmem_base, al + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
                         mma_tf32(tmem_base, ah + adv, bl + adv, idesc, 1u);
@@ -294,25 +320,28 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                         mma_tf32(tmem_base, ah + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
                     }
                 }
-                mma_commit(split_empty);
+                mma_commit(split_empty + s);
+                if (++s == kWgNS) { s = 0; ph ^= 1; }
             }
             mma_commit(tmem_full);
         }
     } else {
-        // warps 0-7: transform every k block; then warps 0-3 run the epilogue
+        // warps 0-7: transpose + split every k block; then warps 0-3 run the epilogue
         const int t = threadIdx.x;
+        int s = 0;
+        uint32_t ph = 0;
         for (int kb = 0; kb < nkb; ++kb) {
-            const int s = kb & 1;
-            const uint32_t ph = (kb >> 1) & 1;
+            uint8_t* sp = smem + kWgSplit + s * kWgSplitStage;
             mbar_wait(raw_full + s, ph);
-            mbar_wait(split_empty, (kb & 1) ^ 1);
-            transpose_split<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawA + s * 16384), smem + kWgAhi,
-                                          smem + kWgAlo, BM, t, x1);
-            transpose_split<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawB + s * 32768), smem + kWgBhi,
-                                          smem + kWgBlo, BN, t, x1);
+            mbar_wait(split_empty + s, ph ^ 1);
+            transpose_split16<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawA + s * 8192), sp, sp + 8192,
+                                            BM, t, x1);
+            transpose_split16<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawB + s * 16384), sp + 16384,
+                                            sp + 32768, BN, t, x1);
             fence_proxy_async();
             mbar_arrive(raw_empty + s);
-            mbar_arrive(split_full);
+            mbar_arrive(split_full + s);
+            if (++s == kWgNS) { s = 0; ph ^= 1; }
         }
         if (warp < 4) {
             mbar_wait(tmem_full, 0);
@@ -353,7 +382,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBh,
                  const __grid_constant__ CUtensorMap tmBl, const KParams p) {
     extern __shared__ uint8_t smem_dyn[];
-    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_dyn) + 1023) & ~uintptr_t(1023));
+    uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);   // keeps the shared state space
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kRowBars);
     uint64_t* full = bars + 0;
     uint64_t* xf = bars + 2;
@@ -630,9 +659,9 @@ int gemm_plan_wgrad(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A
     g.k_chunk_len = (kblocks + want - 1) / want * BK;
     g.k_chunks = (int)((K + g.k_chunk_len - 1) / g.k_chunk_len);
     if (partial_floats) *partial_floats = (size_t)g.k_chunks * (size_t)M * (size_t)N;
-    // A is K x M (M contiguous), B is K x N (N contiguous): raw tiles, transposed in smem
-    int rc = encode2d(&g.tmA, A, M, K, lda, BM, BK, false);
-    if (!rc) rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, BK, false);
+    // A is K x M (M contiguous), B is K x N (N contiguous): raw boxes {M or N, 16 K}, transposed in smem
+    int rc = encode2d(&g.tmA, A, M, K, lda, BM, 16, false);
+    if (!rc) rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, 16, false);
     if (rc) return rc;
     g.grid = g.m_tiles * g.n_tiles * g.k_chunks;   // one CTA per tile
     return 0;
@@ -657,6 +686,7 @@ cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
     kp.k_chunks = g.k_chunks; kp.k_chunk_len = (int)g.k_chunk_len;
     kp.C = g.C; kp.ldc = g.ldc; kp.partial = g.partial; kp.rowscale = g.rowscale;
     kp.flags = g.flags; kp.op2 = g.op == 2;
+
     if (g.op == 2) return launch_wgrad(g, kp, s);
     return launch_rows(g, kp, s);
 }

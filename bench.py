@@ -200,6 +200,7 @@ def main():
 
     import paper_conf_icpp_balinsc22_b200 as mg
     from paper_conf_icpp_balinsc22_b200 import GCN
+    from paper_conf_icpp_balinsc22_b200.dist import max_over_ranks, share_nccl_id
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -217,11 +218,7 @@ def main():
     Ws = [gen.glorot(w.dims[l], w.dims[l + 1], w.seed_W + l) for l in range(len(w.dims) - 1)]
     t_gen = time.perf_counter() - t0
 
-    nccl_id = None
-    if world > 1:
-        obj = [mg.mggcn_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        nccl_id = obj[0]
+    nccl_id = share_nccl_id(dist, mg.mggcn_nccl_unique_id) if world > 1 else None
     flags = mg.MGGCN_F_PROFILE | (0 if args.no_overlap else mg.MGGCN_F_OVERLAP)
     if args.tf32x1:
         flags |= mg.MGGCN_F_TF32X1
@@ -267,10 +264,7 @@ def main():
     ms = ev0.elapsed_time(ev1) / args.steps
     prof = gm.profile(reset=True)
     work = gm.epoch_work()
-    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
+    ms_max = max_over_ranks(dist, ms, device="cuda")
 
     # ---- end to end: host (pinned) inputs through the C ABI, loss read back every step
     e2e = None
@@ -287,10 +281,7 @@ def main():
             epoch(Xh, yh, want_loss=True)
         gm.synchronize()
         e2e_ms = (time.perf_counter() - tw) * 1e3 / args.steps
-        te = torch.tensor([e2e_ms], dtype=torch.float64, device="cuda")
-        if world > 1:
-            dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        e2e = {"value": float(te.item()), "unit": UNIT,
+        e2e = {"value": max_over_ranks(dist, e2e_ms, device="cuda"), "unit": UNIT,
                "h2d_bytes_per_step": int(Xl.nbytes + yl.nbytes), "d2h_bytes_per_step": 16,
                "how": "wall clock over K epochs; X, y copied from pinned host memory inside mggcn_forward; "
                       "loss read back (synchronising) every epoch"}

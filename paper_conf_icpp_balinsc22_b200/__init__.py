@@ -17,7 +17,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmggcn.so")
+LIB_PATH = os.environ.get("MGGCN_LIB") or os.path.join(_HERE, "libmggcn.so")
 
 MGGCN_OK, MGGCN_EINVAL, MGGCN_ENOMEM, MGGCN_ECUDA, MGGCN_ENCCL, MGGCN_ESTATE, MGGCN_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 MGGCN_F_OVERLAP, MGGCN_F_RELU_LAST, MGGCN_F_TF32X1, MGGCN_F_NO_BCAST, MGGCN_F_PROFILE = 1, 2, 4, 16, 32

@@ -42,8 +42,12 @@ def _nvcc():
     return "nvcc"
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, defines=(), out=None) -> str:
+    """Compile + link.  `defines` (e.g. ["MGGCN_SPMM_HINT=1"]) and `out` build an
+    experiment variant into its own object dir / .so (the product is the default)."""
+    build_dir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
+    so = out or SO
+    os.makedirs(build_dir, exist_ok=True)
     inc, lib = _nccl_dirs()
     nvcc = _nvcc()
     headers = glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) + \
@@ -51,10 +55,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
     hdr_t = max(os.path.getmtime(h) for h in headers)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-I", inc, "-I", os.path.join(ROOT, "include")]
+    common += [f"-D{d}" for d in defines]
     jobs = []
     objs = []
     for s in srcs:
-        o = os.path.join(BUILD, os.path.basename(s) + ".o")
+        o = os.path.join(build_dir, os.path.basename(s) + ".o")
         objs.append(o)
         if force or not os.path.exists(o) or os.path.getmtime(o) < max(os.path.getmtime(s), hdr_t):
             cmd = [nvcc] + ARCH + common + ["-c", s, "-o", o]
@@ -74,15 +79,17 @@ def build(force: bool = False, verbose: bool = False) -> str:
                 sys.stderr.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
             if r.returncode:
                 raise RuntimeError(f"nvcc failed: {cmd[-3]}")
-    if force or jobs or not os.path.exists(SO):
-        cmd = [nvcc] + ARCH + ["-shared", "-o", SO] + objs + ["-L", lib, "-l:libnccl.so.2",
+    if force or jobs or not os.path.exists(so):
+        cmd = [nvcc] + ARCH + ["-shared", "-o", so] + objs + ["-L", lib, "-l:libnccl.so.2",
                                                             "-Xlinker", "-rpath=" + lib]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode:
             sys.stderr.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
             raise RuntimeError("link failed")
-    return SO
+    return so
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, defines=defs, out=outs[0] if outs else None))

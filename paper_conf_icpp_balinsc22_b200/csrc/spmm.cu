@@ -22,7 +22,16 @@ namespace mggcn {
 
 namespace {
 
-constexpr int kWarpsPerBlock = 8;
+#ifndef MGGCN_SPMM_WPB
+#define MGGCN_SPMM_WPB 8
+#endif
+#ifndef MGGCN_SPMM_MINB
+#define MGGCN_SPMM_MINB 1
+#endif
+#ifndef MGGCN_SPMM_U2
+#define MGGCN_SPMM_U2 8
+#endif
+constexpr int kWarpsPerBlock = MGGCN_SPMM_WPB;
 
 __device__ __forceinline__ float4 f4_fma(float a, float4 x, float4 acc) {
     acc.x = fmaf(a, x.x, acc.x);
@@ -44,10 +53,40 @@ __device__ __forceinline__ float4 shfl_xor4(float4 v, int off) {
     return v;
 }
 
+#ifndef MGGCN_SPMM_HINT
+#define MGGCN_SPMM_HINT 0
+#endif
+
+__device__ __forceinline__ uint64_t l2_policy_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint64_t l2_policy_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+
 __device__ __forceinline__ int ld_stream_i32(const int32_t* p) {
     int v;
+#if MGGCN_SPMM_HINT >= 1
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(l2_policy_first()));
+#else
     asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+#endif
     return v;
+}
+
+__device__ __forceinline__ float4 ld_gather(const float4* p) {
+#if MGGCN_SPMM_HINT >= 2
+    float4 v;
+    asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(l2_policy_last()));
+    return v;
+#else
+    return __ldg(p);
+#endif
 }
 
 __device__ __forceinline__ float ld_stream_f32(const float* p) {
@@ -75,10 +114,10 @@ __device__ __forceinline__ float4 epilogue(float4 acc, const float4* out_row, in
 // and serialise them); only the last < U*S entries of a 32-entry chunk take
 // the guarded tail path.
 template <int CH>
-__host__ __device__ constexpr int unroll_for() { return CH == 1 ? 16 : CH == 2 ? 8 : CH == 3 ? 5 : 4; }
+__host__ __device__ constexpr int unroll_for() { return CH == 1 ? 16 : CH == 2 ? MGGCN_SPMM_U2 : CH == 3 ? 5 : 4; }
 
 template <int G, int CH, bool VALS>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, MGGCN_SPMM_MINB)
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const float4* __restrict__ B, int64_t ldb4,
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,
@@ -125,7 +164,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                     a[u] = VALS ? __shfl_sync(0xffffffffu, my_v, k) : 1.f;
                     const float4* brow = B + c * ldb;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = __ldg(brow + qc[ch]);
+                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch]);
                 }
 #pragma unroll
                 for (int u = 0; u < U; ++u)
@@ -139,7 +178,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 if (k < cnt) {
                     const float4* brow = B + c * ldb;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(v, __ldg(brow + qc[ch]), acc[ch]);
+                    for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(v, ld_gather(brow + qc[ch]), acc[ch]);
                 }
             }
         }

@@ -1,7 +1,9 @@
 """Builds libmggcn.so (C ABI of include/mggcn.h) in-tree with nvcc for sm_100a.
 
-    python -m paper_conf_icpp_balinsc22_b200.build [--force]
+    python build_mggcn.py [--force] [-v] [-DNAME=VALUE ... --out=path.so]
 
+Kept outside the package so that building never imports (and loads) a stale
+library.
 Objects are rebuilt when their source or any header is newer.  NCCL comes
 from the torch venv (nvidia/nccl), linked with an rpath so the same
 libnccl.so.2 that torch loads is used.
@@ -14,8 +16,8 @@ import os
 import subprocess
 import sys
 
-PKG = os.path.dirname(os.path.abspath(__file__))
-ROOT = os.path.dirname(PKG)
+ROOT = os.path.dirname(os.path.abspath(__file__))
+PKG = os.path.join(ROOT, "paper_conf_icpp_balinsc22_b200")
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(PKG, "_build")
 SO = os.path.join(PKG, "libmggcn.so")

@@ -59,8 +59,12 @@ enum {
                                  3xTF32 (hi/lo split, ~fp32 accuracy)                  */
     MGGCN_F_NO_BCAST = 16u,   /* TIMING ONLY: skip broadcasts; results invalid         */
     MGGCN_F_PROFILE = 32u,    /* record per-op CUDA events (see mggcn_get_profile)     */
-    MGGCN_F_NO_COALESCE = 64u /* keep duplicate entries as separate gathers (default:
+    MGGCN_F_NO_COALESCE = 64u,/* keep duplicate entries as separate gathers (default:
                                  merged on the device copy, value = multiplicity)       */
+    MGGCN_F_CACHE_L0 = 128u   /* X is constant across epochs (full-batch training): layer 0
+                                 runs SpMM-first and T0 = Â'^T X is computed on the first
+                                 forward and reused (exact by associativity,
+                                 Eq. 5-6 and Eq. 10).  mggcn_reset_cache() after X changes. */
 };
 
 typedef struct mggcn_graph_s* mggcn_graph; /* host CSR of A + in-degrees                     */
@@ -148,6 +152,8 @@ int mggcn_get_weights(mggcn_model m, int32_t layer, float* W);
 int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float* loss,
                   float* logits_local);
 int mggcn_backward(mggcn_model m);
+/* Drops the MGGCN_F_CACHE_L0 aggregate; the next forward recomputes it from X. */
+int mggcn_reset_cache(mggcn_model m);
 int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps);
 
 /* Synchronising getters / checkpoint. */

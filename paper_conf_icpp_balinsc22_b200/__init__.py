@@ -1,7 +1,7 @@
 """B200-native MG-GCN hot path (Balın, Sancak, Çatalyürek, ICPP '22).
 
 Thin ctypes binding of the C ABI in include/mggcn.h (libmggcn.so, built
-in-tree for sm_100a by ``paper_conf_icpp_balinsc22_b200.build``).  Functions
+in-tree for sm_100a by ``build_mggcn.py``).  Functions
 keep the C names; this module only marshals arguments.  Every step of the
 path runs in the library's kernels; there is no CPU fallback: if the shared
 library is missing, importing the binding raises.
@@ -22,6 +22,7 @@ LIB_PATH = os.environ.get("MGGCN_LIB") or os.path.join(_HERE, "libmggcn.so")
 MGGCN_OK, MGGCN_EINVAL, MGGCN_ENOMEM, MGGCN_ECUDA, MGGCN_ENCCL, MGGCN_ESTATE, MGGCN_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 MGGCN_F_OVERLAP, MGGCN_F_RELU_LAST, MGGCN_F_TF32X1, MGGCN_F_NO_BCAST, MGGCN_F_PROFILE = 1, 2, 4, 16, 32
 MGGCN_F_NO_COALESCE = 64
+MGGCN_F_CACHE_L0 = 128
 PROFILE_CLASSES = ("spmm", "gemm", "loss", "adam", "bcast", "allreduce", "other")
 
 EXPORTS = (
@@ -30,7 +31,7 @@ EXPORTS = (
     "mggcn_model_create", "mggcn_nccl_unique_id", "mggcn_set_weights", "mggcn_get_weights", "mggcn_forward",
     "mggcn_backward", "mggcn_step", "mggcn_get_loss", "mggcn_get_grad", "mggcn_get_adam", "mggcn_set_adam",
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
-    "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count",
+    "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
 )
 
 
@@ -42,7 +43,7 @@ class MggcnError(RuntimeError):
 
 def _load():
     if not os.path.exists(LIB_PATH):
-        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_icpp_balinsc22_b200.build` "
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python build_mggcn.py` "
                           "(the CUDA library is the only implementation; there is no fallback)")
     try:  # make sure the NCCL that torch bundles is the one resolved
         import torch  # noqa: F401
@@ -80,6 +81,7 @@ def _load():
         "mggcn_debug_spmm": ([P, i32, P, i64, i32, P, i64], ctypes.c_int),
         "mggcn_debug_gemm": ([i32, i64, i64, i64, P, i64, P, i64, P, i64, u32, up], ctypes.c_int),
         "mggcn_kernel_launch_count": ([], ctypes.c_int64),
+        "mggcn_reset_cache": ([P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -220,6 +222,10 @@ def mggcn_forward(m, X, ldx, y, want_loss=True, logits=None):
 
 def mggcn_backward(m):
     _check(_lib.mggcn_backward(m))
+
+
+def mggcn_reset_cache(m):
+    _check(_lib.mggcn_reset_cache(m))
 
 
 def mggcn_step(m, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8):

@@ -165,6 +165,7 @@ struct mggcn_model_s {
     double w_spmm_bytes = 0, w_gather_bytes = 0, w_gemm_flops = 0, w_bcast_bytes = 0;
     // X staging plan bookkeeping
     int layer_ids[64];
+    bool t0_valid = false;          // MGGCN_F_CACHE_L0: T0 = Â'^T X computed
 };
 
 namespace {
@@ -620,6 +621,7 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
     for (int l = 0; l <= L; ++l) m->ld[l] = ld_of(m->d[l]);
     m->order.resize(L);
     for (int l = 0; l < L; ++l) m->order[l] = m->d[l] < m->d[l + 1] ? S_ORDER : G_ORDER;   // §4.4, reading C10
+    if (flags & MGGCN_F_CACHE_L0) m->order[0] = S_ORDER;   // T0 = Â'^T X is reused across epochs
     m->woff.resize(L);
     m->wtotal = 0;
     for (int l = 0; l < L; ++l) {
@@ -678,7 +680,7 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
     };
     for (int l = 0; l < L; ++l) {
         const int64_t w = m->order[l] == G_ORDER ? m->d[l + 1] : m->d[l];
-        spmm_work(0, w);
+        if (!(l == 0 && (flags & MGGCN_F_CACHE_L0))) spmm_work(0, w);   // steady state: T0 cached
         const double gf = 2.0 * (double)m->n_local * (double)m->d[l] * (double)m->d[l + 1];
         m->w_gemm_flops += gf;                       // forward
         m->w_gemm_flops += gf;                       // W_G
@@ -937,10 +939,13 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
     const bool host_x = cudaPointerGetAttributes(&pa, X) != cudaSuccess || pa.type == cudaMemoryTypeHost ||
                         pa.type == cudaMemoryTypeUnregistered;
     cudaGetLastError();   // clear a possible error from the attribute query
+    const bool use_cache = (m->flags & MGGCN_F_CACHE_L0) && m->t0_valid;
     for (auto& r : m->ranks) {
         if (r.rows == 0) continue;
         ProfScope ps(m, PC_OTHER, m->cs);
-        if (host_x && ldx != m->ld[0]) {
+        if (use_cache) {
+            // X is not read again: layer 0 starts from the cached T0
+        } else if (host_x && ldx != m->ld[0]) {
             const int64_t stage_floats = r.rows * std::max<int64_t>(m->hw_ld, 4);
             const int64_t chunk = std::max<int64_t>(1, stage_floats / ldx);
             for (int64_t r0 = 0; r0 < r.rows; r0 += chunk) {
@@ -973,7 +978,8 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
         } else {
             SpmmJob job{0, m->ld[0], m->pattern, false, src_X,
                         [](mggcn_model_s*, Rank& r, const void*) { return r.T0; }, nullptr};
-            RC(staged_spmm(m, job));                                                     // T = Â'^T X (§4.4)
+            if (!use_cache) RC(staged_spmm(m, job));                                     // T = Â'^T X (§4.4)
+            if (m->flags & MGGCN_F_CACHE_L0) m->t0_valid = true;
             for (auto& r : m->ranks)
                 if (r.has_fwd[l]) {
                     ProfScope ps(m, PC_GEMM, m->cs);
@@ -1028,6 +1034,12 @@ extern "C" int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, c
     int rc = forward_impl(m, X_local, ldx, y_local, loss, logits_local);
     if (rc == MGGCN_OK) m->state = ST_FWD;
     return poison(m, rc);
+}
+
+extern "C" int mggcn_reset_cache(mggcn_model m) {
+    MODEL_GUARD(m);
+    m->t0_valid = false;
+    return MGGCN_OK;
 }
 
 extern "C" int mggcn_get_loss(mggcn_model m, float* loss) {

@@ -16,8 +16,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 @pytest.fixture(scope="module")
 def mg():
-    from paper_conf_icpp_balinsc22_b200 import build
-    build.build()
+    import build_mggcn
+    build_mggcn.build()
     import paper_conf_icpp_balinsc22_b200 as mg
     return mg
 

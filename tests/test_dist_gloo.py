@@ -52,8 +52,8 @@ def _free_port():
 
 def test_two_rank_host_path(tmp_path):
     import pickle
-    from paper_conf_icpp_balinsc22_b200 import build
-    build.build()
+    import build_mggcn
+    build_mggcn.build()
     import gen
     import oracle
     script = tmp_path / "worker.py"

@@ -227,7 +227,8 @@ struct ProfScope {
 };
 
 // --------------------------------------------------------------- planning
-int64_t ld_of(int64_t d) { return round_up(d, 4); }
+// 32-B (sector) aligned rows: narrow gathered rows (e.g. 41 -> 48 floats) stay sector aligned
+int64_t ld_of(int64_t d) { return round_up(d, 8); }
 
 int check_dims(int L, const int32_t* dims) {
     if (L < 1 || L > 64 || !dims) {

@@ -89,11 +89,13 @@ cudaError_t launch_splitk_reduce(const float* partial, int k_chunks, int64_t M, 
 // Z (n x C, ld) holds logits on entry and dLoss/dZ on exit (times
 // rowscale[row] if non-null; times [Z > 0] if relu_last).  Per-block fp64
 // partial loss sums into block_partial[grid].
-constexpr int kCeBlocks = 592;
+constexpr int kCeBlocks = 2368;          // 16 per SM; fixed so partial sums are reduced in a fixed order
+constexpr int kCountBlocks = 296;
 cudaError_t launch_softmax_ce(float* Z, int64_t n, int C, int64_t ld, const int32_t* y, const int64_t* ntrain,
                               const float* rowscale, int relu_last, double* block_partial, cudaStream_t s);
 cudaError_t launch_sum_partials(const double* partial, int count, double* out, cudaStream_t s);
-cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* out, cudaStream_t s);
+// |T| = #{y >= 0}: per-block counts into scratch[kCountBlocks], then one ordered sum into *out.
+cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* scratch, int64_t* out, cudaStream_t s);
 cudaError_t launch_adam(float* W, const float* g, float* m, float* v, int64_t count, double lr, double b1,
                         double b2, double eps, int64_t t, cudaStream_t s);
 // out[i] = sum_r in[r][i] in r order (loopback "all-reduce").

@@ -87,14 +87,15 @@ __global__ void sum_partials_kernel(const double* __restrict__ p, int count, dou
 __global__ void count_labelled_kernel(const int32_t* __restrict__ y, int64_t n, int64_t* __restrict__ out) {
     __shared__ long long ws[32];
     long long c = 0;
-    for (int64_t i = threadIdx.x; i < n; i += blockDim.x) c += y[i] >= 0 ? 1 : 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        c += y[i] >= 0 ? 1 : 0;
     for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
     if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
     __syncthreads();
     if (threadIdx.x == 0) {
         long long t = 0;
         for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += ws[w];
-        *out = t;
+        out[blockIdx.x] = t;
     }
 }
 
@@ -171,8 +172,10 @@ cudaError_t launch_sum_partials(const double* partial, int count, double* out, c
     return cudaGetLastError();
 }
 
-cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* out, cudaStream_t s) {
-    count_labelled_kernel<<<1, 1024, 0, s>>>(y, n, out);
+cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* scratch, int64_t* out, cudaStream_t s) {
+    count_labelled_kernel<<<kCountBlocks, 512, 0, s>>>(y, n, scratch);
+    count_launches(1);
+    sum_i64_kernel<<<1, 1, 0, s>>>(scratch, kCountBlocks, out);
     count_launches(1);
     return cudaGetLastError();
 }

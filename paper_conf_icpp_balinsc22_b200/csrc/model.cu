@@ -989,7 +989,8 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
         }
     }
     // ---- loss: |T|, logits out, fused CE fwd+bwd in place (Eq. 19)
-    for (auto& r : m->ranks) CK(launch_count_labelled(r.y, r.rows, r.ntrain_local, m->cs));
+    for (auto& r : m->ranks)
+        CK(launch_count_labelled(r.y, r.rows, reinterpret_cast<int64_t*>(r.ce_partial), r.ntrain_local, m->cs));
     RC(reduce_all(m, true));
     if (logits) {
         for (auto& r : m->ranks)

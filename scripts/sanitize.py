@@ -1,0 +1,31 @@
+"""Small end-to-end run for compute-sanitizer: loopback P=2 Cora-shaped epoch,
+an SpMM-first config, and the three GEMM ops (ragged shapes)."""
+import os, sys
+import numpy as np, torch
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import gen
+import paper_conf_icpp_balinsc22_b200 as mg
+from paper_conf_icpp_balinsc22_b200 import GCN
+for dims, P, n, m in (((1433, 16, 7), 2, 2708, 10556), ((8, 32, 24, 5), 1, 3001, 60000)):
+    rp, col = gen.rmat_csr(n, m, 5)
+    X = gen.features(n, dims[0], 6); y = gen.labels(n, dims[-1], 7, 100)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 8 + l) for l in range(len(dims) - 1)]
+    gm = GCN(n, rp, col, None, dims, P=P, perm_seed=9, loopback=P > 1, flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE)
+    gm.set_weights(Ws)
+    for host in (False, True):
+        Xl, yl = gm.permute_rows(X), gm.permute_rows(y)
+        Xin = Xl if host else torch.from_numpy(Xl).cuda()
+        yin = yl if host else torch.from_numpy(yl).cuda()
+        loss = gm.forward(Xin, yin, logits=torch.empty((n, dims[-1]), device="cuda"))
+        gm.backward(); gm.step()
+    print("epoch ok", dims, P, loss, flush=True)
+    gm.close()
+for op, (M, N, K) in ((0, (300, 41, 602)), (1, (257, 256, 41)), (2, (602, 47, 1000))):
+    rng = np.random.default_rng(op)
+    if op == 0: A, B = rng.standard_normal((M, 608)), rng.standard_normal((K, 48))
+    elif op == 1: A, B = rng.standard_normal((M, 48)), rng.standard_normal((N, 48))
+    else: A, B = rng.standard_normal((K, 608)), rng.standard_normal((K, 48))
+    C = torch.zeros((M, (N + 7) // 8 * 8), device="cuda")
+    mg.mggcn_debug_gemm(op, M, N, K, torch.tensor(A, dtype=torch.float32).cuda(), A.shape[1],
+                        torch.tensor(B, dtype=torch.float32).cuda(), B.shape[1], C, C.shape[1])
+    print("gemm ok", op, flush=True)

@@ -171,15 +171,24 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
 #pragma unroll
                     for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(a[u], x[u][ch], acc[ch]);
             }
-            for (; k0 < cnt; k0 += S) {   // tail: < U*S entries
-                const int k = k0 + slot;
-                const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, my_c, k & 31);
-                const float v = VALS ? __shfl_sync(0xffffffffu, my_v, k & 31) : 1.f;
-                if (k < cnt) {
+            if (k0 < cnt) {   // tail (< U*S entries left): one more unpredicated group; padding lanes
+                float4 x[U][CH];  // re-read the chunk's last entry (a row of this very sum) with weight 0
+                float a[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int k = k0 + u * S + slot;
+                    const int kc = k < cnt ? k : cnt - 1;
+                    const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, my_c, kc);
+                    const float v = VALS ? __shfl_sync(0xffffffffu, my_v, kc) : 1.f;
+                    a[u] = k < cnt ? v : 0.f;
                     const float4* brow = B + c * ldb;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(v, ld_gather(brow + qc[ch]), acc[ch]);
+                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch]);
                 }
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+#pragma unroll
+                    for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(a[u], x[u][ch], acc[ch]);
             }
         }
         // combine the S slots (fixed xor tree => deterministic)

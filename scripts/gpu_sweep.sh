@@ -1,4 +1,3 @@
-for L in "" a b c d e f; do
-  LIB=""; [ -n "$L" ] && LIB=scratch_libs/libmggcn_$L.so
-  echo "VARIANT=$L"; MGGCN_LIB=$LIB timeout -s KILL 300 python scripts/spmm_sweep.py reddit 256 44 2>&1 | grep "dir 0"
-done
+timeout -s KILL 600 python -m pytest tests/test_gpu_kernels.py -q --timeout 120 -k spmm -x 2>&1 | tail -1
+timeout -s KILL 300 python scripts/spmm_sweep.py reddit 256 48 2>&1 | grep "dir 0"
+timeout -s KILL 300 python scripts/spmm_sweep.py products 256 104 48 2>&1 | grep "dir 0"

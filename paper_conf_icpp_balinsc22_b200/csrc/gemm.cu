@@ -371,37 +371,64 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 // ===================================================================== rows
 // Row GEMM (op 0 / op 1): C[M x N] = A[M x K] · B^T with B given PRE-SPLIT as
 // tf32 hi / lo copies in K-major [N x K] layout (the weights; split once per
-// step by launch_split_weights).  Per stage: TMA writes raw A (SW128) and
-// B_hi / B_lo straight into the MMA operand buffers; the 4 transform warps
-// split A IN PLACE (A -> A_hi, A_lo); BN = N up to 256 so A is staged once.
-constexpr int kRowStage = 96 * 1024;        // A 16K | A_lo 16K | B_hi 32K | B_lo 32K
-constexpr int kRowBars = 2 * kRowStage;     // 6 mbarriers + TMEM slot
+// step by launch_split_weights).  K blocks of 16 (SWIZZLE_64B operands), 3
+// stages: TMA writes raw A and B_hi / B_lo straight into the operand buffers;
+// the 4 transform warps split A IN PLACE; BN = N up to 256 so A is staged
+// once.  Epilogue: 32-column chunks go TMEM -> registers -> swizzled smem ->
+// TMA bulk store (full 128-B lines); the old C values for the ReLU' mask of
+// Eq. 8 / Eq. 21 come in by TMA into the same layout.
+constexpr int kRowBK = 16;
+constexpr int kRowNS = 3;
+constexpr int kRowStage = 48 * 1024;            // A 8K | A_lo 8K | B_hi 16K | B_lo 16K
+constexpr int kRowOut = kRowNS * kRowStage;     // 2 x 16 KB output chunks [128 rows][32 cols] SW128
+constexpr int kRowOld = kRowOut + 2 * 16384;    // 2 x 16 KB old-C chunks (mask)
+constexpr int kRowBars = kRowOld + 2 * 16384;
 constexpr int kRowSmem = kRowBars + 256 + 1024;
+
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* tm, int c0, int c1, const void* src) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"((uint64_t)tm),
+                 "r"(c0), "r"(c1), "r"(smem_u32(src))
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+// byte offset of (row r, 16-B chunk q) in a [128][32 fp32] SWIZZLE_128B tile
+__device__ __forceinline__ int sw128_off(int r, int q) { return r * 128 + ((q ^ (r & 7)) << 4); }
 
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBh,
-                 const __grid_constant__ CUtensorMap tmBl, const KParams p) {
+                 const __grid_constant__ CUtensorMap tmBl, const __grid_constant__ CUtensorMap tmC, const KParams p) {
     extern __shared__ uint8_t smem_dyn[];
     uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);   // keeps the shared state space
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kRowBars);
-    uint64_t* full = bars + 0;
-    uint64_t* xf = bars + 2;
-    uint64_t* empty = bars + 4;
-    uint64_t* tmem_full = bars + 6;
-    uint64_t* tmem_empty = bars + 8;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 10);
+    uint64_t* full = bars + 0;           // [3]
+    uint64_t* xf = bars + 3;             // [3]
+    uint64_t* empty = bars + 6;          // [3]
+    uint64_t* tmem_full = bars + 9;      // [2]
+    uint64_t* tmem_empty = bars + 11;    // [2]
+    uint64_t* old_full = bars + 13;      // [2]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 15);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
+    const bool mask = (p.flags & GEMM_MASK) != 0;
     const int BN = p.BN;
     const uint32_t tcols = BN > 128 ? 512u : 256u;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < 2; ++s) {
+        for (int s = 0; s < kRowNS; ++s) {
             mbar_init(full + s, 1);
             mbar_init(xf + s, 128);
             mbar_init(empty + s, 1);
+        }
+        for (int s = 0; s < 2; ++s) {
             mbar_init(tmem_full + s, 1);
             mbar_init(tmem_empty + s, 128);
+            mbar_init(old_full + s, 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -415,38 +442,37 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
     const int total_tiles = p.m_tiles * p.n_tiles;
-    const int nkb = (p.K + BK - 1) / BK;
+    const int nkb = (p.K + kRowBK - 1) / kRowBK;
 
     if (warp == kTmaWarp) {
         if (lane == 0) {
-            const uint32_t bytes = (uint32_t)(BM * BK * 4 + BN * BK * 4 * (x1 ? 1 : 2));
-            uint32_t it = 0;
+            const uint32_t bytes = (uint32_t)(BM * kRowBK * 4 + BN * kRowBK * 4 * (x1 ? 1 : 2));
+            int s = 0;
+            uint32_t ph = 0;
             for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
                 const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
-                for (int kb = 0; kb < nkb; ++kb, ++it) {
-                    const int s = it & 1;
-                    const uint32_t ph = (it >> 1) & 1;
+                for (int kb = 0; kb < nkb; ++kb) {
                     uint8_t* st = smem + s * kRowStage;
                     mbar_wait(empty + s, ph ^ 1);
                     mbar_expect_tx(full + s, bytes);
-                    tma_load_2d(st, &tmA, kb * BK, mt * BM, full + s);
-                    tma_load_2d(st + 32768, &tmBh, kb * BK, nt * BN, full + s);
-                    if (!x1) tma_load_2d(st + 65536, &tmBl, kb * BK, nt * BN, full + s);
+                    tma_load_2d(st, &tmA, kb * kRowBK, mt * BM, full + s);
+                    tma_load_2d(st + 16384, &tmBh, kb * kRowBK, nt * BN, full + s);
+                    if (!x1) tma_load_2d(st + 32768, &tmBl, kb * kRowBK, nt * BN, full + s);
+                    if (++s == kRowNS) { s = 0; ph ^= 1; }
                 }
             }
         }
     } else if (warp >= kXfWarp0 && warp < kXfWarp0 + 4) {
         const int t = threadIdx.x - kXfWarp0 * 32;
-        uint32_t it = 0;
+        int s = 0;
+        uint32_t ph = 0;
         for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
-            for (int kb = 0; kb < nkb; ++kb, ++it) {
-                const int s = it & 1;
-                const uint32_t ph = (it >> 1) & 1;
+            for (int kb = 0; kb < nkb; ++kb) {
                 float4* a = reinterpret_cast<float4*>(smem + s * kRowStage);
-                float4* al = reinterpret_cast<float4*>(smem + s * kRowStage + 16384);
+                float4* al = reinterpret_cast<float4*>(smem + s * kRowStage + 8192);
                 mbar_wait(full + s, ph);
 #pragma unroll
-                for (int c = t; c < BM * 8; c += 128) {
+                for (int c = t; c < BM * 4; c += 128) {
                     float4 v = a[c], h, l;
                     split4(v, h, l, x1);
                     a[c] = h;
@@ -454,29 +480,29 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 }
                 fence_proxy_async();
                 mbar_arrive(xf + s);
+                if (++s == kRowNS) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == kMmaWarp) {
         if (lane == 0) {
             const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
                                    ((uint32_t)(BM >> 4) << 24);
-            uint32_t it = 0, tc = 0;
+            int s = 0;
+            uint32_t ph = 0, tc = 0;
             for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
                 const int acc = tc & 1;
                 const uint32_t aph = (tc >> 1) & 1;
                 mbar_wait(tmem_empty + acc, aph ^ 1);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
-                for (int kb = 0; kb < nkb; ++kb, ++it) {
-                    const int s = it & 1;
-                    const uint32_t ph = (it >> 1) & 1;
+                for (int kb = 0; kb < nkb; ++kb) {
                     mbar_wait(xf + s, ph);
                     tc_fence_after();
                     const uint32_t base = smem_u32(smem + s * kRowStage);
-                    const uint64_t ah = sw128_desc(base), al = sw128_desc(base + 16384);
-                    const uint64_t bh = sw128_desc(base + 32768), bl = sw128_desc(base + 65536);
+                    const uint64_t ah = sw64_desc(base), al = sw64_desc(base + 8192);
+                    const uint64_t bh = sw64_desc(base + 16384), bl = sw64_desc(base + 32768);
 #pragma unroll
-                    for (int kk = 0; kk < BK / 8; ++kk) {
+                    for (int kk = 0; kk < kRowBK / 8; ++kk) {
                         const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);
                         if (!x1) {   // small products first
                             mma_tf32(d_tmem, al + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
@@ -487,31 +513,75 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                         }
                     }
                     mma_commit(empty + s);
+                    if (++s == kRowNS) { s = 0; ph ^= 1; }
                 }
                 mma_commit(tmem_full + acc);
             }
         }
     } else {
-        uint32_t tc = 0;
+        // ---- epilogue warps 0-3: thread = accumulator row (TMEM lane quadrant = warp)
+        const int r = warp * 32 + lane;
+        const bool leader = threadIdx.x == 0;
+        uint32_t tc = 0, chunk_ctr = 0;
+        const int nch = (BN + 31) / 32;
         for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
             const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
             const int acc = tc & 1;
             const uint32_t aph = (tc >> 1) & 1;
+            const int row = mt * BM + r;
+            const float sc = ((p.flags & GEMM_SCALE) && row < p.M) ? __ldg(p.rowscale + row) : 1.f;
+            const uint32_t c_base = chunk_ctr;
+            if (mask && leader)   // prefetch the old values of the first two chunks
+                for (int c = 0; c < 2 && c < nch; ++c) {
+                    const int b = (c_base + c) & 1;
+                    mbar_expect_tx(old_full + b, 16384);
+                    tma_load_2d(smem + kRowOld + b * 16384, &tmC, nt * BN + 32 * c, mt * BM, old_full + b);
+                }
             mbar_wait(tmem_full + acc, aph);
             tc_fence_after();
-            const int row = mt * BM + warp * 32 + lane;
-            const int n0 = nt * BN;
-            const float sc = ((p.flags & GEMM_SCALE) && row < p.M) ? __ldg(p.rowscale + row) : 1.f;
-            for (int c0 = 0; c0 < BN; c0 += 16) {
-                float v[16];
-                tmem_ld16(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)(acc * BN + c0), v);
-                const int nb = n0 + c0;
-                if (row >= p.M || nb >= p.N) continue;
-                store_epilogue(p, row, nb, v, sc);
+            for (int c = 0; c < nch; ++c, ++chunk_ctr) {
+                const int b = chunk_ctr & 1;
+                uint8_t* ob = smem + kRowOut + b * 16384;
+                float v[32];
+                const uint32_t ta = tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)(acc * BN + 32 * c);
+                tmem_ld16(ta, v);
+                tmem_ld16(ta + 16, v + 16);
+                if (leader) bulk_wait_read<1>();   // the store that last used `ob` has read it
+                if (mask) mbar_wait(old_full + b, (chunk_ctr >> 1) & 1);
+                epi_bar();
+                const uint8_t* oldb = smem + kRowOld + b * 16384;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                    float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+                    if (mask) {
+                        const float4 old = *reinterpret_cast<const float4*>(oldb + sw128_off(r, q));
+                        o.x = old.x > 0.f ? o.x : 0.f;
+                        o.y = old.y > 0.f ? o.y : 0.f;
+                        o.z = old.z > 0.f ? o.z : 0.f;
+                        o.w = old.w > 0.f ? o.w : 0.f;
+                    }
+                    o.x *= sc; o.y *= sc; o.z *= sc; o.w *= sc;
+                    if (p.flags & GEMM_RELU) {
+                        o.x = fmaxf(o.x, 0.f); o.y = fmaxf(o.y, 0.f);
+                        o.z = fmaxf(o.z, 0.f); o.w = fmaxf(o.w, 0.f);
+                    }
+                    *reinterpret_cast<float4*>(ob + sw128_off(r, q)) = o;
+                }
+                fence_proxy_async();
+                epi_bar();
+                if (leader) {
+                    tma_store_2d(&tmC, nt * BN + 32 * c, mt * BM, ob);
+                    bulk_commit();
+                    if (mask && c + 2 < nch) {   // old values of chunk c+2 into the buffer just consumed
+                        mbar_expect_tx(old_full + b, 16384);
+                        tma_load_2d(smem + kRowOld + b * 16384, &tmC, nt * BN + 32 * (c + 2), mt * BM, old_full + b);
+                    }
+                }
             }
             tc_fence_before();
             mbar_arrive(tmem_empty + acc);
         }
+        if (leader) bulk_wait_read<0>();
     }
     __syncthreads();
     if (warp == kMmaWarp) {
@@ -576,6 +646,24 @@ int encode2d(CUtensorMap* m, const float* base, int64_t dim0, int64_t dim1, int6
     return r == CUDA_SUCCESS ? 0 : -2;
 }
 
+// as encode2d with an explicit swizzle span (0, 64 or 128 bytes)
+int encode2d_sw(CUtensorMap* m, const float* base, int64_t dim0, int64_t dim1, int64_t ld, int box0, int box1,
+                int swizzle) {
+    EncodeTiledFn fn = get_encode();
+    if (!fn) return -1;
+    cuuint64_t dims[2] = {(cuuint64_t)dim0, (cuuint64_t)dim1};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+    cuuint32_t box[2] = {(cuuint32_t)box0, (cuuint32_t)box1};
+    cuuint32_t es[2] = {1, 1};
+    const CUtensorMapSwizzle sw = swizzle == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                  : swizzle == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                  : CU_TENSOR_MAP_SWIZZLE_NONE;
+    CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, es,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : -2;
+}
+
 int num_sms() {
     static int n = 0;
     if (n == 0) {
@@ -606,7 +694,7 @@ cudaError_t launch_rows(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    gemm_rows_kernel<<<g.grid, kThreads, kRowSmem, s>>>(g.tmA, g.tmB, g.tmB2, kp);
+    gemm_rows_kernel<<<g.grid, kThreads, kRowSmem, s>>>(g.tmA, g.tmB, g.tmB2, g.tmC, kp);
     count_launches(1);
     return cudaGetLastError();
 }
@@ -623,16 +711,20 @@ int gemm_plan_rows(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A,
     g.op = 0;
     g.M = M; g.N = N; g.K = K;
     g.n_tiles = (int)((N + 255) / 256);
-    g.BN = (int)(((N + g.n_tiles - 1) / g.n_tiles + 15) / 16 * 16);
+    // one N tile: multiple of 16 (MMA N); several: multiple of 32 so the 32-column
+    // epilogue chunks never spill into the neighbouring tile
+    g.BN = g.n_tiles == 1 ? (int)((N + 15) / 16 * 16) : (int)(((N + g.n_tiles - 1) / g.n_tiles + 31) / 32 * 32);
     g.m_tiles = (int)((M + BM - 1) / BM);
     g.C = C;
     g.ldc = ldc;
     g.flags = flags;
     g.k_chunks = 1;
     g.k_chunk_len = (K + BK - 1) / BK * BK;
-    int rc = encode2d(&g.tmA, A, K, M, lda, BK, BM, true);
-    if (!rc) rc = encode2d(&g.tmB, Bhi, K, N, ldb, BK, g.BN, true);
-    if (!rc) rc = encode2d(&g.tmB2, Blo, K, N, ldb, BK, g.BN, true);
+    if ((ldc & 3) || (reinterpret_cast<uintptr_t>(C) & 15)) return -1;
+    int rc = encode2d_sw(&g.tmA, A, K, M, lda, 16, BM, 64);
+    if (!rc) rc = encode2d_sw(&g.tmB, Bhi, K, N, ldb, 16, g.BN, 64);
+    if (!rc) rc = encode2d_sw(&g.tmB2, Blo, K, N, ldb, 16, g.BN, 64);
+    if (!rc) rc = encode2d_sw(&g.tmC, C, N, M, ldc, 32, BM, 128);   // epilogue store / old-value load
     if (rc) return rc;
     const int total = g.m_tiles * g.n_tiles;
     g.grid = total < num_sms() ? total : num_sms();

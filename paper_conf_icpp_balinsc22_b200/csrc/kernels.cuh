@@ -56,7 +56,7 @@ struct GemmPlan {
     int64_t M = 0, N = 0, K = 0;
     int BN = 0, m_tiles = 0, n_tiles = 0, k_chunks = 1;
     int64_t k_chunk_len = 0;
-    CUtensorMap tmA, tmB, tmB2;
+    CUtensorMap tmA, tmB, tmB2, tmC;
     float* C = nullptr;
     int64_t ldc = 0;
     float* partial = nullptr;   // op 2: [k_chunks][M][N]

@@ -45,7 +45,7 @@ def _gemm(mg, op, A, B, M, N, K, flags=0):
 
 
 GEMM_SHAPES = [(128, 16, 32), (1000, 41, 602), (300, 256, 100), (517, 7, 1433), (2048, 112, 8),
-               (777, 172, 256), (129, 128, 33), (64, 256, 256)]
+               (777, 172, 256), (129, 128, 33), (64, 256, 256), (300, 602, 48), (129, 300, 64), (65, 513, 17)]
 
 
 @pytest.mark.parametrize("op", [0, 1, 2])

@@ -192,14 +192,16 @@ __device__ __forceinline__ void store_epilogue(const KParams& p, int row, int nb
 // of block kb; warp 9 issues hi.hi + hi.lo + lo.hi per 8-deep k step; warps
 // 0-3 drain the TMEM accumulator into the split-K partial buffer.
 constexpr int kWgBK = 16;
-constexpr int kWgNS = 3;                         // pipeline stages
+constexpr int kWgNR = 5;                         // raw (TMA) stages
+constexpr int kWgNS = 2;                         // split (MMA operand) stages
 constexpr int kWgRawA = 0;                       // 3 x  8 KB  raw A [16 k][128 m]
-constexpr int kWgRawB = kWgNS * 8192;            // 3 x 16 KB  raw B [16 k][<=256 n]
-constexpr int kWgSplit = kWgRawB + kWgNS * 16384;  // 3 x 48 KB: A_hi 8K | A_lo 8K | B_hi 16K | B_lo 16K
+constexpr int kWgRawB = kWgNR * 8192;            // 5 x 16 KB  raw B [16 k][<=256 n]
+constexpr int kWgSplit = kWgRawB + kWgNR * 16384;  // 2 x 48 KB: A_hi 8K | A_lo 8K | B_hi 16K | B_lo 16K
 constexpr int kWgSplitStage = 49152;
 constexpr int kWgBars = kWgSplit + kWgNS * kWgSplitStage;
 constexpr int kWgSmem = kWgBars + 256 + 1024;
-constexpr int kWgXfThreads = 256;
+constexpr int kWgXfThreads = 512;                // warps 0-15 transform (0-3 also epilogue)
+constexpr int kWgTmaWarp = 16, kWgMmaWarp = 17, kWgThreads = 576;
 
 // K-major SWIZZLE_64B descriptor: rows of 64 B (16 tf32), 8-row atoms 512 B apart.
 __device__ __forceinline__ uint64_t sw64_desc(uint32_t saddr) {
@@ -209,49 +211,64 @@ __device__ __forceinline__ uint64_t sw64_desc(uint32_t saddr) {
 
 // raw[kk][r] (pitch `rows`, kk < 16) -> K-major SW64: element (r, k) at
 // r*64 + (((k>>2) ^ ((r>>1)&3)) << 4) + (k&3)*4.  Thread t owns row
-// r = t % rows and the k-quads kq = g, g+G, ... (g = t / rows, G = NT / rows):
-// all its shared loads are issued before the first split (ILP).
-template <int NT>
-__device__ __forceinline__ void transpose_split16(const float* __restrict__ raw, uint8_t* hi, uint8_t* lo, int rows,
-                                                  int t, bool x1) {
+// r = t % rows and the k-quads kq = g, g+G, ... (g = t / rows, G = NT / rows);
+// the offsets are computed once per kernel, and all shared loads of a k block
+// are issued before the first split (ILP).
+struct XfPlan {
+    bool ok[4];       // k-quad j is owned by this thread
+    int ld[4];        // float index of raw[(4 kq) * rows + r]
+    int st[4];        // byte offset in the SW64 operand tile
+    int rows;
+};
+
+__device__ __forceinline__ XfPlan make_xf_plan(int rows, int t, int NT) {
+    XfPlan pl;
+    pl.rows = rows;
     const int G = NT / rows;
     const int g = t / rows, r = t - g * rows;
-    if (g >= G) return;
-    float4 a[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
         const int kq = g + j * G;
-        if (kq < 4) {
-            a[j].x = raw[(4 * kq + 0) * rows + r];
-            a[j].y = raw[(4 * kq + 1) * rows + r];
-            a[j].z = raw[(4 * kq + 2) * rows + r];
-            a[j].w = raw[(4 * kq + 3) * rows + r];
-        }
+        pl.ok[j] = g < G && kq < 4;
+        pl.ld[j] = 4 * kq * rows + r;
+        pl.st[j] = r * 64 + ((kq ^ ((r >> 1) & 3)) << 4);
     }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const int kq = g + j * G;
-        if (kq < 4) {
-            float4 ah, al;
-            split4(a[j], ah, al, x1);
-            const int off = r * 64 + ((kq ^ ((r >> 1) & 3)) << 4);
-            *reinterpret_cast<float4*>(hi + off) = ah;
-            if (!x1) *reinterpret_cast<float4*>(lo + off) = al;
-        }
-    }
+    return pl;
 }
 
-__global__ void __launch_bounds__(kThreads, 1)
+__device__ __forceinline__ void transpose_split16(const float* __restrict__ raw, uint8_t* hi, uint8_t* lo,
+                                                  const XfPlan& pl, bool x1) {
+    float4 a[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+        if (pl.ok[j]) {
+            const float* q = raw + pl.ld[j];
+            a[j].x = q[0];
+            a[j].y = q[pl.rows];
+            a[j].z = q[2 * pl.rows];
+            a[j].w = q[3 * pl.rows];
+        }
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+        if (pl.ok[j]) {
+            float4 ah, al;
+            split4(a[j], ah, al, x1);
+            *reinterpret_cast<float4*>(hi + pl.st[j]) = ah;
+            if (!x1) *reinterpret_cast<float4*>(lo + pl.st[j]) = al;
+        }
+}
+
+__global__ void __launch_bounds__(kWgThreads, 1)
 gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const KParams p) {
     extern __shared__ uint8_t smem_dyn[];
     uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);   // keeps the shared state space
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kWgBars);
-    uint64_t* raw_full = bars + 0;               // [3]
-    uint64_t* raw_empty = bars + 3;              // [3]
-    uint64_t* split_full = bars + 6;             // [3]
-    uint64_t* split_empty = bars + 9;            // [3]
-    uint64_t* tmem_full = bars + 12;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
+    uint64_t* raw_full = bars + 0;               // [kWgNR]
+    uint64_t* raw_empty = bars + kWgNR;          // [kWgNR]
+    uint64_t* split_full = bars + 2 * kWgNR;     // [kWgNS]
+    uint64_t* split_empty = bars + 2 * kWgNR + kWgNS;
+    uint64_t* tmem_full = bars + 2 * kWgNR + 2 * kWgNS;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
     const int BN = p.BN;
@@ -265,16 +282,18 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     const int nkb = (k1 - k0 + kWgBK - 1) / kWgBK;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < kWgNS; ++s) {
+        for (int s = 0; s < kWgNR; ++s) {
             mbar_init(raw_full + s, 1);
             mbar_init(raw_empty + s, kWgXfThreads);
+        }
+        for (int s = 0; s < kWgNS; ++s) {
             mbar_init(split_full + s, kWgXfThreads);
             mbar_init(split_empty + s, 1);
         }
         mbar_init(tmem_full, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (warp == kMmaWarp) {
+    if (warp == kWgMmaWarp) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                      "r"(tcols));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -284,7 +303,7 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
-    if (warp == kTmaWarp) {
+    if (warp == kWgTmaWarp) {
         if (lane == 0) {
             const uint32_t bytes = (uint32_t)(BM * kWgBK * 4 + BN * kWgBK * 4);
             int s = 0;
@@ -294,10 +313,10 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                 mbar_expect_tx(raw_full + s, bytes);
                 tma_load_2d(smem + kWgRawA + s * 8192, &tmA, mt * BM, k0 + kb * kWgBK, raw_full + s);
                 tma_load_2d(smem + kWgRawB + s * 16384, &tmB, nt * BN, k0 + kb * kWgBK, raw_full + s);
-                if (++s == kWgNS) { s = 0; ph ^= 1; }
+                if (++s == kWgNR) { s = 0; ph ^= 1; }
             }
         }
-    } else if (warp == kMmaWarp) {
+    } else if (warp == kWgMmaWarp) {
         if (lane == 0) {
             const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
                                    ((uint32_t)(BM >> 4) << 24);
@@ -328,20 +347,21 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     } else {
         // warps 0-7: transpose + split every k block; then warps 0-3 run the epilogue
         const int t = threadIdx.x;
-        int s = 0;
-        uint32_t ph = 0;
+        const XfPlan pa = make_xf_plan(BM, t, kWgXfThreads), pb = make_xf_plan(BN, t, kWgXfThreads);
+        int rs = 0, ss = 0;
+        uint32_t rph = 0, sph = 0;
         for (int kb = 0; kb < nkb; ++kb) {
-            uint8_t* sp = smem + kWgSplit + s * kWgSplitStage;
-            mbar_wait(raw_full + s, ph);
-            mbar_wait(split_empty + s, ph ^ 1);
-            transpose_split16<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawA + s * 8192), sp, sp + 8192,
-                                            BM, t, x1);
-            transpose_split16<kWgXfThreads>(reinterpret_cast<const float*>(smem + kWgRawB + s * 16384), sp + 16384,
-                                            sp + 32768, BN, t, x1);
+            uint8_t* sp = smem + kWgSplit + ss * kWgSplitStage;
+            mbar_wait(raw_full + rs, rph);
+            mbar_wait(split_empty + ss, sph ^ 1);
+            transpose_split16(reinterpret_cast<const float*>(smem + kWgRawA + rs * 8192), sp, sp + 8192, pa, x1);
+            transpose_split16(reinterpret_cast<const float*>(smem + kWgRawB + rs * 16384), sp + 16384, sp + 32768,
+                              pb, x1);
+            mbar_arrive(raw_empty + rs);     // raw tile consumed (generic reads done)
             fence_proxy_async();
-            mbar_arrive(raw_empty + s);
-            mbar_arrive(split_full + s);
-            if (++s == kWgNS) { s = 0; ph ^= 1; }
+            mbar_arrive(split_full + ss);
+            if (++rs == kWgNR) { rs = 0; rph ^= 1; }
+            if (++ss == kWgNS) { ss = 0; sph ^= 1; }
         }
         if (warp < 4) {
             mbar_wait(tmem_full, 0);
@@ -362,7 +382,7 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
         }
     }
     __syncthreads();
-    if (warp == kMmaWarp) {
+    if (warp == kWgMmaWarp) {
         tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
     }
@@ -682,7 +702,7 @@ cudaError_t launch_wgrad(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    gemm_wgrad_kernel<<<g.grid, kThreads, kWgSmem, s>>>(g.tmA, g.tmB, kp);
+    gemm_wgrad_kernel<<<g.grid, kWgThreads, kWgSmem, s>>>(g.tmA, g.tmB, kp);
     count_launches(1);
     return cudaGetLastError();
 }

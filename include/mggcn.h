@@ -152,6 +152,12 @@ int mggcn_get_weights(mggcn_model m, int32_t layer, float* W);
 int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float* loss,
                   float* logits_local);
 int mggcn_backward(mggcn_model m);
+/* mggcn_prefetch — enqueue the host->device copy of the NEXT forward's inputs
+ * (same arguments as mggcn_forward) on a library-owned copy stream into the
+ * second input buffer, so that it overlaps the current epoch; the next
+ * mggcn_forward(m, NULL, 0, NULL, ...) consumes it.  The caller keeps the
+ * host buffers valid until that forward returns.  ESTATE if one is pending. */
+int mggcn_prefetch(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local);
 /* Drops the MGGCN_F_CACHE_L0 aggregate; the next forward recomputes it from X. */
 int mggcn_reset_cache(mggcn_model m);
 int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps);

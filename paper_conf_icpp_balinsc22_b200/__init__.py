@@ -32,6 +32,7 @@ EXPORTS = (
     "mggcn_backward", "mggcn_step", "mggcn_get_loss", "mggcn_get_grad", "mggcn_get_adam", "mggcn_set_adam",
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
+    "mggcn_prefetch",
 )
 
 
@@ -82,6 +83,7 @@ def _load():
         "mggcn_debug_gemm": ([i32, i64, i64, i64, P, i64, P, i64, P, i64, u32, up], ctypes.c_int),
         "mggcn_kernel_launch_count": ([], ctypes.c_int64),
         "mggcn_reset_cache": ([P], ctypes.c_int),
+        "mggcn_prefetch": ([P, P, i64, P], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -222,6 +224,10 @@ def mggcn_forward(m, X, ldx, y, want_loss=True, logits=None):
 
 def mggcn_backward(m):
     _check(_lib.mggcn_backward(m))
+
+
+def mggcn_prefetch(m, X, ldx, y):
+    _check(_lib.mggcn_prefetch(m, _ptr(X), ldx, _ptr(y)))
 
 
 def mggcn_reset_cache(m):

@@ -110,8 +110,10 @@ struct Rank {
         return part->tileB(j);
     }
     float* inv_deg = nullptr;
-    float* Xs = nullptr;
+    float* Xs = nullptr;             // current input buffer (= Xbuf[xcur])
     int32_t* y = nullptr;
+    float* Xbuf[2] = {nullptr, nullptr};   // double-buffered inputs (mggcn_prefetch)
+    int32_t* ybuf[2] = {nullptr, nullptr};
     float* T0 = nullptr;
     float* HWB = nullptr;
     float* BC[2] = {nullptr, nullptr};
@@ -166,6 +168,12 @@ struct mggcn_model_s {
     // X staging plan bookkeeping
     int layer_ids[64];
     bool t0_valid = false;          // MGGCN_F_CACHE_L0: T0 = Â'^T X computed
+    // input prefetch (mggcn_prefetch): copy stream, staging chunk, buffer events
+    cudaStream_t cp = nullptr;
+    float* xstage = nullptr;
+    int64_t xstage_floats = 0;
+    cudaEvent_t ev_pref = nullptr, ev_xfree[2] = {nullptr, nullptr};
+    int xcur = 0, pref_buf = -1;
 };
 
 namespace {
@@ -259,6 +267,8 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
     m->WG = b.take<float>(m->wtotal);
     m->loss_sum = b.take<double>(1);
     m->ntrain = b.take<int64_t>(1);
+    m->xstage_floats = (int64_t)16 << 20;   // 64 MB host-copy staging chunk for the copy stream
+    m->xstage = b.take<float>(m->xstage_floats);
     m->Wt_hi.assign(L, nullptr); m->Wt_lo.assign(L, nullptr);
     m->Ws_hi.assign(L, nullptr); m->Ws_lo.assign(L, nullptr);
     for (int l = 0; l < L; ++l) {
@@ -294,8 +304,12 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             }
         }
         r.inv_deg = b.take<float>(r.rows);
-        r.Xs = b.take<float>(r.rows * m->ld[0]);
-        r.y = b.take<int32_t>(r.rows);
+        for (int k = 0; k < 2; ++k) {
+            r.Xbuf[k] = b.take<float>(r.rows * m->ld[0]);
+            r.ybuf[k] = b.take<int32_t>(r.rows);
+        }
+        r.Xs = r.Xbuf[0];
+        r.y = r.ybuf[0];
         r.T0 = m->order[0] == S_ORDER ? b.take<float>(r.rows * m->ld[0]) : nullptr;
         r.HWB = b.take<float>(r.rows * std::max<int64_t>(m->hw_ld, 4));
         if (P > 1) {
@@ -348,7 +362,7 @@ int upload_static(mggcn_model_s* m) {
             for (int j = 0; j < pt->P; ++j) r.B[j] = r.F[j];
         CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
         // zero every activation buffer once: padding columns stay 0 forever
-        CK(cudaMemsetAsync(r.Xs, 0, sizeof(float) * r.rows * m->ld[0], m->cs));
+        for (int k = 0; k < 2; ++k) CK(cudaMemsetAsync(r.Xbuf[k], 0, sizeof(float) * r.rows * m->ld[0], m->cs));
         for (int l = 0; l < m->L; ++l)
             CK(cudaMemsetAsync(r.AHWB[l], 0, sizeof(float) * r.rows * m->ld[l + 1], m->cs));
         CK(cudaMemsetAsync(r.HWB, 0, sizeof(float) * r.rows * std::max<int64_t>(m->hw_ld, 4), m->cs));
@@ -372,9 +386,48 @@ int upload_static(mggcn_model_s* m) {
 // The input operand of layer l (H_l): staged X for l = 0, else H'_{l-1} in AHWB_{l-1}.
 float* layer_input(mggcn_model_s* m, Rank& r, int l) { return l == 0 ? r.Xs : r.AHWB[l - 1]; }
 
-int plan_gemms(mggcn_model_s* m) {
+// GEMM plans (tensor maps + tiling) of layer l for one rank; layer 0's depend
+// on the current input buffer r.Xs and are rebuilt when it changes.
+int plan_layer(mggcn_model_s* m, Rank& r, int l) {
     const int L = m->L;
     const int flags = (m->flags & MGGCN_F_TF32X1) ? GEMM_TF32X1 : 0;
+    const bool relu_here = (l < L - 1) || (m->flags & MGGCN_F_RELU_LAST);
+    // forward (Eq. 5): G-order HW = H W -> HWB ; S-order AHW = T W (+ReLU) -> AHWB_l
+    if (m->order[l] == G_ORDER) {
+        if (gemm_plan_rows(r.g_fwd[l], r.rows, m->d[l + 1], m->d[l], layer_input(m, r, l), m->ld[l], m->Wt_hi[l],
+                           m->Wt_lo[l], m->ld[l], r.HWB, m->ld[l + 1], flags))
+            return -1;
+    } else {
+        if (gemm_plan_rows(r.g_fwd[l], r.rows, m->d[l + 1], m->d[l], r.T0, m->ld[0], m->Wt_hi[l], m->Wt_lo[l],
+                           m->ld[l], r.AHWB[l], m->ld[l + 1], flags | (relu_here ? GEMM_RELU : 0)))
+            return -1;
+    }
+    r.has_fwd[l] = 1;
+    // weight gradient (Eq. 10, reading C2): W_G = H^T HW_G (G) or T^T Z_G (S)
+    {
+        const float* Aop = m->order[l] == G_ORDER ? layer_input(m, r, l) : r.T0;
+        const float* Bop = m->order[l] == G_ORDER ? r.HWB : r.AHWB[l];
+        size_t pf = 0;
+        if (gemm_plan_wgrad(r.g_wgrad[l], m->d[l], m->d[l + 1], r.rows, Aop, m->ld[l], Bop, m->ld[l + 1], flags, &pf))
+            return -1;
+        r.g_wgrad[l].partial = r.gemm_partial;
+        r.has_wgrad[l] = 1;
+    }
+    // input gradient (Eq. 11) for l > 0: AHWB_{l-1} = (HW_G W^T) * [H'_{l-1} > 0] (* inv_deg)
+    if (l > 0) {
+        int f = flags | GEMM_MASK;
+        if (m->order[l - 1] == G_ORDER && m->pattern) f |= GEMM_SCALE;
+        if (gemm_plan_rows(r.g_igrad[l], r.rows, m->d[l], m->d[l + 1], r.HWB, m->ld[l + 1], m->Ws_hi[l],
+                           m->Ws_lo[l], m->ld[l + 1], r.AHWB[l - 1], m->ld[l], f))
+            return -1;
+        r.g_igrad[l].rowscale = r.inv_deg;
+        r.has_igrad[l] = 1;
+    }
+    return 0;
+}
+
+int plan_gemms(mggcn_model_s* m) {
+    const int L = m->L;
     for (auto& r : m->ranks) {
         r.g_fwd.assign(L, GemmPlan());
         r.g_wgrad.assign(L, GemmPlan());
@@ -383,47 +436,58 @@ int plan_gemms(mggcn_model_s* m) {
         r.has_wgrad.assign(L, 0);
         r.has_igrad.assign(L, 0);
         if (r.rows == 0) continue;
-        for (int l = 0; l < L; ++l) {
-            const bool relu_here = (l < L - 1) || (m->flags & MGGCN_F_RELU_LAST);
-            // forward (Eq. 5): G-order HW = H W -> HWB ; S-order AHW = T W (+ReLU) -> AHWB_l
-            if (m->order[l] == G_ORDER) {
-                if (gemm_plan_rows(r.g_fwd[l], r.rows, m->d[l + 1], m->d[l], layer_input(m, r, l), m->ld[l],
-                                   m->Wt_hi[l], m->Wt_lo[l], m->ld[l], r.HWB, m->ld[l + 1], flags))
-                    goto fail;
-            } else {
-                if (gemm_plan_rows(r.g_fwd[l], r.rows, m->d[l + 1], m->d[l], r.T0, m->ld[0], m->Wt_hi[l],
-                                   m->Wt_lo[l], m->ld[l], r.AHWB[l], m->ld[l + 1],
-                                   flags | (relu_here ? GEMM_RELU : 0)))
-                    goto fail;
+        for (int l = 0; l < L; ++l)
+            if (plan_layer(m, r, l)) {
+                set_error("model: GEMM plan / tensor-map encoding failed (needs an sm_100 device)");
+                return MGGCN_ECUDA;
             }
-            r.has_fwd[l] = 1;
-            // weight gradient (Eq. 10, reading C2): W_G = H^T HW_G (G) or T^T Z_G (S)
-            {
-                const float* Aop = m->order[l] == G_ORDER ? layer_input(m, r, l) : r.T0;
-                const float* Bop = m->order[l] == G_ORDER ? r.HWB : r.AHWB[l];
-                size_t pf = 0;
-                if (gemm_plan_wgrad(r.g_wgrad[l], m->d[l], m->d[l + 1], r.rows, Aop, m->ld[l], Bop, m->ld[l + 1], flags,
-                                    &pf))
-                    goto fail;
-                r.g_wgrad[l].partial = r.gemm_partial;
-                r.has_wgrad[l] = 1;
-            }
-            // input gradient (Eq. 11) for l > 0: AHWB_{l-1} = (HW_G W^T) * [H'_{l-1} > 0] (* inv_deg)
-            if (l > 0) {
-                int f = flags | GEMM_MASK;
-                if (m->order[l - 1] == G_ORDER && m->pattern) f |= GEMM_SCALE;
-                if (gemm_plan_rows(r.g_igrad[l], r.rows, m->d[l], m->d[l + 1], r.HWB, m->ld[l + 1], m->Ws_hi[l],
-                                   m->Ws_lo[l], m->ld[l + 1], r.AHWB[l - 1], m->ld[l], f))
-                    goto fail;
-                r.g_igrad[l].rowscale = r.inv_deg;
-                r.has_igrad[l] = 1;
-            }
+    }
+    return MGGCN_OK;
+}
+
+// Switch every rank to input buffer k (after a prefetch) and re-plan layer 0.
+int use_input_buffer(mggcn_model_s* m, int k) {
+    if (k == m->xcur) return MGGCN_OK;
+    m->xcur = k;
+    for (auto& r : m->ranks) {
+        r.Xs = r.Xbuf[k];
+        r.y = r.ybuf[k];
+        if (r.rows && plan_layer(m, r, 0)) {
+            set_error("model: GEMM re-plan failed");
+            return MGGCN_ECUDA;
         }
     }
     return MGGCN_OK;
-fail:
-    set_error("model: GEMM plan / tensor-map encoding failed (needs an sm_100 device)");
-    return MGGCN_ECUDA;
+}
+
+// Input copy of (X, y) rows into buffer k on stream s (host or device source).
+// A host X whose pitch differs from the padded ld goes through `stage` in
+// contiguous chunks (1-D H2D, then a device 2-D copy): pitched H2D copies are slow.
+int copy_inputs(mggcn_model_s* m, int k, const float* X, int64_t ldx, const int32_t* y, cudaStream_t s,
+                float* stage, int64_t stage_floats) {
+    cudaPointerAttributes pa;
+    const bool host_x = cudaPointerGetAttributes(&pa, X) != cudaSuccess || pa.type == cudaMemoryTypeHost ||
+                        pa.type == cudaMemoryTypeUnregistered;
+    cudaGetLastError();   // clear a possible error from the attribute query
+    for (auto& r : m->ranks) {
+        if (r.rows == 0) continue;
+        float* dst = r.Xbuf[k];
+        if (host_x && ldx != m->ld[0]) {
+            const int64_t chunk = std::max<int64_t>(1, stage_floats / ldx);
+            for (int64_t r0 = 0; r0 < r.rows; r0 += chunk) {
+                const int64_t nr = std::min(chunk, r.rows - r0);
+                CK(cudaMemcpyAsync(stage, X + (r.row_off + r0) * ldx, sizeof(float) * nr * ldx,
+                                   cudaMemcpyHostToDevice, s));
+                CK(cudaMemcpy2DAsync(dst + r0 * m->ld[0], m->ld[0] * 4, stage, ldx * 4, m->d[0] * 4, nr,
+                                     cudaMemcpyDeviceToDevice, s));
+            }
+        } else {
+            CK(cudaMemcpy2DAsync(dst, m->ld[0] * 4, X + r.row_off * ldx, ldx * 4, m->d[0] * 4, r.rows,
+                                 cudaMemcpyDefault, s));
+        }
+        CK(cudaMemcpyAsync(r.ybuf[k], y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, s));
+    }
+    return MGGCN_OK;
 }
 
 // tf32 hi / lo weight copies for the row GEMMs (after set_weights and Adam).
@@ -731,8 +795,11 @@ static void destroy(mggcn_model_s* m) {
             if (r.ev_bc[s]) cudaEventDestroy(r.ev_bc[s]);
             if (r.ev_free[s]) cudaEventDestroy(r.ev_free[s]);
         }
-    for (cudaEvent_t e : {m->ev_begin, m->ev_comm_end, m->ev_tmp, m->ev_wg, m->ev_comm_done})
+    if (m->cp) cudaStreamSynchronize(m->cp);
+    for (cudaEvent_t e : {m->ev_begin, m->ev_comm_end, m->ev_tmp, m->ev_wg, m->ev_comm_done, m->ev_pref, m->ev_xfree[0],
+                          m->ev_xfree[1]})
         if (e) cudaEventDestroy(e);
+    if (m->cp) cudaStreamDestroy(m->cp);
     for (auto& rec : m->prof_recs) {
         cudaEventDestroy(std::get<1>(rec));
         cudaEventDestroy(std::get<2>(rec));
@@ -787,7 +854,12 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
         destroy(m);
         return code;
     };
-    for (cudaEvent_t* e : {&m->ev_begin, &m->ev_comm_end, &m->ev_tmp, &m->ev_wg, &m->ev_comm_done})
+    if (cudaStreamCreateWithFlags(&m->cp, cudaStreamNonBlocking) != cudaSuccess) {
+        set_error("model_create: cudaStreamCreate failed");
+        return fail(MGGCN_ECUDA);
+    }
+    for (cudaEvent_t* e : {&m->ev_begin, &m->ev_comm_end, &m->ev_tmp, &m->ev_wg, &m->ev_comm_done, &m->ev_pref,
+                           &m->ev_xfree[0], &m->ev_xfree[1]})
         if (cudaEventCreateWithFlags(e, cudaEventDisableTiming) != cudaSuccess) {
             set_error("model_create: cudaEventCreate failed");
             return fail(MGGCN_ECUDA);
@@ -932,35 +1004,24 @@ extern "C" int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, co
 static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int32_t* y, float* loss,
                         float* logits) {
     const int L = m->L;
-    // inputs -> internal buffers (host or device source; this is the e2e H2D when host).
-    // A host X with a row pitch != the padded ld is staged through HWB (free at
-    // this point) in contiguous chunks: one 1-D H2D copy per chunk, then a
-    // device 2-D copy into the padded layout (pitched H2D copies are slow).
-    cudaPointerAttributes pa;
-    const bool host_x = cudaPointerGetAttributes(&pa, X) != cudaSuccess || pa.type == cudaMemoryTypeHost ||
-                        pa.type == cudaMemoryTypeUnregistered;
-    cudaGetLastError();   // clear a possible error from the attribute query
+    // inputs -> internal buffers (this is the e2e H2D when X is host memory).
+    // X == NULL: use the buffer filled by mggcn_prefetch on the copy stream.
     const bool use_cache = (m->flags & MGGCN_F_CACHE_L0) && m->t0_valid;
-    for (auto& r : m->ranks) {
-        if (r.rows == 0) continue;
+    if (!X) {
+        CK(cudaStreamWaitEvent(m->cs, m->ev_pref, 0));
+        RC(use_input_buffer(m, m->pref_buf));
+        m->pref_buf = -1;
+    } else {
         ProfScope ps(m, PC_OTHER, m->cs);
         if (use_cache) {
-            // X is not read again: layer 0 starts from the cached T0
-        } else if (host_x && ldx != m->ld[0]) {
-            const int64_t stage_floats = r.rows * std::max<int64_t>(m->hw_ld, 4);
-            const int64_t chunk = std::max<int64_t>(1, stage_floats / ldx);
-            for (int64_t r0 = 0; r0 < r.rows; r0 += chunk) {
-                const int64_t nr = std::min(chunk, r.rows - r0);
-                CK(cudaMemcpyAsync(r.HWB, X + (r.row_off + r0) * ldx, sizeof(float) * nr * ldx,
-                                   cudaMemcpyHostToDevice, m->cs));
-                CK(cudaMemcpy2DAsync(r.Xs + r0 * m->ld[0], m->ld[0] * 4, r.HWB, ldx * 4, m->d[0] * 4, nr,
-                                     cudaMemcpyDeviceToDevice, m->cs));
-            }
+            // X is not read again (layer 0 starts from the cached T0): only the labels
+            for (auto& r : m->ranks)
+                if (r.rows) CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
         } else {
-            CK(cudaMemcpy2DAsync(r.Xs, m->ld[0] * 4, X + r.row_off * ldx, ldx * 4, m->d[0] * 4, r.rows,
-                                 cudaMemcpyDefault, m->cs));
+            float* stage = m->ranks[0].HWB;   // free at this point of the epoch
+            const int64_t stage_floats = m->ranks[0].rows * std::max<int64_t>(m->hw_ld, 4);
+            RC(copy_inputs(m, m->xcur, X, ldx, y, m->cs, stage, stage_floats));
         }
-        CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
     }
     for (int l = 0; l < L; ++l) {
         const bool relu_here = (l < L - 1) || (m->flags & MGGCN_F_RELU_LAST);
@@ -1028,13 +1089,41 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
 extern "C" int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float* loss,
                              float* logits_local) {
     MODEL_GUARD(m);
-    if (!X_local || !y_local || ldx < m->d[0]) {
-        set_error("forward: NULL X/y or ldx < d_0");
+    if (!X_local) {
+        if (m->pref_buf < 0) {
+            set_error("forward: X is NULL and no mggcn_prefetch is pending");
+            return MGGCN_ESTATE;
+        }
+    } else if (!y_local || ldx < m->d[0]) {
+        set_error("forward: NULL y or ldx < d_0");
         return MGGCN_EINVAL;
     }
     RC(poison(m, wait_wg(m)));
     int rc = forward_impl(m, X_local, ldx, y_local, loss, logits_local);
+    if (rc == MGGCN_OK && cudaEventRecord(m->ev_xfree[m->xcur], m->cs) != cudaSuccess) rc = MGGCN_ECUDA;
     if (rc == MGGCN_OK) m->state = ST_FWD;
+    return poison(m, rc);
+}
+
+extern "C" int mggcn_prefetch(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local) {
+    MODEL_GUARD(m);
+    if (!X_local || !y_local || ldx < m->d[0]) {
+        set_error("prefetch: NULL X/y or ldx < d_0");
+        return MGGCN_EINVAL;
+    }
+    if (m->pref_buf >= 0) {
+        set_error("prefetch: a prefetch is already pending (call mggcn_forward(X = NULL) first)");
+        return MGGCN_ESTATE;
+    }
+    const int k = 1 - m->xcur;
+    auto body = [&]() -> int {
+        CK(cudaStreamWaitEvent(m->cp, m->ev_xfree[k], 0));   // last reader of buffer k is done
+        RC(copy_inputs(m, k, X_local, ldx, y_local, m->cp, m->xstage, m->xstage_floats));
+        CK(cudaEventRecord(m->ev_pref, m->cp));
+        return MGGCN_OK;
+    };
+    int rc = body();
+    if (rc == MGGCN_OK) m->pref_buf = k;
     return poison(m, rc);
 }
 
@@ -1130,6 +1219,7 @@ extern "C" int mggcn_backward(mggcn_model m) {
         return MGGCN_ESTATE;
     }
     int rc = backward_impl(m);
+    if (rc == MGGCN_OK && cudaEventRecord(m->ev_xfree[m->xcur], m->cs) != cudaSuccess) rc = MGGCN_ECUDA;
     if (rc == MGGCN_OK) m->state = ST_BWD;
     return poison(m, rc);
 }

@@ -7,7 +7,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from . import (MGGCN_F_OVERLAP, mggcn_backward, mggcn_epoch_work, mggcn_forward, mggcn_get_adam, mggcn_get_grad,
+from . import (MGGCN_F_OVERLAP, mggcn_backward, mggcn_prefetch, mggcn_epoch_work, mggcn_forward, mggcn_get_adam, mggcn_get_grad,
                mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free, mggcn_load_csr,
                mggcn_model_create, mggcn_model_free, mggcn_part_free, mggcn_part_info, mggcn_partition,
                mggcn_set_adam, mggcn_set_weights, mggcn_step, mggcn_workspace_bytes)
@@ -62,9 +62,24 @@ class GCN:
         return [mggcn_get_weights(self.m, l, (self.dims[l], self.dims[l + 1])) for l in range(self.L)]
 
     # ---------------------------------------------------------- hot path
-    def forward(self, X_local, y_local, want_loss=True, logits=None):
-        """X_local / y_local: numpy (host) or torch (device or pinned host) rows of X', y'."""
+    def prefetch(self, X_local, y_local):
+        """Start the copy of the next forward's inputs (overlaps the current epoch)."""
         torch = self.torch
+        if isinstance(X_local, torch.Tensor) and X_local.is_cuda:
+            torch.cuda.current_stream(self.device).synchronize()
+        self._pref = (X_local, y_local)          # keep the buffers alive until consumed
+        mggcn_prefetch(self.m, X_local, X_local.shape[1], y_local)
+
+    def forward(self, X_local, y_local, want_loss=True, logits=None):
+        """X_local / y_local: numpy (host) or torch (device or pinned host) rows of X', y';
+        X_local = None consumes the inputs of the last prefetch()."""
+        torch = self.torch
+        if X_local is None:
+            loss = mggcn_forward(self.m, None, 0, None, want_loss, logits)
+            self._pref = None
+            if logits is not None:
+                torch.cuda.current_stream(self.device).wait_stream(self.cs)
+            return loss
         if isinstance(X_local, torch.Tensor) and X_local.is_cuda:
             self.cs.wait_stream(torch.cuda.current_stream(self.device))
         ldx = X_local.shape[1] if X_local.ndim == 2 else self.dims[0]

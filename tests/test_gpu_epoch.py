@@ -225,6 +225,41 @@ def test_multi_step_training_decreases_loss(mg):
     gm2.close()
 
 
+def test_prefetch_matches_direct_inputs(mg):
+    """mggcn_prefetch (next epoch's host inputs copied on the copy stream into the
+    second input buffer) gives bitwise the same training as passing X each forward."""
+    n, m = 3001, 60000
+    rp, col = gen.rmat_csr(n, m, 61)
+    dims = (602, 32, 7)
+    X = gen.features(n, dims[0], 62)
+    y = gen.labels(n, dims[-1], 63, 100)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 64 + l) for l in range(2)]
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    runs = []
+    for use_prefetch in (False, True):
+        gm = GCN(n, rp, col, None, dims, P=2, perm_seed=65, loopback=True)
+        gm.set_weights(Ws)
+        Xh = torch.from_numpy(gm.permute_rows(X)).pin_memory()
+        yh = torch.from_numpy(gm.permute_rows(y)).pin_memory()
+        losses = []
+        if use_prefetch:
+            gm.prefetch(Xh, yh)
+        for k in range(4):
+            if use_prefetch:
+                losses.append(gm.forward(None, None))
+                if k < 3:
+                    gm.prefetch(Xh, yh)
+            else:
+                losses.append(gm.forward(Xh, yh))
+            gm.backward()
+            gm.step()
+        runs.append((losses, gm.get_weights()))
+        gm.close()
+    assert runs[0][0] == runs[1][0]
+    for a, b in zip(runs[0][1], runs[1][1]):
+        assert np.array_equal(a, b)
+
+
 def test_state_errors(mg):
     from paper_conf_icpp_balinsc22_b200 import GCN
     rp, col = gen.rmat_csr(200, 2000, 1)
@@ -234,6 +269,9 @@ def test_state_errors(mg):
     assert e.value.code == mg.MGGCN_ESTATE
     with pytest.raises(mg.MggcnError) as e:
         gm.step()
+    assert e.value.code == mg.MGGCN_ESTATE
+    with pytest.raises(mg.MggcnError) as e:
+        gm.forward(None, None)                       # no prefetch pending
     assert e.value.code == mg.MGGCN_ESTATE
     gm.close()
     with pytest.raises(mg.MggcnError) as e:

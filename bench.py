@@ -235,7 +235,7 @@ def main():
     Xl = gm.permute_rows(X)
     yl = gm.permute_rows(y)
     del X
-    Xd = torch.from_numpy(Xl).cuda()
+    Xd = gm.device_inputs(Xl)          # padded device layout: layer 0 reads it in place
     yd = torch.from_numpy(yl).cuda()
     torch.cuda.synchronize()
 

@@ -140,7 +140,11 @@ int mggcn_get_weights(mggcn_model m, int32_t layer, float* W);
  *   X_local  fp32 rows of X' owned by this model (rows p(rank)..p(rank+1)-1
  *            of the PERMUTED features; all n rows in loopback mode), row
  *            stride ldx >= d_0.  Host or device pointer (host: copied on the
- *            compute stream; this is the end-to-end path).
+ *            compute stream; this is the end-to-end path).  A device X whose
+ *            stride is the library's padded ld (d_0 rounded up to 8) and that
+ *            is 16-B aligned is read IN PLACE (no copy): it must then stay valid
+ *            and unchanged until this epoch's mggcn_backward has completed.
+ *            NULL: use the inputs of the pending mggcn_prefetch.
  *   y_local  int32 labels of the same rows (host or device); -1 = unlabelled.
  *   loss     host out: global mean CE over labelled vertices (reading C5), or
  *            NULL (no host synchronisation).

@@ -45,7 +45,12 @@ struct HostItems {
     int64_t nslots = 0;
 };
 
-void build_items(const HostTile& t, HostItems& h) {
+// Work items of one tile: hub rows (> kSplit entries) are cut into segments
+// (first, so the long work starts early); every other row is one item, in
+// `order` (the rows sorted by ORIGINAL vertex id: neighbouring original ids
+// share neighbourhoods in the skewed input order, so warps of one SM that run
+// consecutive items reuse gathered rows in L1/L2; numbering is unchanged).
+void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& order) {
     const auto& rp = t.rowptr;
     for (int64_t r = 0; r < t.nrows; ++r) {
         const int64_t len = rp[r + 1] - rp[r];
@@ -59,9 +64,9 @@ void build_items(const HostTile& t, HostItems& h) {
             h.nslots += nseg;
         }
     }
-    for (int64_t r = 0; r < t.nrows; ++r) {
+    for (int32_t r : order) {
         const int64_t len = rp[r + 1] - rp[r];
-        if (len <= kSplit) h.items.push_back(make_int4((int)r, rp[r], rp[r + 1], -1));
+        if (len <= kSplit) h.items.push_back(make_int4(r, rp[r], rp[r + 1], -1));
     }
 }
 
@@ -445,19 +450,41 @@ int plan_gemms(mggcn_model_s* m) {
     return MGGCN_OK;
 }
 
-// Switch every rank to input buffer k (after a prefetch) and re-plan layer 0.
-int use_input_buffer(mggcn_model_s* m, int k) {
-    if (k == m->xcur) return MGGCN_OK;
-    m->xcur = k;
+// Point every rank's layer-0 input at `Xrank(r)` and re-plan layer 0's GEMMs
+// (tensor maps) if it changed.
+template <typename F>
+int set_layer0_input(mggcn_model_s* m, F Xrank) {
     for (auto& r : m->ranks) {
-        r.Xs = r.Xbuf[k];
-        r.y = r.ybuf[k];
+        float* x = Xrank(r);
+        if (r.Xs == x) continue;
+        r.Xs = x;
         if (r.rows && plan_layer(m, r, 0)) {
             set_error("model: GEMM re-plan failed");
             return MGGCN_ECUDA;
         }
     }
     return MGGCN_OK;
+}
+
+// Switch every rank to input buffer k (after a prefetch).
+int use_input_buffer(mggcn_model_s* m, int k) {
+    m->xcur = k;
+    for (auto& r : m->ranks) r.y = r.ybuf[k];
+    return set_layer0_input(m, [k](Rank& r) { return r.Xbuf[k]; });
+}
+
+// A device X with the padded row stride and 16-B alignment is used in place.
+bool device_zero_copy(mggcn_model_s* m, const float* X, int64_t ldx) {
+    if (ldx != m->ld[0] || (reinterpret_cast<uintptr_t>(X) & 15)) return false;
+    cudaPointerAttributes pa;
+    const bool dev = cudaPointerGetAttributes(&pa, X) == cudaSuccess && pa.type == cudaMemoryTypeDevice;
+    cudaGetLastError();
+    return dev;
+}
+
+int use_external_input(mggcn_model_s* m, const float* X) {
+    for (auto& r : m->ranks) r.y = r.ybuf[m->xcur];
+    return set_layer0_input(m, [&](Rank& r) { return const_cast<float*>(X) + r.row_off * m->ld[0]; });
 }
 
 // Input copy of (X, y) rows into buffer k on stream s (host or device source).
@@ -725,12 +752,30 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
                 for (int j = 0; j < m->P; ++j) coalesce(r.part->B[j], r.cB[j]);
             }
         }
+        std::vector<int32_t> order(r.rows);
+        {
+            const mggcn_part_s* pt = r.part;
+            std::vector<int64_t> orig(r.rows);           // original id of local row rr
+            const int64_t lo = pt->p[pt->rank];
+            for (int64_t v = 0; v < pt->n; ++v) {
+                const int64_t nv = pt->perm[v];
+                if (nv >= lo && nv < lo + r.rows) orig[nv - lo] = v;
+            }
+            for (int64_t rr = 0; rr < r.rows; ++rr) order[rr] = (int32_t)rr;
+            std::sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return orig[a] < orig[b]; });
+        }
         for (int j = 0; j < m->P; ++j) {
-            build_items(r.tF(j), r.hF[j]);
-            if (!r.part->shared_fb) build_items(r.tB(j), r.hB[j]);
+            build_items(r.tF(j), r.hF[j], order);
+            if (!r.part->shared_fb) build_items(r.tB(j), r.hB[j], order);
         }
     }
     m->n_local = off;
+    // the SpMM gathers address B with 32-bit float4 offsets: rows * ld/4 < 2^32
+    if ((double)m->max_rows_j * (double)(std::max(m->bc_ld, m->ld[0]) / 4) >= 4294967296.0 ||
+        (double)off * (double)(std::max(m->bc_ld, m->ld[0]) / 4) >= 4294967296.0) {
+        set_error("model: a feature block exceeds 2^32 float4 (use more parts)");
+        return MGGCN_EUNSUPPORTED;
+    }
     // epoch work model, per this model's rows
     auto spmm_work = [&](int dir, int64_t width) {
         for (auto& r : m->ranks)
@@ -1017,7 +1062,14 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
             // X is not read again (layer 0 starts from the cached T0): only the labels
             for (auto& r : m->ranks)
                 if (r.rows) CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
+        } else if (device_zero_copy(m, X, ldx)) {
+            // device X already in the padded layout: layer 0 reads it in place (it must stay
+            // valid until this epoch's backward has run); labels are still copied
+            RC(use_external_input(m, X));
+            for (auto& r : m->ranks)
+                if (r.rows) CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
         } else {
+            RC(use_input_buffer(m, m->xcur));
             float* stage = m->ranks[0].HWB;   // free at this point of the epoch
             const int64_t stage_floats = m->ranks[0].rows * std::max<int64_t>(m->hw_ld, 4);
             RC(copy_inputs(m, m->xcur, X, ldx, y, m->cs, stage, stage_floats));

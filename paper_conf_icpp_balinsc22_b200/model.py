@@ -47,6 +47,18 @@ class GCN:
                                     self.cs.cuda_stream, self.ms.cuda_stream)
 
     # ---------------------------------------------------------------- data
+    @property
+    def ld0(self):
+        """Padded input row stride: a device X with this stride is read in place."""
+        return (self.dims[0] + 7) // 8 * 8
+
+    def device_inputs(self, X_local):
+        """Device copy of X_local in the padded layout the library reads without copying."""
+        torch = self.torch
+        Xd = torch.zeros((X_local.shape[0], self.ld0), dtype=torch.float32, device=self.device)
+        Xd[:, :X_local.shape[1]] = torch.as_tensor(X_local, device=self.device)
+        return Xd
+
     def permute_rows(self, X):
         """Rows owned by this model of the permuted matrix X' (X'[perm[v]] = X[v])."""
         X = np.asarray(X)

@@ -260,6 +260,32 @@ def test_prefetch_matches_direct_inputs(mg):
         assert np.array_equal(a, b)
 
 
+def test_device_zero_copy_inputs(mg):
+    """A device X in the padded layout (ld = d0 rounded to 8) is read in place:
+    bitwise the same epoch as the staged copy."""
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    out = []
+    for padded in (False, True):
+        gm = GCN(w.n, rp, col, None, w.dims, perm_seed=w.perm_seed)
+        gm.set_weights(Ws)
+        Xl = gm.permute_rows(X)
+        Xd = gm.device_inputs(Xl) if padded else torch.from_numpy(Xl).cuda()
+        assert (Xd.shape[1] == 1440) == padded
+        yd = torch.from_numpy(gm.permute_rows(y)).cuda()
+        losses = []
+        for _ in range(3):
+            losses.append(gm.forward(Xd, yd))
+            gm.backward()
+            gm.step()
+        out.append((losses, gm.get_weights()))
+        gm.close()
+    assert out[0][0] == out[1][0]
+    for a, b in zip(out[0][1], out[1][1]):
+        assert np.array_equal(a, b)
+
+
 def test_state_errors(mg):
     from paper_conf_icpp_balinsc22_b200 import GCN
     rp, col = gen.rmat_csr(200, 2000, 1)

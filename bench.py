@@ -43,6 +43,9 @@ def parse():
     ap.add_argument("--workload", default="reddit", choices=sorted(gen.WORKLOADS))
     ap.add_argument("--impl", default="mggcn", choices=["mggcn", "reference"])
     ap.add_argument("--no-overlap", action="store_true")
+    ap.add_argument("--comm", default="nccl", choices=["nccl", "ipc"],
+                    help="N > 1 exchange backend: the library's NCCL communicator, or MGGCN_F_IPC "
+                         "(copy-engine pulls from CUDA-IPC-mapped peer workspaces)")
     ap.add_argument("--tf32x1", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -202,13 +205,13 @@ def main():
 
     import paper_conf_icpp_balinsc22_b200 as mg
     from paper_conf_icpp_balinsc22_b200 import GCN
-    from paper_conf_icpp_balinsc22_b200.dist import max_over_ranks, share_nccl_id
+    from paper_conf_icpp_balinsc22_b200.dist import ipc_exchange, max_over_ranks, share_nccl_id
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     P = world
-    torch.cuda.set_device(local)
+    torch.cuda.set_device(local % torch.cuda.device_count())   # (IPC ranks may share a GPU in tests)
     if world > 1:
         # control plane only (NCCL unique id, barriers, max over ranks): gloo.  The data
         # path's broadcasts and all-reduces run on the library's own NCCL communicator.
@@ -222,14 +225,20 @@ def main():
     Ws = [gen.glorot(w.dims[l], w.dims[l + 1], w.seed_W + l) for l in range(len(w.dims) - 1)]
     t_gen = time.perf_counter() - t0
 
-    nccl_id = share_nccl_id(dist, mg.mggcn_nccl_unique_id) if world > 1 else None
+
+    def comm_kw():
+        if world == 1:
+            return {}
+        if args.comm == "ipc":
+            return {"comm": "ipc", "ipc_exchange": ipc_exchange(dist)}
+        return {"nccl_id": share_nccl_id(dist, mg.mggcn_nccl_unique_id)}
     flags = mg.MGGCN_F_PROFILE | (0 if args.no_overlap else mg.MGGCN_F_OVERLAP)
     if args.tf32x1:
         flags |= mg.MGGCN_F_TF32X1
     t0 = time.perf_counter()
     graph = mg.mggcn_load_csr(w.n, rp, col)
-    gm = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed, flags=flags, nccl_id=nccl_id,
-             graph=graph)
+    gm = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed, flags=flags, graph=graph,
+             **comm_kw())
     t_setup = time.perf_counter() - t0
     gm.set_weights(Ws)
     Xl = gm.permute_rows(X)
@@ -313,9 +322,8 @@ def main():
         gm.close()
         del gm
         torch.cuda.empty_cache()
-        nid2 = share_nccl_id(dist, mg.mggcn_nccl_unique_id) if world > 1 else None
         gc = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed,
-                 flags=flags | mg.MGGCN_F_CACHE_L0, nccl_id=nid2, graph=graph)
+                 flags=flags | mg.MGGCN_F_CACHE_L0, graph=graph, **comm_kw())
         gc.set_weights(Ws_now)
         for _ in range(max(args.warmup, 1)):
             gc.forward(Xd, yd, want_loss=False)
@@ -375,7 +383,9 @@ def main():
         "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": False, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": workload_desc(w, P) | {"overlap": not args.no_overlap,
-                                         "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)"},
+                                         "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)",
+                                         "comm": (args.comm if P > 1 else "none"),
+                                         "parallelism": f"dp{P} (1D row partition)"},
         "e2e": e2e,
         "gpu_launches": int(launches),
         "clocks": clk,

@@ -61,11 +61,23 @@ enum {
     MGGCN_F_PROFILE = 32u,    /* record per-op CUDA events (see mggcn_get_profile)     */
     MGGCN_F_NO_COALESCE = 64u,/* keep duplicate entries as separate gathers (default:
                                  merged on the device copy, value = multiplicity)       */
-    MGGCN_F_CACHE_L0 = 128u   /* X is constant across epochs (full-batch training): layer 0
+    MGGCN_F_CACHE_L0 = 128u,  /* X is constant across epochs (full-batch training): layer 0
                                  runs SpMM-first and T0 = Â'^T X is computed on the first
                                  forward and reused (exact by associativity,
                                  Eq. 5-6 and Eq. 10).  mggcn_reset_cache() after X changes. */
+    MGGCN_F_IPC = 256u        /* nlocal = 1, P > 1 without NCCL: peers map each
+                                 other's workspaces (CUDA IPC, mggcn_ipc_export / _connect);
+                                 each receiver PULLS the broadcast blocks with copy engines in
+                                 rotated order (no SMs taken from the SpMM), W_G and the loss
+                                 scalars are summed in rank order over peer memory, and
+                                 cross-process order uses device sequence flags written and
+                                 awaited by stream memory operations.  All ranks must issue
+                                 the same sequence of calls with the same kind of X argument
+                                 (host / device / prefetch); device X is always copied. */
 };
+
+/* Size of one rank's IPC descriptor (mggcn_ipc_export). */
+#define MGGCN_IPC_BLOB_BYTES 128
 
 typedef struct mggcn_graph_s* mggcn_graph; /* host CSR of A + in-degrees                     */
 typedef struct mggcn_part_s* mggcn_part;   /* one rank's permuted 1D partition (host)        */
@@ -129,6 +141,19 @@ int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32_t L, const
                        const void* nccl_id128, void* workspace, size_t ws_bytes, uintptr_t compute_stream,
                        uintptr_t comm_stream, mggcn_model* out);
 int mggcn_nccl_unique_id(void* out128);
+/* MGGCN_F_IPC models (P > 1, nlocal = 1, nccl_id128 = NULL): every rank calls
+ * mggcn_ipc_export (writes MGGCN_IPC_BLOB_BYTES host bytes: the CUDA IPC
+ * handle of the allocation that holds its workspace + the offset, rank, P and
+ * symmetric-region size), the caller exchanges the P blobs (e.g. all_gather over
+ * torch.distributed), then every rank calls mggcn_ipc_connect with the P blobs
+ * in rank order (host, P * MGGCN_IPC_BLOB_BYTES bytes), which maps the peers'
+ * workspaces (cudaIpcOpenMemHandle; unmapped by mggcn_model_free).  The
+ * workspace must then stay allocated in every process until all models are
+ * freed.  EINVAL: not an IPC model, blobs of another P / plan / rank order, or
+ * connect called twice; ECUDA: the IPC calls failed (e.g. no P2P between the
+ * devices); ESTATE from mggcn_forward until connected. */
+int mggcn_ipc_export(mggcn_model m, void* blob);
+int mggcn_ipc_connect(mggcn_model m, const void* blobs);
 
 /* Weights W_l (d_l x d_{l+1}, host fp32).  set_weights resets Adam (t = 0). */
 int mggcn_set_weights(mggcn_model m, int32_t layer, const float* W);

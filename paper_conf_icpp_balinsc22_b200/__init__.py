@@ -23,6 +23,8 @@ MGGCN_OK, MGGCN_EINVAL, MGGCN_ENOMEM, MGGCN_ECUDA, MGGCN_ENCCL, MGGCN_ESTATE, MG
 MGGCN_F_OVERLAP, MGGCN_F_RELU_LAST, MGGCN_F_TF32X1, MGGCN_F_NO_BCAST, MGGCN_F_PROFILE = 1, 2, 4, 16, 32
 MGGCN_F_NO_COALESCE = 64
 MGGCN_F_CACHE_L0 = 128
+MGGCN_F_IPC = 256
+MGGCN_IPC_BLOB_BYTES = 128
 PROFILE_CLASSES = ("spmm", "gemm", "loss", "adam", "bcast", "allreduce", "other")
 
 EXPORTS = (
@@ -32,7 +34,7 @@ EXPORTS = (
     "mggcn_backward", "mggcn_step", "mggcn_get_loss", "mggcn_get_grad", "mggcn_get_adam", "mggcn_set_adam",
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
-    "mggcn_prefetch",
+    "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect",
 )
 
 
@@ -65,6 +67,8 @@ def _load():
         "mggcn_workspace_bytes": ([P, i32, i32, P, u32, P], ctypes.c_int),
         "mggcn_model_create": ([P, i32, i32, P, u32, P, P, sz, up, up, P], ctypes.c_int),
         "mggcn_nccl_unique_id": ([P], ctypes.c_int),
+        "mggcn_ipc_export": ([P, P], ctypes.c_int),
+        "mggcn_ipc_connect": ([P, P], ctypes.c_int),
         "mggcn_set_weights": ([P, i32, P], ctypes.c_int),
         "mggcn_get_weights": ([P, i32, P], ctypes.c_int),
         "mggcn_forward": ([P, P, i64, P, P, P], ctypes.c_int),
@@ -194,6 +198,21 @@ def mggcn_nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(_lib.mggcn_nccl_unique_id(buf))
     return buf.raw
+
+
+def mggcn_ipc_export(m) -> bytes:
+    buf = ctypes.create_string_buffer(MGGCN_IPC_BLOB_BYTES)
+    _check(_lib.mggcn_ipc_export(m, buf))
+    return buf.raw
+
+
+def mggcn_ipc_connect(m, blobs):
+    """blobs: the P exports in rank order."""
+    raw = b"".join(blobs)
+    if len(raw) != MGGCN_IPC_BLOB_BYTES * len(blobs):
+        raise ValueError("mggcn_ipc_connect: each blob must be MGGCN_IPC_BLOB_BYTES long")
+    buf = ctypes.create_string_buffer(raw, len(raw))
+    _check(_lib.mggcn_ipc_connect(m, buf))
 
 
 def mggcn_model_create(parts, dims, flags, nccl_id, workspace_ptr, ws_bytes, compute_stream, comm_stream):

@@ -105,4 +105,18 @@ cudaError_t launch_sum_f64(const double* in, int nin, double* out, cudaStream_t 
 cudaError_t launch_scale_rows(const float* in, int64_t ldi, float* out, int64_t ldo, int64_t n, int width,
                               const float* rowscale, cudaStream_t s);
 
+// ------------------------------------------------------------------- IPC
+// (ipc.cu) stream memory operations, allocation base lookup and rank-ordered
+// sums over peer buffers mapped with cudaIpcOpenMemHandle.
+struct PtrArrayF { const float* p[64]; };
+struct PtrArrayD { const double* p[64]; };
+struct PtrArrayI { const int64_t* p[64]; };
+bool ipc_stream_memops_available();
+cudaError_t stream_write_u32(cudaStream_t s, uint32_t* addr, uint32_t value);
+cudaError_t stream_wait_u32(cudaStream_t s, const uint32_t* addr, uint32_t value);
+int ipc_alloc_base(const void* ptr, void** base, size_t* size);
+cudaError_t launch_sum_ranks_f32(const float* const* in, int nin, float* out, int64_t count, cudaStream_t s);
+cudaError_t launch_sum_ranks_scalar(const double* const* in_d, const int64_t* const* in_i, int nin, double* out_d,
+                                    int64_t* out_i, cudaStream_t s);
+
 }  // namespace mggcn

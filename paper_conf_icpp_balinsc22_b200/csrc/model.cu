@@ -174,6 +174,18 @@ struct mggcn_model_s {
     int layer_ids[64];
     bool t0_valid = false;          // MGGCN_F_CACHE_L0: T0 = Â'^T X computed
     // input prefetch (mggcn_prefetch): copy stream, staging chunk, buffer events
+    // SM-free IPC exchange (MGGCN_F_IPC, NEXT-1): peers' workspaces, sequence flags
+    uint32_t* flags_dev = nullptr;  // [0] spmm ready [1] spmm done [2] wg ready [3] wg done [4] sc ready [5] sc done
+    float* WGp = nullptr;           // this rank's W_G partial (read by peers)
+    char* ws_base = nullptr;        // this rank's workspace
+    std::vector<char*> peer_ws;     // peers' workspaces mapped here (own = ws_base)
+    std::vector<void*> ipc_opened;
+    void* ipc_alloc = nullptr;
+    size_t ipc_alloc_off = 0;
+    bool ipc = false, ipc_connected = false;
+    size_t ws_bytes = 0;             // planned workspace bytes
+    size_t sym_bytes = 0;            // symmetric region [0, sym_bytes) (IPC peers must agree)
+    uint32_t spmm_seq = 0, wg_seq = 0, sc_seq = 0;
     cudaStream_t cp = nullptr;
     float* xstage = nullptr;
     int64_t xstage_floats = 0;
@@ -266,6 +278,20 @@ int check_dims(int L, const int32_t* dims) {
 // Lays out (or sizes, when bump.base == nullptr) every device buffer.
 void plan_buffers(mggcn_model_s* m, Bump& b) {
     const int L = m->L;
+    // ---- symmetric region: identical offsets on every rank of a multi-process run
+    // (sizes use max_j n_j), so peers address each other's buffers by offset (IPC)
+    m->flags_dev = b.take<uint32_t>(64);
+    m->WGp = b.take<float>(m->wtotal);
+    for (auto& r : m->ranks) {
+        r.loss_local = b.take<double>(1);
+        r.ntrain_local = b.take<int64_t>(1);
+        for (int k = 0; k < 2; ++k) r.Xbuf[k] = b.take<float>(m->max_rows_j * m->ld[0]);
+        r.HWB = b.take<float>(m->max_rows_j * std::max<int64_t>(m->hw_ld, 4));
+        r.AHWB.assign(L, nullptr);
+        for (int l = 0; l < L; ++l) r.AHWB[l] = b.take<float>(m->max_rows_j * m->ld[l + 1]);
+    }
+    m->sym_bytes = b.off;   // same on every rank (sizes use max_rows_j)
+    // ---- private region
     m->W = b.take<float>(m->wtotal);
     m->Mom = b.take<float>(m->wtotal);
     m->Vel = b.take<float>(m->wtotal);
@@ -309,20 +335,14 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             }
         }
         r.inv_deg = b.take<float>(r.rows);
-        for (int k = 0; k < 2; ++k) {
-            r.Xbuf[k] = b.take<float>(r.rows * m->ld[0]);
-            r.ybuf[k] = b.take<int32_t>(r.rows);
-        }
+        for (int k = 0; k < 2; ++k) r.ybuf[k] = b.take<int32_t>(r.rows);
         r.Xs = r.Xbuf[0];
         r.y = r.ybuf[0];
         r.T0 = m->order[0] == S_ORDER ? b.take<float>(r.rows * m->ld[0]) : nullptr;
-        r.HWB = b.take<float>(r.rows * std::max<int64_t>(m->hw_ld, 4));
         if (P > 1) {
             r.BC[0] = b.take<float>(m->max_rows_j * m->bc_ld);
             r.BC[1] = b.take<float>(m->max_rows_j * m->bc_ld);
         }
-        r.AHWB.assign(L, nullptr);
-        for (int l = 0; l < L; ++l) r.AHWB[l] = b.take<float>(r.rows * m->ld[l + 1]);
         int64_t slots = 0;
         for (int j = 0; j < P; ++j) {
             slots = std::max(slots, r.hF[j].nslots);
@@ -330,8 +350,6 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
         }
         r.spmm_partial = b.take<float>(slots * std::min<int64_t>(m->bc_ld, 512));
         r.ce_partial = b.take<double>(kCeBlocks);
-        r.loss_local = b.take<double>(1);
-        r.ntrain_local = b.take<int64_t>(1);
         r.WG_local = (m->nlocal > 1) ? b.take<float>(m->wtotal) : nullptr;
         // split-K partials for W_G (Eq. 10)
         size_t gp = 0;
@@ -376,6 +394,8 @@ int upload_static(mggcn_model_s* m) {
             if (r.BC[s]) CK(cudaMemsetAsync(r.BC[s], 0, sizeof(float) * m->max_rows_j * m->bc_ld, m->cs));
     }
     CK(cudaMemsetAsync(m->W, 0, sizeof(float) * m->wtotal, m->cs));
+    CK(cudaMemsetAsync(m->flags_dev, 0, sizeof(uint32_t) * 64, m->cs));
+    CK(cudaMemsetAsync(m->WGp, 0, sizeof(float) * m->wtotal, m->cs));
     for (int l = 0; l < m->L; ++l) {
         CK(cudaMemsetAsync(m->Wt_hi[l], 0, sizeof(float) * m->d[l + 1] * m->ld[l], m->cs));
         CK(cudaMemsetAsync(m->Wt_lo[l], 0, sizeof(float) * m->d[l + 1] * m->ld[l], m->cs));
@@ -526,6 +546,26 @@ int refresh_weight_splits(mggcn_model_s* m) {
     return MGGCN_OK;
 }
 
+// --------------------------------------------------------------------- IPC
+// Address of `mine` (a buffer in this rank's symmetric region) inside peer q.
+template <typename T>
+T* peer_ptr(mggcn_model_s* m, int q, T* mine) {
+    return reinterpret_cast<T*>(m->peer_ws[q] + (reinterpret_cast<char*>(mine) - m->ws_base));
+}
+
+int ipc_signal(mggcn_model_s* m, cudaStream_t s, int flag, uint32_t seq) {
+    CK(stream_write_u32(s, m->flags_dev + flag, seq));
+    return MGGCN_OK;
+}
+
+// stream s waits until every peer's flag >= seq
+int ipc_wait_peers(mggcn_model_s* m, cudaStream_t s, int flag, uint32_t seq) {
+    const int me = m->ranks[0].rank;
+    for (int q = 0; q < m->P; ++q)
+        if (q != me) CK(stream_wait_u32(s, peer_ptr(m, q, m->flags_dev) + flag, seq));
+    return MGGCN_OK;
+}
+
 // --------------------------------------------------------- staged SpMM
 // C_r (+)= sum_j T_rj · S_j over stages; S_j = src(j) rows of rank j.
 // Local stage first, then ascending j (reading C13); broadcast q goes into
@@ -552,6 +592,41 @@ int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const flo
 
 int remote_index(int q, int self) { return q < self ? q : q - 1; }
 
+// NEXT-1 (SM-free exchange): every receiver PULLS the peers' blocks with copy
+// engines in rotated order (stage s reads block (i + s) mod P, so each GPU
+// serves one reader per step); sequence flags order producer -> pull -> reuse.
+int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
+    const int P = m->P;
+    Rank& r = m->ranks[0];
+    const int me = r.rank;
+    const uint32_t seq = ++m->spmm_seq;
+    const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
+    float* mysrc = job.src(m, r, job.ctx);
+    CK(cudaEventRecord(m->ev_begin, m->cs));            // my source produced; BC slots free
+    RC(ipc_signal(m, m->cs, 0, seq));                   // peers may pull my block
+    CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
+    if (r.rows > 0) RC(launch_stage(m, r, job, me, mysrc, 0));
+    for (int st = 1; st < P; ++st) {
+        const int q = (me + st) % P, k = st - 1, slot = k & 1;
+        {
+            ProfScope ps(m, PC_BCAST, m->ms);
+            if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+            CK(stream_wait_u32(m->ms, peer_ptr(m, q, m->flags_dev) + 0, seq));   // block q is ready
+            const size_t bytes = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width * sizeof(float);
+            if (!nob && bytes) CK(cudaMemcpyAsync(r.BC[slot], peer_ptr(m, q, mysrc), bytes, cudaMemcpyDefault, m->ms));
+            CK(cudaEventRecord(r.ev_bc[slot], m->ms));
+        }
+        CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
+        if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], SPMM_ACCUM | (st == P - 1 ? SPMM_LAST : 0)));
+        CK(cudaEventRecord(r.ev_free[slot], m->cs));
+    }
+    RC(ipc_signal(m, m->ms, 1, seq));                   // I have read every peer's block
+    CK(cudaEventRecord(m->ev_comm_end, m->ms));
+    CK(cudaStreamWaitEvent(m->cs, m->ev_comm_end, 0));
+    RC(ipc_wait_peers(m, m->cs, 1, seq));               // ... and the peers have read mine
+    return MGGCN_OK;
+}
+
 int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
     const int P = m->P;
     const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
@@ -560,6 +635,7 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
         CK(cudaEventRecord(m->ev_begin, m->cs));
         CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
     }
+    if (m->ipc) return staged_spmm_ipc(m, job);
     // local stage
     for (auto& r : m->ranks) {
         if (r.rows == 0) continue;
@@ -622,7 +698,21 @@ float* src_AHWB(mggcn_model_s*, Rank& r, const void* ctx) { return r.AHWB[*stati
 // on the comm stream fenced by events, or a copy when P == 1.
 int reduce_scalars(mggcn_model_s* m, bool ntrain) {
     Rank& r = m->ranks[0];
-    if (m->comm) {
+    if (m->ipc) {
+        // every rank sums all P partials in rank order (identical results on all ranks)
+        const uint32_t seq = ++m->sc_seq;
+        RC(ipc_signal(m, m->cs, 4, seq));
+        RC(ipc_wait_peers(m, m->cs, 4, seq));
+        std::vector<const double*> pd(m->P);
+        std::vector<const int64_t*> pi(m->P);
+        for (int q = 0; q < m->P; ++q) {
+            pd[q] = peer_ptr(m, q, r.loss_local);
+            pi[q] = peer_ptr(m, q, r.ntrain_local);
+        }
+        if (ntrain) CK(launch_sum_ranks_scalar(nullptr, pi.data(), m->P, nullptr, m->ntrain, m->cs));
+        else CK(launch_sum_ranks_scalar(pd.data(), nullptr, m->P, m->loss_sum, nullptr, m->cs));
+        RC(ipc_signal(m, m->cs, 5, seq));
+    } else if (m->comm) {
         CK(cudaEventRecord(m->ev_tmp, m->cs));
         CK(cudaStreamWaitEvent(m->ms, m->ev_tmp, 0));
         if (ntrain) NK(ncclAllReduce(r.ntrain_local, m->ntrain, 1, ncclInt64, ncclSum, m->comm, m->ms));
@@ -851,6 +941,8 @@ static void destroy(mggcn_model_s* m) {
     }
     for (auto e : m->prof_pool) cudaEventDestroy(e);
     if (m->comm) ncclCommDestroy(m->comm);
+    for (void* p : m->ipc_opened)
+        if (p) cudaIpcCloseMemHandle(p);
     delete m;
 }
 
@@ -878,8 +970,19 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
         delete m;
         return rc;
     }
-    if (m->P > 1 && nlocal == 1 && !nccl_id128) {
-        set_error("model_create: P > 1 with nlocal = 1 needs an NCCL unique id");
+    m->ipc = (flags & MGGCN_F_IPC) && m->P > 1 && nlocal == 1;
+    if ((flags & MGGCN_F_IPC) && (nlocal != 1 || nccl_id128)) {
+        set_error("model_create: MGGCN_F_IPC needs nlocal = 1 and nccl_id128 = NULL");
+        delete m;
+        return MGGCN_EINVAL;
+    }
+    if (m->ipc && !ipc_stream_memops_available()) {
+        set_error("model_create: MGGCN_F_IPC needs cuStreamWaitValue32 / cuStreamWriteValue32");
+        delete m;
+        return MGGCN_EUNSUPPORTED;
+    }
+    if (m->P > 1 && nlocal == 1 && !nccl_id128 && !m->ipc) {
+        set_error("model_create: P > 1 with nlocal = 1 needs an NCCL unique id (or MGGCN_F_IPC)");
         delete m;
         return MGGCN_EINVAL;
     }
@@ -893,6 +996,8 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
     Bump b;
     b.base = static_cast<char*>(workspace);
     plan_buffers(m, b);
+    m->ws_base = static_cast<char*>(workspace);
+    m->ws_bytes = sz.off;
     m->cs = reinterpret_cast<cudaStream_t>(compute_stream);
     m->ms = reinterpret_cast<cudaStream_t>(comm_stream);
     auto fail = [&](int code) {
@@ -920,7 +1025,7 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
     if (rc != MGGCN_OK) return fail(rc);
     rc = plan_gemms(m);
     if (rc != MGGCN_OK) return fail(rc);
-    if (m->P > 1 && nlocal == 1) {
+    if (m->P > 1 && nlocal == 1 && !m->ipc) {
         ncclUniqueId id;
         std::memcpy(&id, nccl_id128, 128);
         ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
@@ -942,6 +1047,80 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
 }
 
 extern "C" void mggcn_model_free(mggcn_model m) { destroy(m); }
+
+// ------------------------------------------------------------------ IPC
+// Blob layout (MGGCN_IPC_BLOB_BYTES = 128): cudaIpcMemHandle_t (64 B) of the
+// allocation holding the workspace | uint64 offset of the workspace in it |
+// int32 rank | int32 P | uint64 symmetric-region bytes | zero padding.
+namespace {
+struct IpcBlob {
+    cudaIpcMemHandle_t h;
+    uint64_t off;
+    int32_t rank, P;
+    uint64_t ws_bytes;
+    char pad[128 - sizeof(cudaIpcMemHandle_t) - 24];
+};
+static_assert(sizeof(IpcBlob) == MGGCN_IPC_BLOB_BYTES, "IPC blob size");
+}  // namespace
+
+extern "C" int mggcn_ipc_export(mggcn_model m, void* blob) {
+    MODEL_GUARD(m);
+    if (!m->ipc || !blob) {
+        set_error("ipc_export: model not created with MGGCN_F_IPC (P > 1), or NULL blob");
+        return MGGCN_EINVAL;
+    }
+    void* base = nullptr;
+    size_t size = 0;
+    if (ipc_alloc_base(m->ws_base, &base, &size)) {
+        set_error("ipc_export: cannot find the allocation holding the workspace");
+        return MGGCN_ECUDA;
+    }
+    IpcBlob b{};
+    if (cudaIpcGetMemHandle(&b.h, base) != cudaSuccess) {
+        set_error(std::string("ipc_export: cudaIpcGetMemHandle: ") + cudaGetErrorString(cudaGetLastError()));
+        return MGGCN_ECUDA;
+    }
+    b.off = (uint64_t)(m->ws_base - static_cast<char*>(base));
+    b.rank = m->ranks[0].rank;
+    b.P = m->P;
+    b.ws_bytes = m->sym_bytes;
+    std::memcpy(blob, &b, sizeof b);
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_ipc_connect(mggcn_model m, const void* blobs) {
+    MODEL_GUARD(m);
+    if (!m->ipc || !blobs || m->ipc_connected) {
+        set_error("ipc_connect: not an MGGCN_F_IPC model, NULL blobs, or already connected");
+        return MGGCN_EINVAL;
+    }
+    const int P = m->P, me = m->ranks[0].rank;
+    std::vector<IpcBlob> bl(P);
+    std::memcpy(bl.data(), blobs, sizeof(IpcBlob) * P);
+    for (int q = 0; q < P; ++q)
+        if (bl[q].rank != q || bl[q].P != P || bl[q].ws_bytes != m->sym_bytes) {
+            set_error("ipc_connect: blobs must be rank-ordered exports of models with the same P and plan");
+            return MGGCN_EINVAL;
+        }
+    m->peer_ws.assign(P, nullptr);
+    m->ipc_opened.assign(P, nullptr);
+    for (int q = 0; q < P; ++q) {
+        if (q == me) {
+            m->peer_ws[q] = m->ws_base;
+            continue;
+        }
+        void* p = nullptr;
+        if (cudaIpcOpenMemHandle(&p, bl[q].h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+            set_error(std::string("ipc_connect: cudaIpcOpenMemHandle(rank ") + std::to_string(q) +
+                      "): " + cudaGetErrorString(cudaGetLastError()));
+            return MGGCN_ECUDA;
+        }
+        m->ipc_opened[q] = p;
+        m->peer_ws[q] = static_cast<char*>(p) + bl[q].off;
+    }
+    m->ipc_connected = true;
+    return MGGCN_OK;
+}
 
 // ---------------------------------------------------------------- weights
 static int check_layer(mggcn_model_s* m, int32_t layer) {
@@ -1062,7 +1241,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
             // X is not read again (layer 0 starts from the cached T0): only the labels
             for (auto& r : m->ranks)
                 if (r.rows) CK(cudaMemcpyAsync(r.y, y + r.row_off, sizeof(int32_t) * r.rows, cudaMemcpyDefault, m->cs));
-        } else if (device_zero_copy(m, X, ldx)) {
+        } else if (!m->ipc && device_zero_copy(m, X, ldx)) {
             // device X already in the padded layout: layer 0 reads it in place (it must stay
             // valid until this epoch's backward has run); labels are still copied
             RC(use_external_input(m, X));
@@ -1102,6 +1281,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
         }
     }
     // ---- loss: |T|, logits out, fused CE fwd+bwd in place (Eq. 19)
+    if (m->ipc && m->sc_seq) RC(ipc_wait_peers(m, m->cs, 5, m->sc_seq));   // peers read my last scalars
     for (auto& r : m->ranks)
         CK(launch_count_labelled(r.y, r.rows, reinterpret_cast<int64_t*>(r.ce_partial), r.ntrain_local, m->cs));
     RC(reduce_all(m, true));
@@ -1149,6 +1329,10 @@ extern "C" int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, c
     } else if (!y_local || ldx < m->d[0]) {
         set_error("forward: NULL y or ldx < d_0");
         return MGGCN_EINVAL;
+    }
+    if (m->ipc && !m->ipc_connected) {
+        set_error("forward: MGGCN_F_IPC model needs mggcn_ipc_connect first");
+        return MGGCN_ESTATE;
     }
     RC(poison(m, wait_wg(m)));
     int rc = forward_impl(m, X_local, ldx, y_local, loss, logits_local);
@@ -1209,7 +1393,9 @@ static int wgrad_reduce(mggcn_model_s* m, int l) {
     // per-rank partial W_G (Eq. 10) -> sum over ranks (reading C23)
     const int64_t din = m->d[l], dout = m->d[l + 1], ld = m->ld[l + 1];
     for (auto& r : m->ranks) {
-        float* dst = (m->nlocal > 1 ? r.WG_local : m->WG) + m->woff[l];
+        float* dst = (m->nlocal > 1 ? r.WG_local : m->ipc ? m->WGp : m->WG) + m->woff[l];
+        if (m->ipc && m->wg_seq >= (uint32_t)m->L)
+            RC(ipc_wait_peers(m, m->cs, 3, m->wg_seq + 1 - m->L));   // peers finished reading this slice
         if (r.has_wgrad[l]) {
             {
                 ProfScope ps(m, PC_GEMM, m->cs);
@@ -1225,6 +1411,22 @@ static int wgrad_reduce(mggcn_model_s* m, int l) {
         for (auto& r : m->ranks) in.push_back(r.WG_local + m->woff[l]);
         ProfScope ps(m, PC_ALLRED, m->cs);
         CK(launch_sum_buffers(in.data(), (int)in.size(), m->WG + m->woff[l], din * ld, m->cs));
+    } else if (m->ipc) {
+        // W_G all-reduce as a pull-sum over peer memory, rank order (bitwise identical on all ranks)
+        const uint32_t seq = ++m->wg_seq;
+        RC(ipc_signal(m, m->cs, 2, seq));
+        CK(cudaEventRecord(m->ev_tmp, m->cs));
+        CK(cudaStreamWaitEvent(m->ms, m->ev_tmp, 0));
+        {
+            ProfScope ps(m, PC_ALLRED, m->ms);
+            RC(ipc_wait_peers(m, m->ms, 2, seq));
+            std::vector<const float*> in(m->P);
+            for (int q = 0; q < m->P; ++q) in[q] = peer_ptr(m, q, m->WGp) + m->woff[l];
+            CK(launch_sum_ranks_f32(in.data(), m->P, m->WG + m->woff[l], din * ld, m->ms));
+        }
+        RC(ipc_signal(m, m->ms, 3, seq));
+        CK(cudaEventRecord(m->ev_wg, m->ms));
+        m->need_wg_wait = true;
     } else if (m->comm) {
         CK(cudaEventRecord(m->ev_tmp, m->cs));
         CK(cudaStreamWaitEvent(m->ms, m->ev_tmp, 0));

@@ -1,8 +1,9 @@
 """Multi-process plumbing around the C ABI (one process per GPU).
 
 torch.distributed only carries the 128-byte ncclUniqueId (the library builds
-its own NCCL communicator, because torch does not expose its ncclComm_t) and
-the max-over-ranks timing.  All data movement of the hot path is inside the
+its own NCCL communicator, because torch does not expose its ncclComm_t) or
+the 128-byte CUDA-IPC descriptors of the MGGCN_F_IPC backend, and the
+max-over-ranks timing.  All data movement of the hot path is inside the
 library (P-stage broadcasts, W_G all-reduce).
 """
 from __future__ import annotations
@@ -13,6 +14,15 @@ def share_nccl_id(dist, make_id):
     obj = [make_id() if dist.get_rank() == 0 else None]
     dist.broadcast_object_list(obj, src=0)
     return obj[0]
+
+
+def ipc_exchange(dist):
+    """Returns f(blob) -> the P MGGCN_F_IPC blobs in rank order (all_gather over `dist`)."""
+    def f(blob):
+        out = [None] * dist.get_world_size()
+        dist.all_gather_object(out, blob)
+        return out
+    return f
 
 
 def local_rows(perm, p, rank, M):

@@ -7,10 +7,11 @@ from __future__ import annotations
 
 import numpy as np
 
-from . import (MGGCN_F_OVERLAP, mggcn_backward, mggcn_prefetch, mggcn_epoch_work, mggcn_forward, mggcn_get_adam, mggcn_get_grad,
-               mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free, mggcn_load_csr,
-               mggcn_model_create, mggcn_model_free, mggcn_part_free, mggcn_part_info, mggcn_partition,
-               mggcn_set_adam, mggcn_set_weights, mggcn_step, mggcn_workspace_bytes)
+from . import (MGGCN_F_IPC, MGGCN_F_OVERLAP, mggcn_backward, mggcn_epoch_work, mggcn_forward, mggcn_get_adam,
+               mggcn_get_grad, mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free,
+               mggcn_ipc_connect, mggcn_ipc_export, mggcn_load_csr, mggcn_model_create, mggcn_model_free,
+               mggcn_part_free, mggcn_part_info, mggcn_partition, mggcn_prefetch, mggcn_set_adam,
+               mggcn_set_weights, mggcn_step, mggcn_workspace_bytes)
 
 
 class GCN:
@@ -20,7 +21,10 @@ class GCN:
     """
 
     def __init__(self, n, rowptr, col, vals, dims, P=1, rank=0, perm_seed=0, flags=MGGCN_F_OVERLAP,
-                 loopback=False, nccl_id=None, device=None, graph=None):
+                 loopback=False, nccl_id=None, device=None, graph=None, comm="nccl", ipc_exchange=None):
+        """comm = "nccl" (nccl_id from mggcn_nccl_unique_id, shared by the caller) or "ipc"
+        (MGGCN_F_IPC: peers map each other's workspaces; ipc_exchange(blob) -> list of the P
+        blobs in rank order, e.g. dist.ipc_exchange over torch.distributed)."""
         import torch
         self.torch = torch
         self.dims = tuple(int(d) for d in dims)
@@ -39,12 +43,20 @@ class GCN:
         self.row0 = 0 if loopback else int(self.p[rank])
         self.rows = n if loopback else int(self.p[rank + 1] - self.p[rank])
         self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        self.comm = "loopback" if loopback or P == 1 else comm
+        if self.comm == "ipc":
+            if ipc_exchange is None:
+                raise ValueError("GCN(comm='ipc') needs ipc_exchange")
+            flags |= MGGCN_F_IPC
+            nccl_id = None
         self.ws_bytes = mggcn_workspace_bytes(self.parts, self.dims, flags)
         self.workspace = torch.empty(self.ws_bytes, dtype=torch.uint8, device=self.device)
         self.cs = torch.cuda.Stream(device=self.device)
         self.ms = torch.cuda.Stream(device=self.device)
         self.m = mggcn_model_create(self.parts, self.dims, flags, nccl_id, self.workspace.data_ptr(), self.ws_bytes,
                                     self.cs.cuda_stream, self.ms.cuda_stream)
+        if self.comm == "ipc":
+            mggcn_ipc_connect(self.m, ipc_exchange(mggcn_ipc_export(self.m)))
 
     # ---------------------------------------------------------------- data
     @property

@@ -231,6 +231,14 @@ int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int64_t ldb, in
                      int64_t ldo);
 int mggcn_debug_gemm(int32_t op, int64_t M, int64_t N, int64_t K, const float* A, int64_t lda, const float* B,
                      int64_t ldb, float* C, int64_t ldc, uint32_t flags, uintptr_t stream);
+/* mggcn_debug_layer: copies the layer-l activation buffer AHWB_l (this
+ * model's rows, all n in loopback; d_{l+1} columns) into dst (host or device,
+ * row stride ld >= d_{l+1}); synchronises.  Contents (Eq. 17-21):
+ * after mggcn_forward, H_{l+1} = ReLU(Z_l) for l < L-1 and the softmax-CE
+ * gradient for l = L-1; after mggcn_backward, for l < L-1, Z_{G,l} = dLoss/dZ_l
+ * (Eq. 8 / 21), pre-scaled row-wise by inv_deg when layer l is GeMM-first (its
+ * backward SpMM then runs on the pattern, reading C20).  EINVAL: bad layer/ld. */
+int mggcn_debug_layer(mggcn_model m, int32_t layer, float* dst, int64_t ld);
 
 #ifdef __cplusplus
 }

@@ -60,6 +60,7 @@ def _L():
         i64, i32, u64, dbl = ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_double
         lib.orc_permutation.argtypes = [i64, u64, P]
         lib.orc_splitmix64_next.argtypes = [P]
+        lib.orc_csr_order.argtypes = [i64, i64, P, P, P, P]
         lib.orc_splitmix64_next.restype = u64
         for s in ("f32", "f64"):
             getattr(lib, f"orc_spmm_{s}").argtypes = [i64, P, P, P, P, i64, i64, P, i64]
@@ -145,12 +146,17 @@ class PermutedGraph:
 
 
 def _csr_from_triplets(n, rows, cols, tie, vals):
-    """Sort by (row, col, tie) and build a CSR (numpy lexsort = library sort)."""
-    order = np.lexsort((tie, cols, rows))
-    rowptr = np.zeros(n + 1, dtype=np.int64)
-    counts = np.bincount(rows, minlength=n)
-    rowptr[1:] = np.cumsum(counts)
-    return CSR(rowptr, cols[order].astype(np.int64), vals[order]), order
+    """Sort by (row, col, tie) and build a CSR.  `tie` must be ascending in
+    input order (the original CSR position, O4's tie rule), so a stable sort
+    by (row, col) is that order (orc_csr_order: stable bucket sort by row, then
+    a stable sort of each row by column)."""
+    assert tie.shape[0] < 2 or np.all(np.diff(tie) > 0)
+    rows = np.ascontiguousarray(rows, dtype=np.int64)
+    cols = np.ascontiguousarray(cols, dtype=np.int64)
+    rowptr = np.empty(n + 1, dtype=np.int64)
+    order = np.empty(rows.shape[0], dtype=np.int64)
+    _L().orc_csr_order(n, rows.shape[0], _p(rows), _p(cols), _p(rowptr), _p(order))
+    return CSR(rowptr, cols[order], vals[order]), order
 
 
 def permute_graph(n, rowptr, col, vals=None, seed=0, dtype=np.float32) -> PermutedGraph:

@@ -13,9 +13,11 @@
 //
 // Parity pins for every function are listed in oracle/__init__.py and
 // DESIGN.md §4 (tests/test_oracle_*.py).
+#include <algorithm>
 #include <cmath>
 #include <cstdint>
 #include <cstring>
+#include <vector>
 
 namespace {
 
@@ -149,6 +151,26 @@ void orc_permutation(int64_t n, uint64_t seed, int64_t* perm) {
         const int64_t tmp = perm[k];
         perm[k] = perm[j];
         perm[j] = tmp;
+    }
+}
+
+// CSR from triplets (O4's ordering): entries sorted by (row, col) with ties
+// kept in input order.  Plain bucket sort: count per row, scatter in input
+// order (stable), then a stable sort of each row by column.  order[k] = input
+// index of the k-th output entry; rowptr int64[n+1].
+void orc_csr_order(int64_t n, int64_t nnz, const int64_t* rows, const int64_t* cols, int64_t* rowptr,
+                   int64_t* order) {
+    std::vector<int64_t> next(n + 1, 0);
+    for (int64_t e = 0; e < nnz; ++e) next[rows[e] + 1] += 1;
+    for (int64_t r = 0; r < n; ++r) next[r + 1] += next[r];
+    for (int64_t r = 0; r <= n; ++r) rowptr[r] = next[r];
+    for (int64_t e = 0; e < nnz; ++e) order[next[rows[e]]++] = e;
+    std::vector<std::pair<int64_t, int64_t>> row;   // (col, input index): ties by input index = stable
+    for (int64_t r = 0; r < n; ++r) {
+        row.clear();
+        for (int64_t k = rowptr[r]; k < rowptr[r + 1]; ++k) row.emplace_back(cols[order[k]], order[k]);
+        std::sort(row.begin(), row.end());
+        for (int64_t k = rowptr[r]; k < rowptr[r + 1]; ++k) order[k] = row[k - rowptr[r]].second;
     }
 }
 

@@ -34,7 +34,7 @@ EXPORTS = (
     "mggcn_backward", "mggcn_step", "mggcn_get_loss", "mggcn_get_grad", "mggcn_get_adam", "mggcn_set_adam",
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
-    "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect",
+    "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer",
 )
 
 
@@ -84,6 +84,7 @@ def _load():
         "mggcn_part_free": ([P], None),
         "mggcn_model_free": ([P], None),
         "mggcn_debug_spmm": ([P, i32, P, i64, i32, P, i64], ctypes.c_int),
+        "mggcn_debug_layer": ([P, i32, P, i64], ctypes.c_int),
         "mggcn_debug_gemm": ([i32, i64, i64, i64, P, i64, P, i64, P, i64, u32, up], ctypes.c_int),
         "mggcn_kernel_launch_count": ([], ctypes.c_int64),
         "mggcn_reset_cache": ([P], ctypes.c_int),
@@ -314,6 +315,13 @@ def mggcn_model_free(m):
 
 def mggcn_debug_spmm(m, direction, B, ldb, width, out, ldo):
     _check(_lib.mggcn_debug_spmm(m, direction, _ptr(B), ldb, width, _ptr(out), ldo))
+
+
+def mggcn_debug_layer(m, layer, shape):
+    """Host copy (rows x d_{l+1}) of AHWB_l (see include/mggcn.h)."""
+    out = np.empty(shape, dtype=np.float32)
+    _check(_lib.mggcn_debug_layer(m, layer, _ptr(out), shape[1]))
+    return out
 
 
 def mggcn_debug_gemm(op, M, N, K, A, lda, B, ldb, C, ldc, flags=0, stream=0):

@@ -1541,6 +1541,25 @@ extern "C" int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* gathe
 }
 
 // ------------------------------------------------------------- test hooks
+extern "C" int mggcn_debug_layer(mggcn_model m, int32_t layer, float* dst, int64_t ld) {
+    MODEL_GUARD(m);
+    RC(check_layer(m, layer));
+    const int64_t w = m->d[layer + 1];
+    if (!dst || ld < w) {
+        set_error("debug_layer: NULL dst or ld < d_{l+1}");
+        return MGGCN_EINVAL;
+    }
+    auto body = [&]() -> int {
+        for (auto& r : m->ranks)
+            if (r.rows)
+                CK(cudaMemcpy2DAsync(dst + r.row_off * ld, ld * 4, r.AHWB[layer],
+                                     m->ld[layer + 1] * 4, w * 4, r.rows, cudaMemcpyDefault, m->cs));
+        CK(cudaStreamSynchronize(m->cs));
+        return MGGCN_OK;
+    };
+    return poison(m, body());
+}
+
 extern "C" int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int64_t ldb, int32_t width, float* out,
                                 int64_t ldo) {
     MODEL_GUARD(m);

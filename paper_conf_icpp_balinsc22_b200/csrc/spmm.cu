@@ -14,6 +14,7 @@
 //   - epilogue fused: accumulate into the previous stage's output (RMW), and
 //     on the last stage the 1/deg row scale (Eq. 2 for pattern-only graphs)
 //     and ReLU (Eq. 7 / Eq. 18 in place).
+#include <cstdio>
 #include <cstdlib>
 
 #include "kernels.cuh"
@@ -292,6 +293,14 @@ cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4
     }
     MGGCN_SPMM_SHAPES(MGGCN_PICK)
 #undef MGGCN_PICK
+    {   // experiment hook: MGGCN_SPMM_SHAPE="G,CH" forces an instantiated shape that covers w4
+        static int fg = -1, fc = 0;
+        if (fg < 0) {
+            fg = 0;
+            if (const char* e = getenv("MGGCN_SPMM_SHAPE")) sscanf(e, "%d,%d", &fg, &fc);
+        }
+        if (fg > 0 && fg * fc >= w4) { bg = fg; bc = fc; }
+    }
 #define MGGCN_CALL(g, c) \
     if (bg == g && bc == c) return launch_gc<g, c>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, s);
     MGGCN_SPMM_SHAPES(MGGCN_CALL)

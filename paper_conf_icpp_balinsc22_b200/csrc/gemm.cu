@@ -19,6 +19,7 @@
 // accumulator[2] MMA -> epilogue (double-buffered TMEM, 2 x 128 columns).
 #include <cuda.h>
 
+#include <cstdio>
 #include <cstdlib>
 #include <mutex>
 
@@ -54,6 +55,7 @@ struct KParams {
     const float* rowscale;
     int flags;
     int op2;
+    uint32_t desc_mn[3];
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -388,6 +390,175 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     }
 }
 
+// ------------------------------------------------ wgrad, MN-major variant
+// Same product and split-K tiling as gemm_wgrad_kernel, but the K-outer
+// operands are consumed in place: tcgen05 kind::tf32 accepts MN-major
+// shared-memory operands in the 128B-swizzle / 32B-atom layout
+// (SWIZZLE_128B_BASE32B: LBO = stride of 32-float MN chunks, SBO = stride of
+// 4-row k groups), which TMA writes directly (CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B,
+// boxes of 32 MN-contiguous floats x 16 k rows).  No transpose.
+// 3xTF32: the MMA reads an fp32 operand as tf32 by ignoring the low 13
+// mantissa bits, i.e. as hi = x & 0xFFFFE000 -- so the raw TMA tile IS the hi
+// operand and 4 warps only compute lo = x - hi into a separate ring (1xTF32:
+// the raw tile is rounded to nearest in place instead).  Rings: 6 raw stages
+// (TMA -> MMA, 24 KB) and 2 lo stages; 192 threads: warps 0-3 lo + epilogue,
+// warp 4 TMA, warp 5 TMEM allocator + MMA issuer.
+constexpr int kMnBK = 16;
+constexpr int kMnNR = 6, kMnNL = 2;
+constexpr int kMnRaw = 24576;                    // A 8K (4 boxes) | B 16K (<= 8 boxes)
+constexpr int kMnLo0 = kMnNR * kMnRaw;
+constexpr int kMnBars = kMnLo0 + kMnNL * kMnRaw;
+constexpr int kMnSmem = kMnBars + 256 + 1024;
+#ifndef MGGCN_MN_LO_WARPS
+#define MGGCN_MN_LO_WARPS 12
+#endif
+constexpr int kMnLoWarps = MGGCN_MN_LO_WARPS;    // lo-split warps (0-3 also run the epilogue)
+constexpr int kMnThreads = (kMnLoWarps + 2) * 32, kMnTmaWarp = kMnLoWarps, kMnMmaWarp = kMnLoWarps + 1;
+
+__device__ __forceinline__ uint64_t mn_desc(uint32_t saddr, const uint32_t* d) {
+    return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)((d[1] >> 4) & 0x3FFFu) << 16) |
+           ((uint64_t)((d[2] >> 4) & 0x3FFFu) << 32) | ((uint64_t)1 << 46) | ((uint64_t)(d[0] & 7u) << 61);
+}
+
+__global__ void __launch_bounds__(kMnThreads, 1)
+gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                     const KParams p) {
+    extern __shared__ uint8_t smem_dyn[];
+    uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kMnBars);
+    uint64_t* full = bars;                       // [kMnNR] TMA -> lo warps
+    uint64_t* ready = bars + kMnNR;              // [kMnNR] lo warps -> MMA
+    uint64_t* empty = bars + 2 * kMnNR;          // [kMnNR] MMA -> TMA
+    uint64_t* lo_free = bars + 3 * kMnNR;        // [kMnNL] MMA -> lo warps
+    uint64_t* tmem_full = bars + 3 * kMnNR + kMnNL;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const bool x1 = (p.flags & GEMM_TF32X1) != 0;
+    const int BN = p.BN;
+    const uint32_t tcols = BN > 128 ? 256u : BN > 64 ? 128u : 64u;
+    const int tile = blockIdx.x;
+    const int nt = tile % p.n_tiles;
+    const int mt = (tile / p.n_tiles) % p.m_tiles;
+    const int kc = tile / (p.n_tiles * p.m_tiles);
+    const int k0 = kc * p.k_chunk_len;
+    const int k1 = min(p.K, k0 + p.k_chunk_len);
+    const int nkb = (k1 - k0 + kMnBK - 1) / kMnBK;
+    const int nbox_b = BN / 32;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kMnNR; ++s) {
+            mbar_init(full + s, 1);
+            mbar_init(ready + s, kMnLoWarps * 32);
+            mbar_init(empty + s, 1);
+        }
+        for (int s = 0; s < kMnNL; ++s) mbar_init(lo_free + s, 1);
+        mbar_init(tmem_full, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == kMnMmaWarp) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(tcols));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == kMnTmaWarp) {
+        if (lane == 0) {
+            const uint32_t bytes = (uint32_t)((4 + nbox_b) * 2048);
+            int s = 0;
+            uint32_t ph = 0;
+            for (int kb = 0; kb < nkb; ++kb) {
+                uint8_t* st = smem + s * kMnRaw;
+                mbar_wait(empty + s, ph ^ 1);
+                mbar_expect_tx(full + s, bytes);
+                const int kr = k0 + kb * kMnBK;
+                for (int j = 0; j < 4; ++j) tma_load_2d(st + j * 2048, &tmA, mt * BM + 32 * j, kr, full + s);
+                for (int j = 0; j < nbox_b; ++j)
+                    tma_load_2d(st + 8192 + j * 2048, &tmB, nt * BN + 32 * j, kr, full + s);
+                if (++s == kMnNR) { s = 0; ph ^= 1; }
+            }
+        }
+    } else if (warp == kMnMmaWarp) {
+        if (lane == 0) {
+            const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 15) | (1u << 16) |
+                                   ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+            int s = 0, l = 0;
+            uint32_t ph = 0;
+            for (int kb = 0; kb < nkb; ++kb) {
+                mbar_wait(ready + s, ph);
+                tc_fence_after();
+                const uint32_t raw = smem_u32(smem + s * kMnRaw), lo = smem_u32(smem + kMnLo0 + l * kMnRaw);
+#pragma unroll
+                for (int kk = 0; kk < kMnBK / 8; ++kk) {
+                    const uint32_t off = kk * 8 * 128;   // 8 k rows of 128 B
+                    const uint64_t ah = mn_desc(raw + off, p.desc_mn), bh = mn_desc(raw + 8192 + off, p.desc_mn);
+                    if (!x1) {
+                        const uint64_t al = mn_desc(lo + off, p.desc_mn), bl = mn_desc(lo + 8192 + off, p.desc_mn);
+                        mma_tf32(tmem_base, al, bh, idesc, (kb | kk) ? 1u : 0u);
+                        mma_tf32(tmem_base, ah, bl, idesc, 1u);
+                        mma_tf32(tmem_base, ah, bh, idesc, 1u);
+                    } else {
+                        mma_tf32(tmem_base, ah, bh, idesc, (kb | kk) ? 1u : 0u);
+                    }
+                }
+                mma_commit(empty + s);
+                mma_commit(lo_free + l);
+                if (++s == kMnNR) { s = 0; ph ^= 1; }
+                if (++l == kMnNL) l = 0;
+            }
+            mma_commit(tmem_full);
+        }
+    } else {
+        // warps 0-3: lo = x - hi of every staged tile (1xTF32: round the tile in place)
+        const int t = threadIdx.x;
+        const int nA4 = 4 * 2048 / 16, nT4 = nA4 + nbox_b * 2048 / 16;   // float4 counts
+        int s = 0, l = 0;
+        uint32_t ph = 0, lph = 0;
+        for (int kb = 0; kb < nkb; ++kb) {
+            uint8_t* st = smem + s * kMnRaw;
+            uint8_t* lb = smem + kMnLo0 + l * kMnRaw;
+            mbar_wait(full + s, ph);
+            if (!x1) mbar_wait(lo_free + l, lph ^ 1);
+            for (int i = t; i < nT4; i += kMnLoWarps * 32) {
+                float4* hp = reinterpret_cast<float4*>(st + i * 16);
+                float4 hi, lo;
+                split4(*hp, hi, lo, x1);
+                if (x1) *hp = hi;
+                else *reinterpret_cast<float4*>(lb + i * 16) = lo;
+            }
+            fence_proxy_async();
+            mbar_arrive(ready + s);
+            if (++s == kMnNR) { s = 0; ph ^= 1; }
+            if (++l == kMnNL) { l = 0; lph ^= 1; }
+        }
+        if (warp < 4) {
+            mbar_wait(tmem_full, 0);
+            tc_fence_after();
+            const int row = mt * BM + warp * 32 + lane;
+            const int n0 = nt * BN;
+            for (int c0 = 0; c0 < BN; c0 += 16) {
+                float v[16];
+                tmem_ld16(tmem_base + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0, v);
+                const int nb = n0 + c0;
+                if (row >= p.M || nb >= p.N) continue;
+                float* dst = p.partial + ((int64_t)kc * p.M + row) * (int64_t)p.N + nb;
+#pragma unroll
+                for (int i = 0; i < 16; ++i)
+                    if (nb + i < p.N) dst[i] = v[i];
+            }
+            tc_fence_before();
+        }
+    }
+    __syncthreads();
+    if (warp == kMnMmaWarp) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
+    }
+}
+
 // ===================================================================== rows
 // Row GEMM (op 0 / op 1): C[M x N] = A[M x K] · B^T with B given PRE-SPLIT as
 // tf32 hi / lo copies in K-major [N x K] layout (the weights; split once per
@@ -684,6 +855,21 @@ int encode2d_sw(CUtensorMap* m, const float* base, int64_t dim0, int64_t dim1, i
     return r == CUDA_SUCCESS ? 0 : -2;
 }
 
+// as encode2d with an explicit CUtensorMapSwizzle
+int encode2d_mode(CUtensorMap* m, const float* base, int64_t dim0, int64_t dim1, int64_t ld, int box0, int box1,
+                  CUtensorMapSwizzle sw) {
+    EncodeTiledFn fn = get_encode();
+    if (!fn) return -1;
+    cuuint64_t dims[2] = {(cuuint64_t)dim0, (cuuint64_t)dim1};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+    cuuint32_t box[2] = {(cuuint32_t)box0, (cuuint32_t)box1};
+    cuuint32_t es[2] = {1, 1};
+    CUresult r = fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, es,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : -2;
+}
+
 int num_sms() {
     static int n = 0;
     if (n == 0) {
@@ -703,6 +889,19 @@ cudaError_t launch_wgrad(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
         attr_set = true;
     }
     gemm_wgrad_kernel<<<g.grid, kWgThreads, kWgSmem, s>>>(g.tmA, g.tmB, kp);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_wgrad_mn(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaError_t e =
+            cudaFuncSetAttribute(gemm_wgrad_mn_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kMnSmem);
+        if (e != cudaSuccess) return e;
+        attr_set = true;
+    }
+    gemm_wgrad_mn_kernel<<<g.grid, kMnThreads, kMnSmem, s>>>(g.tmA, g.tmB, kp);
     count_launches(1);
     return cudaGetLastError();
 }
@@ -764,16 +963,39 @@ int gemm_plan_wgrad(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A
     g.m_tiles = (int)((M + BM - 1) / BM);
     g.flags = flags;
     const int mn = g.m_tiles * g.n_tiles;
-    int want = (num_sms() + mn - 1) / mn;
+    int want = num_sms() / mn;   // one wave: (M, N, K-chunk) tiles <= #SMs (1 CTA / SM)
     const int64_t kblocks = (K + BK - 1) / BK;
     if (want > kblocks) want = (int)kblocks;
     if (want < 1) want = 1;
     g.k_chunk_len = (kblocks + want - 1) / want * BK;
     g.k_chunks = (int)((K + g.k_chunk_len - 1) / g.k_chunk_len);
     if (partial_floats) *partial_floats = (size_t)g.k_chunks * (size_t)M * (size_t)N;
-    // A is K x M (M contiguous), B is K x N (N contiguous): raw boxes {M or N, 16 K}, transposed in smem
-    int rc = encode2d(&g.tmA, A, M, K, lda, BM, 16, false);
-    if (!rc) rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, 16, false);
+    // A is K x M (M contiguous), B is K x N (N contiguous)
+    static int variant = -1, tsw = 0;
+    static uint32_t dmn[3] = {1, 2048, 512};
+    if (variant < 0) {
+        const char* e = getenv("MGGCN_WGRAD");
+        variant = (e && e[0] == 'x') ? 0 : 1;     // default: MN-major operands (no transpose)
+        if (const char* d = getenv("MGGCN_WG_DESC")) sscanf(d, "%u,%u,%u", &dmn[0], &dmn[1], &dmn[2]);
+        if (const char* t = getenv("MGGCN_WG_TMASW")) tsw = atoi(t);
+    }
+    g.variant = variant;
+    int rc;
+    if (variant == 1) {
+        // boxes of 32 MN-contiguous floats x 16 k rows, 128B swizzle with 32B atoms
+        g.BN = (int)(((N + g.n_tiles - 1) / g.n_tiles + 31) / 32 * 32);
+        for (int i = 0; i < 3; ++i) g.desc_mn[i] = dmn[i];
+        const CUtensorMapSwizzle sw = tsw == 1 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B_FLIP_8B
+                                      : tsw == 2 ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_64B
+                                      : tsw == 3 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                                 : CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B;
+        rc = encode2d_mode(&g.tmA, A, M, K, lda, 32, 16, sw);
+        if (!rc) rc = encode2d_mode(&g.tmB, B, N, K, ldb, 32, 16, sw);
+    } else {
+        // raw boxes {M or N, 16 K}, transposed in smem
+        rc = encode2d(&g.tmA, A, M, K, lda, BM, 16, false);
+        if (!rc) rc = encode2d(&g.tmB, B, N, K, ldb, g.BN, 16, false);
+    }
     if (rc) return rc;
     g.grid = g.m_tiles * g.n_tiles * g.k_chunks;   // one CTA per tile
     return 0;
@@ -783,7 +1005,7 @@ size_t gemm_wgrad_partial_floats(int64_t M, int64_t N, int64_t K) {
     const int n_tiles = (int)((N + 255) / 256);
     const int m_tiles = (int)((M + BM - 1) / BM);
     const int mn = m_tiles * n_tiles;
-    int want = (num_sms() + mn - 1) / mn;
+    int want = num_sms() / mn;   // one wave: (M, N, K-chunk) tiles <= #SMs (1 CTA / SM)
     const int64_t kblocks = (K + BK - 1) / BK;
     if (want > kblocks) want = (int)kblocks;
     if (want < 1) want = 1;
@@ -798,8 +1020,9 @@ cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
     kp.k_chunks = g.k_chunks; kp.k_chunk_len = (int)g.k_chunk_len;
     kp.C = g.C; kp.ldc = g.ldc; kp.partial = g.partial; kp.rowscale = g.rowscale;
     kp.flags = g.flags; kp.op2 = g.op == 2;
+    for (int i = 0; i < 3; ++i) kp.desc_mn[i] = g.desc_mn[i];
 
-    if (g.op == 2) return launch_wgrad(g, kp, s);
+    if (g.op == 2) return g.variant == 1 ? launch_wgrad_mn(g, kp, s) : launch_wgrad(g, kp, s);
     return launch_rows(g, kp, s);
 }
 

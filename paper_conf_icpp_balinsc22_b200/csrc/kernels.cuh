@@ -63,6 +63,8 @@ struct GemmPlan {
     const float* rowscale = nullptr;
     int flags = 0;
     int grid = 0;
+    int variant = 0;            // op 2: 1 = MN-major operands straight from TMA (no transpose)
+    uint32_t desc_mn[3] = {1, 2048, 512};   // op 2 variant 1: layout type, LBO, SBO (bytes)
 };
 
 // Row GEMM (op 0 and op 1 of the comment above): C = A · B^T with B given

@@ -666,8 +666,8 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 for (int c = t; c < BM * 4; c += 128) {
                     float4 v = a[c], h, l;
                     split4(v, h, l, x1);
-                    a[c] = h;
-                    if (!x1) al[c] = l;
+                    if (x1) a[c] = h;      // 3xTF32: the MMA reads x as hi = x & 0xFFFFE000 itself
+                    else al[c] = l;
                 }
                 fence_proxy_async();
                 mbar_arrive(xf + s);

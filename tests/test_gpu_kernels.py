@@ -172,3 +172,22 @@ def test_spmm_power_law_exact_hub(mg):
     expect0 = B[1:].astype(np.float64).sum(axis=0) / 9000.0
     np.testing.assert_allclose(got[0], expect0, rtol=1e-6, atol=1e-7)
     gm.close()
+
+
+@pytest.mark.parametrize("win", [64, 128])
+def test_spmm_column_windows(win):
+    """The windowed gather (launch_spmm splits the width into column windows,
+    automatic for L2-sized blocks) against the oracle: re-runs the R-MAT hub
+    cases in a fresh process with the window forced to `win` floats."""
+    import os
+    import subprocess
+    import sys
+    if os.environ.get("MGGCN_SPMM_WIN"):
+        pytest.skip("already inside a forced-window run")
+    here = os.path.dirname(os.path.abspath(__file__))
+    env = dict(os.environ, MGGCN_SPMM_WIN=str(win))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", os.path.join(here, "test_gpu_kernels.py"),
+                        "-k", "rmat_hubs and (172 or 256 or 512 or 600) and True"], env=env, cwd=os.path.dirname(here),
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout

@@ -163,6 +163,50 @@ def oracle_epoch_sample(w, rp, col, rows_per_step, seed=0):
     return (t_row * (n / R) + t_fixed) * 1e3, time.perf_counter() - wall0, R
 
 
+# Measured ceiling of the SpMM's real bound: uniform random 512-B row gathers
+# (LDG.128, 16 rows in flight per lane) from an L2-resident 29 MB table on this
+# B200 (bench_micro/dsmem_gather.cu, mode 0, x = 0; profiles/r01_dsmem_gather.jsonl).
+L2_GATHER_PEAK_GBPS = 19480.5
+
+
+def spmm_widths(dims):
+    """Widths of the SpMMs of one epoch (§4.4 order rule C10, first-layer skip C11)."""
+    ws = []
+    for l in range(len(dims) - 1):
+        if dims[l] < dims[l + 1]:          # SpMM-first (layer 0 only): forward T0 = A'^T X; no backward SpMM
+            ws.append(dims[l])
+        else:                              # GeMM-first: forward A'^T HW and backward A' AHW_G
+            ws += [dims[l + 1], dims[l + 1]]
+    return ws
+
+
+def line_bytes(width):
+    """Bytes of 128-B L2 lines one gathered row touches: the kernel reads ceil(width/4) float4
+    of a row whose stride is ld = round_up(width, 8) floats (window of <= 128 floats when the
+    library splits the width), averaged over the row start offsets mod 128 B."""
+    tot = 0
+    c0 = 0
+    while c0 < width:
+        w = min(128 if width > 128 else width, width - c0)
+        ld_b = ((width + 7) // 8 * 8) * 4
+        rd = (w + 3) // 4 * 16
+        offs = sorted({(r * ld_b + c0 * 4) % 128 for r in range(128)})
+        tot += sum(((o + rd + 127) // 128) * 128 for o in offs) / len(offs)
+        c0 += w
+    return tot
+
+
+def l2_gather_roofline(dims, work, spmm_ms_per_epoch, cache=False):
+    ws = spmm_widths(dims)
+    nnz = work["spmm_gather_bytes"] / (4.0 * sum(ws))          # coalesced non-zeros per SpMM (all ranks' tiles)
+    lb = nnz * sum(line_bytes(x) for x in ws)
+    ach = lb / (spmm_ms_per_epoch * 1e-3) / 1e9 if spmm_ms_per_epoch > 0 else 0.0
+    return {"bound": "l2 (SM<-L2 line rate of random row gathers)", "achieved": ach, "peak": L2_GATHER_PEAK_GBPS,
+            "unit": "GB/s", "frac": ach / L2_GATHER_PEAK_GBPS, "line_bytes_per_epoch": lb,
+            "peak_source": "bench_micro/dsmem_gather.cu: uniform 512-B row gathers from an L2-resident table "
+                           "(profiles/r01_dsmem_gather.jsonl)"}
+
+
 def auto_rows(w):
     # about 3 s of single-core oracle work per sampled epoch
     per_row = (w.m / w.n) * sum(w.dims) * 2 + 3 * sum(w.dims[l] * w.dims[l + 1] for l in range(len(w.dims) - 1))
@@ -375,6 +419,7 @@ def main():
             traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
         except Exception:
             traffic = None
+    l2_gather = l2_gather_roofline(w.dims, work, spmm_ms / args.steps, cache=False)
     gemm_ms, gemm_n = prof["gemm"]
     tf32_peak = float(peaks.get("bf16_tflops_sustained", 1352.7)) / 2.0
 
@@ -396,7 +441,9 @@ def main():
                      "launch_ms": spmm_launch_ms, "launches_per_epoch": launches_per_epoch,
                      "gather_model_GBps": gather_gbs,
                      "note": "achieved = compulsory bytes (indices + rowptr + each input and output row once, "
-                             "SURVEY §8d) / measured launch time; gather_model_GBps = nnz*width*4 B / time"},
+                             "SURVEY §8d) / measured launch time; gather_model_GBps = nnz*width*4 B / time; "
+                             "a launch = one SpMM stage (its column-window kernels + hub fix-up)",
+                     "l2_gather": l2_gather},
         "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
         "gemm": {"tflops": work["gemm_flops"] / (gemm_ms / args.steps * 1e-3) / 1e12 if gemm_ms else None,
                  "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps},

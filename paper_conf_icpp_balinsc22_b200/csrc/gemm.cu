@@ -404,11 +404,20 @@ gemm_wgrad_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
 // (TMA -> MMA, 24 KB) and 2 lo stages; 192 threads: warps 0-3 lo + epilogue,
 // warp 4 TMA, warp 5 TMEM allocator + MMA issuer.
 constexpr int kMnBK = 16;
-constexpr int kMnNR = 6, kMnNL = 2;
-constexpr int kMnRaw = 24576;                    // A 8K (4 boxes) | B 16K (<= 8 boxes)
-constexpr int kMnLo0 = kMnNR * kMnRaw;
-constexpr int kMnBars = kMnLo0 + kMnNL * kMnRaw;
-constexpr int kMnSmem = kMnBars + 256 + 1024;
+// Rings of stages of A 8K (4 boxes) | B nbox_b x 2K: raw (TMA -> MMA) and lo
+// (split -> MMA), sized from BN so narrow-N products keep more k blocks of
+// the streamed operands in flight (BN = 256: 6 raw + 2 lo stages of 24 KB;
+// BN = 64: 10 raw + 4 lo stages of 12 KB).
+constexpr int kMnBudget = 8 * 24576;
+constexpr int kMnMaxNR = 10, kMnMaxNL = 4;
+constexpr int kMnBars = kMnBudget;
+constexpr int kMnSmem = kMnBars + 512 + 1024;
+__host__ __device__ __forceinline__ int mn_stage_bytes(int BN) { return 8192 + (BN / 32) * 2048; }
+__host__ __device__ __forceinline__ int mn_lo_stages(int BN) { return mn_stage_bytes(BN) <= 12288 ? kMnMaxNL : 2; }
+__host__ __device__ __forceinline__ int mn_raw_stages(int BN) {
+    const int nr = (kMnBudget - mn_lo_stages(BN) * mn_stage_bytes(BN)) / mn_stage_bytes(BN);
+    return nr < kMnMaxNR ? nr : kMnMaxNR;
+}
 #ifndef MGGCN_MN_LO_WARPS
 #define MGGCN_MN_LO_WARPS 12
 #endif
@@ -426,11 +435,11 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     extern __shared__ uint8_t smem_dyn[];
     uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kMnBars);
-    uint64_t* full = bars;                       // [kMnNR] TMA -> lo warps
-    uint64_t* ready = bars + kMnNR;              // [kMnNR] lo warps -> MMA
-    uint64_t* empty = bars + 2 * kMnNR;          // [kMnNR] MMA -> TMA
-    uint64_t* lo_free = bars + 3 * kMnNR;        // [kMnNL] MMA -> lo warps
-    uint64_t* tmem_full = bars + 3 * kMnNR + kMnNL;
+    uint64_t* full = bars;                       // [NR] TMA -> lo warps
+    uint64_t* ready = bars + kMnMaxNR;           // [NR] lo warps -> MMA
+    uint64_t* empty = bars + 2 * kMnMaxNR;       // [NR] MMA -> TMA
+    uint64_t* lo_free = bars + 3 * kMnMaxNR;     // [NL] MMA -> lo warps
+    uint64_t* tmem_full = lo_free + kMnMaxNL;
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 1);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
@@ -444,14 +453,16 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     const int k1 = min(p.K, k0 + p.k_chunk_len);
     const int nkb = (k1 - k0 + kMnBK - 1) / kMnBK;
     const int nbox_b = BN / 32;
+    const int SB = mn_stage_bytes(BN), NR = mn_raw_stages(BN), NL = mn_lo_stages(BN);
+    uint8_t* const lo0 = smem + NR * SB;
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < kMnNR; ++s) {
+        for (int s = 0; s < NR; ++s) {
             mbar_init(full + s, 1);
             mbar_init(ready + s, kMnLoWarps * 32);
             mbar_init(empty + s, 1);
         }
-        for (int s = 0; s < kMnNL; ++s) mbar_init(lo_free + s, 1);
+        for (int s = 0; s < NL; ++s) mbar_init(lo_free + s, 1);
         mbar_init(tmem_full, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -471,14 +482,14 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
             int s = 0;
             uint32_t ph = 0;
             for (int kb = 0; kb < nkb; ++kb) {
-                uint8_t* st = smem + s * kMnRaw;
+                uint8_t* st = smem + s * SB;
                 mbar_wait(empty + s, ph ^ 1);
                 mbar_expect_tx(full + s, bytes);
                 const int kr = k0 + kb * kMnBK;
                 for (int j = 0; j < 4; ++j) tma_load_2d(st + j * 2048, &tmA, mt * BM + 32 * j, kr, full + s);
                 for (int j = 0; j < nbox_b; ++j)
                     tma_load_2d(st + 8192 + j * 2048, &tmB, nt * BN + 32 * j, kr, full + s);
-                if (++s == kMnNR) { s = 0; ph ^= 1; }
+                if (++s == NR) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == kMnMmaWarp) {
@@ -490,7 +501,7 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
             for (int kb = 0; kb < nkb; ++kb) {
                 mbar_wait(ready + s, ph);
                 tc_fence_after();
-                const uint32_t raw = smem_u32(smem + s * kMnRaw), lo = smem_u32(smem + kMnLo0 + l * kMnRaw);
+                const uint32_t raw = smem_u32(smem + s * SB), lo = smem_u32(lo0 + l * SB);
 #pragma unroll
                 for (int kk = 0; kk < kMnBK / 8; ++kk) {
                     const uint32_t off = kk * 8 * 128;   // 8 k rows of 128 B
@@ -506,8 +517,8 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
                 }
                 mma_commit(empty + s);
                 mma_commit(lo_free + l);
-                if (++s == kMnNR) { s = 0; ph ^= 1; }
-                if (++l == kMnNL) l = 0;
+                if (++s == NR) { s = 0; ph ^= 1; }
+                if (++l == NL) l = 0;
             }
             mma_commit(tmem_full);
         }
@@ -518,8 +529,8 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
         int s = 0, l = 0;
         uint32_t ph = 0, lph = 0;
         for (int kb = 0; kb < nkb; ++kb) {
-            uint8_t* st = smem + s * kMnRaw;
-            uint8_t* lb = smem + kMnLo0 + l * kMnRaw;
+            uint8_t* st = smem + s * SB;
+            uint8_t* lb = lo0 + l * SB;
             mbar_wait(full + s, ph);
             if (!x1) mbar_wait(lo_free + l, lph ^ 1);
             for (int i = t; i < nT4; i += kMnLoWarps * 32) {
@@ -531,8 +542,8 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
             }
             fence_proxy_async();
             mbar_arrive(ready + s);
-            if (++s == kMnNR) { s = 0; ph ^= 1; }
-            if (++l == kMnNL) { l = 0; lph ^= 1; }
+            if (++s == NR) { s = 0; ph ^= 1; }
+            if (++l == NL) { l = 0; lph ^= 1; }
         }
         if (warp < 4) {
             mbar_wait(tmem_full, 0);
@@ -569,12 +580,24 @@ gemm_wgrad_mn_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
 // TMA bulk store (full 128-B lines); the old C values for the ReLU' mask of
 // Eq. 8 / Eq. 21 come in by TMA into the same layout.
 constexpr int kRowBK = 16;
-constexpr int kRowNS = 3;
-constexpr int kRowStage = 48 * 1024;            // A 8K | A_lo 8K | B_hi 16K | B_lo 16K
-constexpr int kRowOut = kRowNS * kRowStage;     // 2 x 16 KB output chunks [128 rows][32 cols] SW128
-constexpr int kRowOld = kRowOut + 2 * 16384;    // 2 x 16 KB old-C chunks (mask)
-constexpr int kRowBars = kRowOld + 2 * 16384;
+// shared memory: 2 x 16 KB output chunks [128 rows][32 cols] SW128, 2 x 16 KB
+// old-C chunks (mask), then the operand ring: stages of A 8K | A_lo 8K |
+// B_hi BN x 64 B | B_lo BN x 64 B, as many as fit the budget (3 for BN = 256,
+// 7 for BN = 48): narrow-N products are bound by the A stream, which needs
+// more k blocks in flight than the MMAs do.
+constexpr int kRowOut = 0;
+constexpr int kRowOld = 2 * 16384;
+constexpr int kRowStage0 = 4 * 16384;
+constexpr int kRowStageBudget = 160 * 1024;
+constexpr int kRowMaxNS = 8;
+constexpr int kRowBars = kRowStage0 + kRowStageBudget;
 constexpr int kRowSmem = kRowBars + 256 + 1024;
+
+__host__ __device__ __forceinline__ int row_stage_bytes(int BN) { return (16384 + 2 * BN * 64 + 1023) / 1024 * 1024; }
+__host__ __device__ __forceinline__ int row_stages(int BN) {
+    const int ns = kRowStageBudget / row_stage_bytes(BN);
+    return ns < kRowMaxNS ? ns : kRowMaxNS;
+}
 
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* tm, int c0, int c1, const void* src) {
     asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"((uint64_t)tm),
@@ -597,21 +620,23 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     extern __shared__ uint8_t smem_dyn[];
     uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);   // keeps the shared state space
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kRowBars);
-    uint64_t* full = bars + 0;           // [3]
-    uint64_t* xf = bars + 3;             // [3]
-    uint64_t* empty = bars + 6;          // [3]
-    uint64_t* tmem_full = bars + 9;      // [2]
-    uint64_t* tmem_empty = bars + 11;    // [2]
-    uint64_t* old_full = bars + 13;      // [2]
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 15);
+    uint64_t* full = bars + 0;                   // [kRowMaxNS]
+    uint64_t* xf = bars + kRowMaxNS;             // [kRowMaxNS]
+    uint64_t* empty = bars + 2 * kRowMaxNS;      // [kRowMaxNS]
+    uint64_t* tmem_full = bars + 3 * kRowMaxNS;  // [2]
+    uint64_t* tmem_empty = tmem_full + 2;        // [2]
+    uint64_t* old_full = tmem_full + 4;          // [2]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tmem_full + 6);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
     const bool mask = (p.flags & GEMM_MASK) != 0;
     const int BN = p.BN;
     const uint32_t tcols = BN > 128 ? 512u : 256u;
+    const int NS = row_stages(BN), SB = row_stage_bytes(BN);
+    const int kBlo = 16384 + BN * 64;            // B_lo offset within a stage
 
     if (threadIdx.x == 0) {
-        for (int s = 0; s < kRowNS; ++s) {
+        for (int s = 0; s < NS; ++s) {
             mbar_init(full + s, 1);
             mbar_init(xf + s, 128);
             mbar_init(empty + s, 1);
@@ -643,13 +668,13 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
             for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
                 const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
                 for (int kb = 0; kb < nkb; ++kb) {
-                    uint8_t* st = smem + s * kRowStage;
+                    uint8_t* st = smem + kRowStage0 + s * SB;
                     mbar_wait(empty + s, ph ^ 1);
                     mbar_expect_tx(full + s, bytes);
                     tma_load_2d(st, &tmA, kb * kRowBK, mt * BM, full + s);
                     tma_load_2d(st + 16384, &tmBh, kb * kRowBK, nt * BN, full + s);
-                    if (!x1) tma_load_2d(st + 32768, &tmBl, kb * kRowBK, nt * BN, full + s);
-                    if (++s == kRowNS) { s = 0; ph ^= 1; }
+                    if (!x1) tma_load_2d(st + kBlo, &tmBl, kb * kRowBK, nt * BN, full + s);
+                    if (++s == NS) { s = 0; ph ^= 1; }
                 }
             }
         }
@@ -659,8 +684,8 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         uint32_t ph = 0;
         for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
             for (int kb = 0; kb < nkb; ++kb) {
-                float4* a = reinterpret_cast<float4*>(smem + s * kRowStage);
-                float4* al = reinterpret_cast<float4*>(smem + s * kRowStage + 8192);
+                float4* a = reinterpret_cast<float4*>(smem + kRowStage0 + s * SB);
+                float4* al = reinterpret_cast<float4*>(smem + kRowStage0 + s * SB + 8192);
                 mbar_wait(full + s, ph);
 #pragma unroll
                 for (int c = t; c < BM * 4; c += 128) {
@@ -671,7 +696,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 }
                 fence_proxy_async();
                 mbar_arrive(xf + s);
-                if (++s == kRowNS) { s = 0; ph ^= 1; }
+                if (++s == NS) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == kMmaWarp) {
@@ -689,9 +714,9 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 for (int kb = 0; kb < nkb; ++kb) {
                     mbar_wait(xf + s, ph);
                     tc_fence_after();
-                    const uint32_t base = smem_u32(smem + s * kRowStage);
+                    const uint32_t base = smem_u32(smem + kRowStage0 + s * SB);
                     const uint64_t ah = sw64_desc(base), al = sw64_desc(base + 8192);
-                    const uint64_t bh = sw64_desc(base + 16384), bl = sw64_desc(base + 32768);
+                    const uint64_t bh = sw64_desc(base + 16384), bl = sw64_desc(base + kBlo);
 #pragma unroll
                     for (int kk = 0; kk < kRowBK / 8; ++kk) {
                         const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);
@@ -704,7 +729,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                         }
                     }
                     mma_commit(empty + s);
-                    if (++s == kRowNS) { s = 0; ph ^= 1; }
+                    if (++s == NS) { s = 0; ph ^= 1; }
                 }
                 mma_commit(tmem_full + acc);
             }

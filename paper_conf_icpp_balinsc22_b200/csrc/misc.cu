@@ -76,6 +76,128 @@ softmax_ce_kernel(float* __restrict__ Z, int64_t n, int C, int64_t ld, const int
     }
 }
 
+// Vectorised variant for C <= 256: a row is held by a group of G lanes, CH
+// float4 per lane, so a warp works on 32/G rows at once and U row groups are
+// loaded before any arithmetic (one read and one write of each row, all loads
+// in flight together).  Same arithmetic per row as softmax_ce_kernel: fp32
+// max, sum of exp(z - max), lse = max + log(sum), gradient (exp(z - lse) -
+// [c == y]) * inv_nt * rowscale (Eq. 19), loss lse - z_y summed in fp64; the
+// group sums use a fixed xor tree and the per-row losses are added in a fixed
+// order (lane-group, then iteration, then warp), so results are deterministic.
+template <int G, int CH>
+__device__ __forceinline__ float group_max(float v) {
+#pragma unroll
+    for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+template <int G>
+__device__ __forceinline__ float group_sum(float v) {
+#pragma unroll
+    for (int o = G / 2; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+template <int G, int CH, int U>
+__global__ void __launch_bounds__(kCeWarps * 32)
+softmax_ce_vec_kernel(float* __restrict__ Z, int64_t n, int C, int64_t ld, const int32_t* __restrict__ y,
+                      const int64_t* __restrict__ ntrain, const float* __restrict__ rowscale, int relu_last,
+                      double* __restrict__ block_partial) {
+    constexpr int R = 32 / G;          // rows per warp step
+    __shared__ double wsum[kCeWarps];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int sub = lane / G, gl = lane % G;
+    const int64_t gw = (int64_t)blockIdx.x * kCeWarps + wid, nw = (int64_t)gridDim.x * kCeWarps;
+    const float inv_nt = 1.0f / (float)(*ntrain > 0 ? *ntrain : 1);
+    double lsum = 0.0;
+    for (int64_t r0 = gw * (R * U); r0 < n; r0 += nw * (R * U)) {
+        float4 x[U][CH];
+        int lab[U];
+        float sc[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t r = r0 + u * R + sub;
+            const bool ok = r < n;
+            const float4* zr = reinterpret_cast<const float4*>(Z + (ok ? r : 0) * ld);
+#pragma unroll
+            for (int ch = 0; ch < CH; ++ch) {
+                const int q = gl + ch * G;
+                x[u][ch] = (4 * q < C) ? zr[q] : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+            lab[u] = ok ? y[r] : -1;
+            sc[u] = ok && rowscale ? rowscale[r] : 1.f;
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t r = r0 + u * R + sub;
+            float mx = -INFINITY;
+#pragma unroll
+            for (int ch = 0; ch < CH; ++ch) {
+                const int c = 4 * (gl + ch * G);
+                if (c + 0 < C) mx = fmaxf(mx, x[u][ch].x);
+                if (c + 1 < C) mx = fmaxf(mx, x[u][ch].y);
+                if (c + 2 < C) mx = fmaxf(mx, x[u][ch].z);
+                if (c + 3 < C) mx = fmaxf(mx, x[u][ch].w);
+            }
+            mx = group_max<G, CH>(mx);
+            float sm = 0.f;
+#pragma unroll
+            for (int ch = 0; ch < CH; ++ch) {
+                const int c = 4 * (gl + ch * G);
+                if (c + 0 < C) sm += expf(x[u][ch].x - mx);
+                if (c + 1 < C) sm += expf(x[u][ch].y - mx);
+                if (c + 2 < C) sm += expf(x[u][ch].z - mx);
+                if (c + 3 < C) sm += expf(x[u][ch].w - mx);
+            }
+            sm = group_sum<G>(sm);
+            const float lse = mx + logf(sm);
+            const int l = lab[u];
+            // z_y from the lane that holds column l
+            float zy = 0.f;
+            const int ql = l >= 0 ? l >> 2 : 0;
+            if (l >= 0 && gl == ql % G) {
+#pragma unroll
+                for (int ch = 0; ch < CH; ++ch)
+                    if (ch == ql / G) {
+                        const float4 v = x[u][ch];
+                        zy = (l & 3) == 0 ? v.x : (l & 3) == 1 ? v.y : (l & 3) == 2 ? v.z : v.w;
+                    }
+            }
+            zy = group_sum<G>(zy);       // one non-zero term: exact
+            if (r >= n) continue;
+            if (gl == 0 && l >= 0) lsum += (double)lse - (double)zy;
+            const float s2 = inv_nt * sc[u];
+            float* zr = Z + r * ld;
+#pragma unroll
+            for (int ch = 0; ch < CH; ++ch) {
+                const int q = gl + ch * G, c = 4 * q;
+                if (c >= C) continue;
+                float o[4] = {x[u][ch].x, x[u][ch].y, x[u][ch].z, x[u][ch].w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    const float zc = o[e];
+                    float g = expf(zc - lse) - (c + e == l ? 1.f : 0.f);
+                    if (relu_last && !(zc > 0.f)) g = 0.f;
+                    o[e] = l >= 0 ? g * s2 : 0.f;
+                }
+                if (c + 4 <= C) {
+                    reinterpret_cast<float4*>(zr)[q] = make_float4(o[0], o[1], o[2], o[3]);
+                } else {
+                    for (int e = 0; c + e < C; ++e) zr[c + e] = o[e];
+                }
+            }
+        }
+    }
+    // fixed-order reduction: lane-group leaders' sums in lane order, then warps
+    lsum = warp_sum_d(lsum);
+    if (lane == 0) wsum[wid] = lsum;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < kCeWarps; ++w) t += wsum[w];
+        block_partial[blockIdx.x] = t;
+    }
+}
+
 __global__ void sum_partials_kernel(const double* __restrict__ p, int count, double* __restrict__ out) {
     // one warp, strided lane sums then fixed xor tree
     double t = 0.0;
@@ -161,7 +283,21 @@ __global__ void splitk_reduce_kernel(const float* __restrict__ partial, int k_ch
 
 cudaError_t launch_softmax_ce(float* Z, int64_t n, int C, int64_t ld, const int32_t* y, const int64_t* ntrain,
                               const float* rowscale, int relu_last, double* block_partial, cudaStream_t s) {
-    softmax_ce_kernel<<<kCeBlocks, kCeWarps * 32, 0, s>>>(Z, n, C, ld, y, ntrain, rowscale, relu_last, block_partial);
+    // row-group shapes: G lanes x CH float4 per lane cover C columns (ld is a multiple of 4)
+#define MGGCN_CE(G, CH, U) \
+    softmax_ce_vec_kernel<G, CH, U><<<kCeBlocks, kCeWarps * 32, 0, s>>>(Z, n, C, ld, y, ntrain, rowscale, relu_last, \
+                                                                        block_partial)
+    if ((ld & 3) == 0 && (reinterpret_cast<uintptr_t>(Z) & 15) == 0 && C <= 256) {
+        if (C <= 16) MGGCN_CE(4, 1, 4);
+        else if (C <= 32) MGGCN_CE(8, 1, 4);
+        else if (C <= 64) MGGCN_CE(16, 1, 4);
+        else if (C <= 128) MGGCN_CE(32, 1, 4);
+        else MGGCN_CE(32, 2, 2);
+    } else {
+        softmax_ce_kernel<<<kCeBlocks, kCeWarps * 32, 0, s>>>(Z, n, C, ld, y, ntrain, rowscale, relu_last,
+                                                              block_partial);
+    }
+#undef MGGCN_CE
     count_launches(1);
     return cudaGetLastError();
 }

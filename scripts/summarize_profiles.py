@@ -124,13 +124,17 @@ def main():
             traffic[name + "_ms"] = float(d["gpu__time_duration.sum"][1]) * (
                 1e-3 if d["gpu__time_duration.sum"][0] == "us" else 1.0)
     if "spmm_wide" in traffic:
-        # an epoch has 4 wide (256) and 2 narrow (41 -> 44) SpMM launches for the Reddit config
-        wide, narrow = traffic["spmm_wide"], traffic.get("spmm_narrow", traffic["spmm_wide"])
+        # an epoch has 4 wide (256) and 2 narrow (41 -> 48) SpMM stages for the Reddit config; a wide
+        # stage is 2 column-window launches of 128 floats (spmm.cu launch_spmm), the capture is one window
+        nwin = int(os.environ.get("WIDE_WINDOWS", "2" if wl == "reddit" else "1"))
+        wide, narrow = nwin * traffic["spmm_wide"], traffic.get("spmm_narrow", traffic["spmm_wide"])
         avg = (4 * wide + 2 * narrow) / 6 if wl == "reddit" else wide
         json.dump({"workload": wl, "P": 1, "tag": tag, "dram_bytes_per_launch": avg,
                    "dram_bytes_wide_launch": wide, "dram_bytes_narrow_launch": narrow,
-                   "how": "ncu --set full, dram__bytes_read.sum + dram__bytes_write.sum, one launch each; "
-                          "epoch average = (4 wide + 2 narrow) / 6 for reddit"},
+                   "wide_windows": nwin,
+                   "how": "ncu --set full, dram__bytes_read.sum + dram__bytes_write.sum, one launch each "
+                          "(a wide stage = wide_windows window launches); epoch average = (4 wide + 2 narrow) / 6 "
+                          "for reddit"},
                   open(os.path.join(PROF, f"spmm_traffic_{wl}_P1.json"), "w"), indent=1)
     open(os.path.join(PROF, f"{tag}_summary.md"), "w").write("\n".join(lines) + "\n")
     print("\n".join(lines))

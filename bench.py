@@ -46,6 +46,9 @@ def parse():
     ap.add_argument("--comm", default="nccl", choices=["nccl", "ipc"],
                     help="N > 1 exchange backend: the library's NCCL communicator, or MGGCN_F_IPC "
                          "(copy-engine pulls from CUDA-IPC-mapped peer workspaces)")
+    ap.add_argument("--replicas", type=int, default=1, choices=[1, 2],
+                    help="2 = 1.5D partitioning (MGGCN_F_REPL2, SURVEY NEXT-4): N/2 row blocks, each held by two "
+                         "ranks that split the broadcast stages and sum their partials; N must be a multiple of 4")
     ap.add_argument("--tf32x1", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -281,8 +284,10 @@ def main():
         flags |= mg.MGGCN_F_TF32X1
     t0 = time.perf_counter()
     graph = mg.mggcn_load_csr(w.n, rp, col)
+    if args.replicas > 1 and (P % (2 * args.replicas) or args.comm == "ipc"):
+        raise SystemExit("--replicas 2 needs N a multiple of 4 and the NCCL backend")
     gm = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed, flags=flags, graph=graph,
-             **comm_kw())
+             replicas=args.replicas, **comm_kw())
     t_setup = time.perf_counter() - t0
     gm.set_weights(Ws)
     Xl = gm.permute_rows(X)
@@ -367,7 +372,7 @@ def main():
         del gm
         torch.cuda.empty_cache()
         gc = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed,
-                 flags=flags | mg.MGGCN_F_CACHE_L0, graph=graph, **comm_kw())
+                 flags=flags | mg.MGGCN_F_CACHE_L0, graph=graph, replicas=args.replicas, **comm_kw())
         gc.set_weights(Ws_now)
         for _ in range(max(args.warmup, 1)):
             gc.forward(Xd, yd, want_loss=False)
@@ -430,7 +435,8 @@ def main():
         "config": workload_desc(w, P) | {"overlap": not args.no_overlap,
                                          "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)",
                                          "comm": (args.comm if P > 1 else "none"),
-                                         "parallelism": f"dp{P} (1D row partition)"},
+                                         "parallelism": (f"dp{P} (1D row partition)" if args.replicas == 1 else
+                                                         f"dp{P} (1.5D: {P // 2} row blocks x 2 replicas)")},
         "e2e": e2e,
         "gpu_launches": int(launches),
         "clocks": clk,

@@ -65,7 +65,7 @@ enum {
                                  runs SpMM-first and T0 = Â'^T X is computed on the first
                                  forward and reused (exact by associativity,
                                  Eq. 5-6 and Eq. 10).  mggcn_reset_cache() after X changes. */
-    MGGCN_F_IPC = 256u        /* nlocal = 1, P > 1 without NCCL: peers map each
+    MGGCN_F_IPC = 256u,       /* nlocal = 1, P > 1 without NCCL: peers map each
                                  other's workspaces (CUDA IPC, mggcn_ipc_export / _connect);
                                  each receiver PULLS the broadcast blocks with copy engines in
                                  rotated order (no SMs taken from the SpMM), W_G and the loss
@@ -74,6 +74,22 @@ enum {
                                  awaited by stream memory operations.  All ranks must issue
                                  the same sequence of calls with the same kind of X argument
                                  (host / device / prefetch); device X is always copied. */
+    MGGCN_F_REPL2 = 512u,     /* 1.5D partitioning with replication factor c = 2 (
+                                 §5.1, the 1.5D algorithm of the paper's ref [35]).
+                                 The parts are P'-way partitions (P' even) and the job has
+                                 2P' ranks: rank (i, r) = r * P' + i holds row block i of Â'
+                                 and H (every block twice), computes the partial SpMM over the
+                                 column blocks j with j mod 2 = r (P'/2 stages; block j is
+                                 broadcast inside replica group r only, so each rank receives
+                                 n d / 2 values per SpMM instead of (P-1)/P n d), then the two
+                                 replicas of a row block sum their partials (pair all-reduce)
+                                 and apply the row scale / ReLU.  GEMMs run on both replicas;
+                                 W_G, the loss and |T| are contributed by replica 0 only.
+                                 Loopback: nlocal = 2P', parts[k] = part k mod P' (replica
+                                 k / P').  NCCL: nlocal = 1, nccl id shared by all 2P'
+                                 processes, MGGCN_F_REPLICA1 on the replica-1 processes.
+                                 Not with MGGCN_F_IPC (EUNSUPPORTED). */
+    MGGCN_F_REPLICA1 = 1024u  /* with MGGCN_F_REPL2 and nlocal = 1: this process is replica 1 */
 };
 
 /* Size of one rank's IPC descriptor (mggcn_ipc_export). */

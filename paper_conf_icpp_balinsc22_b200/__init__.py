@@ -24,6 +24,8 @@ MGGCN_F_OVERLAP, MGGCN_F_RELU_LAST, MGGCN_F_TF32X1, MGGCN_F_NO_BCAST, MGGCN_F_PR
 MGGCN_F_NO_COALESCE = 64
 MGGCN_F_CACHE_L0 = 128
 MGGCN_F_IPC = 256
+MGGCN_F_REPL2 = 512        # 1.5D, replication factor c = 2
+MGGCN_F_REPLICA1 = 1024    # with MGGCN_F_REPL2, nlocal = 1: this process is replica 1
 MGGCN_IPC_BLOB_BYTES = 128
 PROFILE_CLASSES = ("spmm", "gemm", "loss", "adam", "bcast", "allreduce", "other")
 

@@ -117,6 +117,15 @@ bool ipc_stream_memops_available();
 cudaError_t stream_write_u32(cudaStream_t s, uint32_t* addr, uint32_t value);
 cudaError_t stream_wait_u32(cudaStream_t s, const uint32_t* addr, uint32_t value);
 int ipc_alloc_base(const void* ptr, void** base, size_t* size);
+// 1.5D (c = 2) SpMM finish: the two replicas of
+// a row block hold partial sums over disjoint column-block sets; pair_sum adds
+// them (a + b, commutative: both copies end bitwise equal) and applies the
+// last-stage epilogue (row scale of Eq. 2, ReLU of Eq. 7) to both copies;
+// rows_epilogue applies it in place after an NCCL pair all-reduce.
+cudaError_t launch_pair_sum_epilogue(float* a, float* b, int64_t rows, int width, int64_t ld, const float* rowscale,
+                                     int relu, cudaStream_t s);
+cudaError_t launch_rows_epilogue(float* a, int64_t rows, int width, int64_t ld, const float* rowscale, int relu,
+                                 cudaStream_t s);
 cudaError_t launch_sum_ranks_f32(const float* const* in, int nin, float* out, int64_t count, cudaStream_t s);
 cudaError_t launch_sum_ranks_scalar(const double* const* in_d, const int64_t* const* in_i, int nin, double* out_d,
                                     int64_t* out_i, cudaStream_t s);

@@ -279,6 +279,32 @@ __global__ void splitk_reduce_kernel(const float* __restrict__ partial, int k_ch
     }
 }
 
+// 1.5D pair finish: v = (a + b) [* rowscale[r]] [max(., 0)], written to a
+// (and b when given).  float4 over the first ceil(width / 4) * 4 columns
+// (ld is a multiple of 4; padding columns stay 0 + 0 = 0).
+__global__ void pair_epilogue_kernel(float4* __restrict__ a, float4* __restrict__ b, int64_t rows, int w4,
+                                     int64_t ld4, const float* __restrict__ rowscale, int relu) {
+    const int64_t total = rows * w4;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = i / w4;
+        const int64_t o = r * ld4 + (i - r * w4);
+        float4 v = a[o];
+        if (b) {
+            const float4 u = b[o];
+            v.x += u.x; v.y += u.y; v.z += u.z; v.w += u.w;
+        }
+        if (rowscale) {
+            const float sc = rowscale[r];
+            v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
+        }
+        if (relu) {
+            v.x = fmaxf(v.x, 0.f); v.y = fmaxf(v.y, 0.f); v.z = fmaxf(v.z, 0.f); v.w = fmaxf(v.w, 0.f);
+        }
+        a[o] = v;
+        if (b) b[o] = v;
+    }
+}
+
 }  // namespace
 
 cudaError_t launch_softmax_ce(float* Z, int64_t n, int C, int64_t ld, const int32_t* y, const int64_t* ntrain,
@@ -381,3 +407,32 @@ void count_launches(int n) { g_launches.fetch_add(n, std::memory_order_relaxed);
 }  // namespace mggcn
 
 extern "C" int64_t mggcn_kernel_launch_count(void) { return (int64_t)mggcn::g_launches.load(); }
+
+namespace mggcn {
+
+static cudaError_t launch_pair(float* a, float* b, int64_t rows, int width, int64_t ld, const float* rowscale,
+                               int relu, cudaStream_t s) {
+    if (rows <= 0) return cudaSuccess;
+    if ((ld & 3) || (reinterpret_cast<uintptr_t>(a) & 15) || (reinterpret_cast<uintptr_t>(b) & 15))
+        return cudaErrorInvalidValue;
+    const int w4 = (width + 3) / 4;
+    const int64_t total = rows * w4;
+    int64_t blocks = (total + 255) / 256;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    pair_epilogue_kernel<<<(unsigned)blocks, 256, 0, s>>>(reinterpret_cast<float4*>(a), reinterpret_cast<float4*>(b),
+                                                          rows, w4, ld / 4, rowscale, relu);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pair_sum_epilogue(float* a, float* b, int64_t rows, int width, int64_t ld, const float* rowscale,
+                                     int relu, cudaStream_t s) {
+    return launch_pair(a, b, rows, width, ld, rowscale, relu, s);
+}
+
+cudaError_t launch_rows_epilogue(float* a, int64_t rows, int width, int64_t ld, const float* rowscale, int relu,
+                                 cudaStream_t s) {
+    return launch_pair(a, nullptr, rows, width, ld, rowscale, relu, s);
+}
+
+}  // namespace mggcn

@@ -101,6 +101,7 @@ void coalesce(const HostTile& t, HostTile& o) {
 struct Rank {
     const mggcn_part_s* part = nullptr;
     int rank = 0;
+    int rep = 0;                     // replica index (MGGCN_F_REPL2: rank (i, r) = r * P' + i)
     int64_t rows = 0, row_off = 0;   // row_off: offset inside the model's local rows
     std::vector<SpmmTile> F, B;
     std::vector<HostItems> hF, hB;
@@ -138,7 +139,8 @@ struct Rank {
 }  // namespace
 
 struct mggcn_model_s {
-    int P = 1, nlocal = 1;
+    int P = 1, nlocal = 1;          // P: row blocks of the partition (P' under MGGCN_F_REPL2)
+    int c = 1;                      // replication factor (2 with MGGCN_F_REPL2)
     uint32_t flags = 0;
     int L = 0;
     std::vector<int64_t> d, ld;     // dims and padded leading dims (multiple of 4)
@@ -159,6 +161,7 @@ struct mggcn_model_s {
     cudaStream_t cs = nullptr, ms = nullptr;
     cudaEvent_t ev_begin = nullptr, ev_comm_end = nullptr, ev_tmp = nullptr, ev_wg = nullptr, ev_comm_done = nullptr;
     ncclComm_t comm = nullptr;
+    ncclComm_t comm_bc = nullptr, comm_pair = nullptr;   // 1.5D: replica group, row-block pair
     int state = ST_READY;
     int poisoned = 0;
     int64_t t = 0;
@@ -218,6 +221,9 @@ namespace {
         int _rc = (expr);                \
         if (_rc != MGGCN_OK) return _rc; \
     } while (0)
+
+// 1.5D: replica `rep` computes the stages of the column blocks j with j mod c == rep
+inline bool in_set(const mggcn_model_s* m, int rep, int j) { return m->c == 1 || j % m->c == rep; }
 
 // ---------------------------------------------------------------- profiling
 cudaEvent_t prof_event(mggcn_model_s* m) {
@@ -627,7 +633,110 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
     return MGGCN_OK;
 }
 
+// 1.5D (c = 2): rank (i, r) runs the stages of
+// the column blocks j in J_r = {j : j mod c = r} (its own block first when
+// i is in J_r, then ascending j); block j is broadcast by rank (j, r) inside
+// replica group r only, into BC[k % 2] for the k-th remote stage with the
+// same slot rule as the 1D schedule.  No stage applies the last-stage
+// epilogue: the two replicas' partial sums are added (NCCL all-reduce over
+// the row-block pair, or one loopback kernel per pair writing both copies)
+// and then scaled by 1/deg (Eq. 2) and passed through ReLU (Eq. 7).
+int remote_index_15d(const mggcn_model_s* m, int q, const Rank& r) {
+    int k = 0;
+    for (int j = 0; j < q; ++j)
+        if (j != r.rank && in_set(m, r.rep, j)) ++k;
+    return k;
+}
+
+int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
+    const int P = m->P, c = m->c;
+    const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
+    const bool overlap = (m->flags & MGGCN_F_OVERLAP) != 0;
+    CK(cudaEventRecord(m->ev_begin, m->cs));
+    CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
+    std::vector<char> started(m->ranks.size(), 0);
+    for (size_t k = 0; k < m->ranks.size(); ++k) {      // own block first
+        Rank& r = m->ranks[k];
+        if (!in_set(m, r.rep, r.rank)) continue;
+        if (r.rows > 0) RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), 0));
+        started[k] = 1;
+    }
+    for (int q = 0; q < P; ++q) {
+        const int rq = q % c;                            // the replica group that needs block q
+        {
+            ProfScope ps(m, PC_BCAST, m->ms);
+            if (m->comm) {
+                Rank& r = m->ranks[0];
+                if (r.rep == rq) {
+                    const size_t count = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width;
+                    if (q == r.rank) {
+                        float* s = job.src(m, r, job.ctx);
+                        if (!nob && count) NK(ncclBroadcast(s, s, count, ncclFloat32, q, m->comm_bc, m->ms));
+                    } else {
+                        const int k = remote_index_15d(m, q, r), slot = k & 1;
+                        if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                        if (!nob && count)
+                            NK(ncclBroadcast(r.BC[slot], r.BC[slot], count, ncclFloat32, q, m->comm_bc, m->ms));
+                        CK(cudaEventRecord(r.ev_bc[slot], m->ms));
+                    }
+                }
+            } else {
+                Rank& root = m->ranks[rq * P + q];
+                const size_t bytes = (size_t)root.rows * (size_t)job.width * sizeof(float);
+                for (auto& r : m->ranks) {
+                    if (r.rep != rq || r.rank == q) continue;
+                    const int k = remote_index_15d(m, q, r), slot = k & 1;
+                    if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (!nob && bytes)
+                        CK(cudaMemcpyAsync(r.BC[slot], job.src(m, root, job.ctx), bytes, cudaMemcpyDeviceToDevice,
+                                           m->ms));
+                    CK(cudaEventRecord(r.ev_bc[slot], m->ms));
+                }
+            }
+        }
+        for (size_t i = 0; i < m->ranks.size(); ++i) {
+            Rank& r = m->ranks[i];
+            if (r.rep != rq || r.rank == q) continue;
+            const int k = remote_index_15d(m, q, r), slot = k & 1;
+            CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
+            if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], started[i] ? SPMM_ACCUM : 0));
+            started[i] = 1;
+            CK(cudaEventRecord(r.ev_free[slot], m->cs));
+        }
+    }
+    CK(cudaEventRecord(m->ev_comm_end, m->ms));
+    CK(cudaStreamWaitEvent(m->cs, m->ev_comm_end, 0));
+    // ---- pair reduction of the replicas' partial sums, then the last-stage epilogue
+    const int relu = job.relu ? 1 : 0;
+    if (m->comm) {
+        Rank& r = m->ranks[0];
+        float* out = job.dst(m, r, job.ctx);
+        CK(cudaEventRecord(m->ev_tmp, m->cs));
+        CK(cudaStreamWaitEvent(m->ms, m->ev_tmp, 0));
+        {
+            ProfScope ps(m, PC_ALLRED, m->ms);
+            if (r.rows) NK(ncclAllReduce(out, out, (size_t)r.rows * (size_t)job.width, ncclFloat32, ncclSum,
+                                         m->comm_pair, m->ms));
+        }
+        CK(cudaEventRecord(m->ev_tmp, m->ms));
+        CK(cudaStreamWaitEvent(m->cs, m->ev_tmp, 0));
+        ProfScope ps(m, PC_SPMM, m->cs);
+        CK(launch_rows_epilogue(out, r.rows, (int)job.width, job.width, job.use_rowscale ? r.inv_deg : nullptr, relu,
+                                m->cs));
+    } else {
+        ProfScope ps(m, PC_SPMM, m->cs);
+        for (int i = 0; i < P; ++i) {
+            Rank& a = m->ranks[i];
+            Rank& b = m->ranks[P + i];
+            CK(launch_pair_sum_epilogue(job.dst(m, a, job.ctx), job.dst(m, b, job.ctx), a.rows, (int)job.width,
+                                        job.width, job.use_rowscale ? a.inv_deg : nullptr, relu, m->cs));
+        }
+    }
+    return MGGCN_OK;
+}
+
 int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
+    if (m->c > 1) return staged_spmm_15d(m, job);
     const int P = m->P;
     const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
     const bool overlap = (m->flags & MGGCN_F_OVERLAP) != 0;
@@ -785,14 +894,27 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
     m->nlocal = nlocal;
     m->flags = flags;
     m->L = L;
-    if (nlocal != 1 && nlocal != m->P) {
-        set_error("model: nlocal must be 1 or P (loopback)");
+    m->c = (flags & MGGCN_F_REPL2) ? 2 : 1;
+    if ((flags & MGGCN_F_REPLICA1) && (m->c == 1 || nlocal != 1)) {
+        set_error("model: MGGCN_F_REPLICA1 needs MGGCN_F_REPL2 and nlocal = 1");
+        return MGGCN_EINVAL;
+    }
+    if (m->c > 1 && (m->P < 2 || m->P % m->c)) {
+        set_error("model: MGGCN_F_REPL2 needs an even number P' >= 2 of row blocks");
+        return MGGCN_EINVAL;
+    }
+    if (m->c > 1 && (flags & MGGCN_F_IPC)) {
+        set_error("model: MGGCN_F_REPL2 is not implemented for MGGCN_F_IPC");
+        return MGGCN_EUNSUPPORTED;
+    }
+    if (nlocal != 1 && nlocal != m->c * m->P) {
+        set_error("model: nlocal must be 1 or P (loopback; 2P' with MGGCN_F_REPL2)");
         return MGGCN_EINVAL;
     }
     for (int i = 0; i < nlocal; ++i) {
         const mggcn_part_s* pi = parts[i];
         if (!pi || pi->P != m->P || pi->n != p0->n || pi->pattern != p0->pattern ||
-            (nlocal > 1 && pi->rank != i) || pi->perm != p0->perm) {
+            (nlocal > 1 && pi->rank != i % m->P) || pi->perm != p0->perm) {
             set_error("model: parts must come from the same graph / P / seed (and be ranks 0..P-1 in loopback)");
             return MGGCN_EINVAL;
         }
@@ -828,6 +950,7 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         Rank& r = m->ranks[i];
         r.part = parts[i];
         r.rank = parts[i]->rank;
+        r.rep = nlocal > 1 ? i / m->P : ((flags & MGGCN_F_REPLICA1) ? 1 : 0);
         r.rows = parts[i]->nrows();
         r.row_off = off;
         off += r.rows;
@@ -870,6 +993,7 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
     auto spmm_work = [&](int dir, int64_t width) {
         for (auto& r : m->ranks)
             for (int j = 0; j < m->P; ++j) {
+                if (!in_set(m, r.rep, j)) continue;      // 1.5D: the other replica's stages
                 const HostTile& t = dir == 0 ? r.tF(j) : r.tB(j);
                 const double nnz = (double)t.rowptr.back();
                 m->w_spmm_bytes += nnz * (t.val.empty() ? 4.0 : 8.0) + 4.0 * (double)(t.nrows + 1) +
@@ -940,6 +1064,8 @@ static void destroy(mggcn_model_s* m) {
         cudaEventDestroy(std::get<2>(rec));
     }
     for (auto e : m->prof_pool) cudaEventDestroy(e);
+    if (m->comm_bc) ncclCommDestroy(m->comm_bc);
+    if (m->comm_pair) ncclCommDestroy(m->comm_pair);
     if (m->comm) ncclCommDestroy(m->comm);
     for (void* p : m->ipc_opened)
         if (p) cudaIpcCloseMemHandle(p);
@@ -1031,11 +1157,20 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
         ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
         const char* mc = getenv("MGGCN_NCCL_MAX_CTAS");
         cfg.maxCTAs = mc ? atoi(mc) : 16;
-        ncclResult_t nr = ncclCommInitRankConfig(&m->comm, m->P, id, m->ranks[0].rank, &cfg);
+        const Rank& r0 = m->ranks[0];
+        ncclResult_t nr = ncclCommInitRankConfig(&m->comm, m->c * m->P, id, r0.rep * m->P + r0.rank, &cfg);
         if (nr != ncclSuccess) {
             set_error(std::string("model_create: ncclCommInitRankConfig: ") + ncclGetErrorString(nr));
             m->comm = nullptr;
             return fail(MGGCN_ENCCL);
+        }
+        if (m->c > 1) {   // 1.5D: replica group (broadcasts, rank = block index) and row-block pair
+            nr = ncclCommSplit(m->comm, r0.rep, r0.rank, &m->comm_bc, &cfg);
+            if (nr == ncclSuccess) nr = ncclCommSplit(m->comm, r0.rank, r0.rep, &m->comm_pair, &cfg);
+            if (nr != ncclSuccess) {
+                set_error(std::string("model_create: ncclCommSplit: ") + ncclGetErrorString(nr));
+                return fail(MGGCN_ENCCL);
+            }
         }
     }
     if (cudaStreamSynchronize(m->cs) != cudaSuccess) {
@@ -1282,8 +1417,10 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
     }
     // ---- loss: |T|, logits out, fused CE fwd+bwd in place (Eq. 19)
     if (m->ipc && m->sc_seq) RC(ipc_wait_peers(m, m->cs, 5, m->sc_seq));   // peers read my last scalars
-    for (auto& r : m->ranks)
+    for (auto& r : m->ranks) {
         CK(launch_count_labelled(r.y, r.rows, reinterpret_cast<int64_t*>(r.ce_partial), r.ntrain_local, m->cs));
+        if (r.rep) CK(cudaMemsetAsync(r.ntrain_local, 0, 8, m->cs));   // 1.5D: counted once (replica 0)
+    }
     RC(reduce_all(m, true));
     if (logits) {
         for (auto& r : m->ranks)
@@ -1298,6 +1435,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
                              prescale ? r.inv_deg : nullptr, (m->flags & MGGCN_F_RELU_LAST) ? 1 : 0, r.ce_partial,
                              m->cs));
         CK(launch_sum_partials(r.ce_partial, kCeBlocks, r.loss_local, m->cs));
+        if (r.rep) CK(cudaMemsetAsync(r.loss_local, 0, 8, m->cs));
     }
     RC(reduce_all(m, false));
     if (loss) {
@@ -1396,7 +1534,7 @@ static int wgrad_reduce(mggcn_model_s* m, int l) {
         float* dst = (m->nlocal > 1 ? r.WG_local : m->ipc ? m->WGp : m->WG) + m->woff[l];
         if (m->ipc && m->wg_seq >= (uint32_t)m->L)
             RC(ipc_wait_peers(m, m->cs, 3, m->wg_seq + 1 - m->L));   // peers finished reading this slice
-        if (r.has_wgrad[l]) {
+        if (r.has_wgrad[l] && r.rep == 0) {      // 1.5D: replica 0 contributes W_G (replica 1: zeros)
             {
                 ProfScope ps(m, PC_GEMM, m->cs);
                 CK(gemm_launch(r.g_wgrad[l], m->cs));

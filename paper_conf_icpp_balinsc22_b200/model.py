@@ -7,8 +7,8 @@ from __future__ import annotations
 
 import numpy as np
 
-from . import (MGGCN_F_IPC, MGGCN_F_OVERLAP, mggcn_backward, mggcn_epoch_work, mggcn_forward, mggcn_get_adam,
-               mggcn_get_grad, mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free,
+from . import (MGGCN_F_IPC, MGGCN_F_OVERLAP, MGGCN_F_REPL2, MGGCN_F_REPLICA1, mggcn_backward, mggcn_epoch_work,
+               mggcn_forward, mggcn_get_adam, mggcn_get_grad, mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free,
                mggcn_ipc_connect, mggcn_ipc_export, mggcn_load_csr, mggcn_model_create, mggcn_model_free,
                mggcn_part_free, mggcn_part_info, mggcn_partition, mggcn_prefetch, mggcn_set_adam,
                mggcn_set_weights, mggcn_step, mggcn_workspace_bytes)
@@ -21,27 +21,40 @@ class GCN:
     """
 
     def __init__(self, n, rowptr, col, vals, dims, P=1, rank=0, perm_seed=0, flags=MGGCN_F_OVERLAP,
-                 loopback=False, nccl_id=None, device=None, graph=None, comm="nccl", ipc_exchange=None):
+                 loopback=False, nccl_id=None, device=None, graph=None, comm="nccl", ipc_exchange=None,
+                 replicas=1):
         """comm = "nccl" (nccl_id from mggcn_nccl_unique_id, shared by the caller) or "ipc"
         (MGGCN_F_IPC: peers map each other's workspaces; ipc_exchange(blob) -> list of the P
-        blobs in rank order, e.g. dist.ipc_exchange over torch.distributed)."""
+        blobs in rank order, e.g. dist.ipc_exchange over torch.distributed).
+
+        replicas = 2: 1.5D (MGGCN_F_REPL2).  P is then the TOTAL number of
+        ranks (P/2 row blocks); `rank` = replica * P/2 + block.  In loopback the model's
+        rows are the n permuted rows twice (replica 0 then replica 1)."""
         import torch
         self.torch = torch
         self.dims = tuple(int(d) for d in dims)
         self.L = len(self.dims) - 1
         self.P, self.rank, self.loopback = P, rank, loopback
         own_graph = graph is None
+        if replicas not in (1, 2) or P % replicas:
+            raise ValueError("replicas must be 1 or 2 and divide P")
+        self.replicas = replicas
+        Pb = P // replicas                                   # row blocks
+        if replicas == 2:
+            flags |= MGGCN_F_REPL2
+            if not loopback and rank // Pb == 1:
+                flags |= MGGCN_F_REPLICA1
         g = mggcn_load_csr(n, rowptr, col, vals) if own_graph else graph
         try:
             ranks = list(range(P)) if loopback else [rank]
-            self.parts = [mggcn_partition(g, P, r, perm_seed) for r in ranks]
+            self.parts = [mggcn_partition(g, Pb, r % Pb, perm_seed) for r in ranks]
         finally:
             if own_graph:
                 mggcn_graph_free(g)
         info = mggcn_part_info(self.parts[0])
         self.n, self.p, self.perm = info["n"], info["p"], info["perm"]
-        self.row0 = 0 if loopback else int(self.p[rank])
-        self.rows = n if loopback else int(self.p[rank + 1] - self.p[rank])
+        self.row0 = 0 if loopback else int(self.p[rank % Pb])
+        self.rows = n if loopback else int(self.p[rank % Pb + 1] - self.p[rank % Pb])
         self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
         self.comm = "loopback" if loopback or P == 1 else comm
         if self.comm == "ipc":
@@ -76,7 +89,10 @@ class GCN:
         X = np.asarray(X)
         Xp = np.empty_like(X)
         Xp[self.perm] = X
-        return np.ascontiguousarray(Xp[self.row0:self.row0 + self.rows])
+        own = Xp[self.row0:self.row0 + self.rows]
+        if self.loopback and self.replicas > 1:          # every replica holds the rows again
+            own = np.concatenate([own] * self.replicas)
+        return np.ascontiguousarray(own)
 
     def set_weights(self, Ws):
         for l, W in enumerate(Ws):

@@ -127,3 +127,37 @@ def test_partition_cora_shaped_p1(mg):
     w = gen.WORKLOADS["cora"]
     rp, col = gen.rmat_csr(w.n, w.m, w.seed_G)
     _compare_part(mg, w.n, rp, col, None, 1, seed=w.perm_seed)
+
+
+def test_repl2_model_plan_validation(mg):
+    """1.5D (MGGCN_F_REPL2) host-side plan checks: loopback needs the
+    2P' parts replica-major (part k mod P'), P' must be even, replica 1 is per-process
+    only, and the IPC backend is not implemented for it.  The per-rank buffer plan of
+    a replicated rank equals that of the 1D rank owning the same row block."""
+    n, m = 4096, 60000
+    rp, col = gen.rmat_csr(n, m, 5)
+    g = mg.mggcn_load_csr(n, rp, col)
+    dims = (16, 32, 8)
+    R2, R1, IPC = mg.MGGCN_F_REPL2, mg.MGGCN_F_REPLICA1, mg.MGGCN_F_IPC
+    try:
+        parts2 = [mg.mggcn_partition(g, 2, i, 3) for i in range(2)]
+        parts3 = [mg.mggcn_partition(g, 3, i, 3) for i in range(3)]
+        b_loop = mg.mggcn_workspace_bytes(parts2 + parts2, dims, R2)
+        b_1d = mg.mggcn_workspace_bytes(parts2, dims, 0)
+        assert b_loop > b_1d
+        one = mg.mggcn_workspace_bytes(parts2[:1], dims, R2)
+        assert one == mg.mggcn_workspace_bytes(parts2[:1], dims, R2 | R1) == mg.mggcn_workspace_bytes(parts2[:1], dims, 0)
+        bad = [(parts2 + parts2[::-1], R2, mg.MGGCN_EINVAL),       # replica-major order violated
+               (parts2, R2, mg.MGGCN_EINVAL),                       # loopback needs 2P' parts
+               (parts3 + parts3, R2, mg.MGGCN_EINVAL),              # P' odd
+               (parts2[:1], R1, mg.MGGCN_EINVAL),                   # REPLICA1 without REPL2
+               (parts2 + parts2, R2 | R1, mg.MGGCN_EINVAL),         # REPLICA1 in loopback
+               (parts2[:1], R2 | IPC, mg.MGGCN_EUNSUPPORTED)]
+        for parts, flags, code in bad:
+            with pytest.raises(mg.MggcnError) as ei:
+                mg.mggcn_workspace_bytes(parts, dims, flags)
+            assert ei.value.code == code, (flags, ei.value)
+        for p in parts2 + parts3:
+            mg.mggcn_part_free(p)
+    finally:
+        mg.mggcn_graph_free(g)

@@ -83,8 +83,10 @@ enum {
                                  broadcast inside replica group r only, so each rank receives
                                  n d / 2 values per SpMM instead of (P-1)/P n d), then the two
                                  replicas of a row block sum their partials (pair all-reduce)
-                                 and apply the row scale / ReLU.  GEMMs run on both replicas;
-                                 W_G, the loss and |T| are contributed by replica 0 only.
+                                 and apply the row scale / ReLU.  Only the ROOT replica of a
+                                 row block (r = i mod 2, the one that broadcasts it) computes
+                                 its GEMM products (H W, the input gradient) and contributes
+                                 W_G, the loss and |T|; the other replica adds zeros.
                                  Loopback: nlocal = 2P', parts[k] = part k mod P' (replica
                                  k / P').  NCCL: nlocal = 1, nccl id shared by all 2P'
                                  processes, MGGCN_F_REPLICA1 on the replica-1 processes.

@@ -224,6 +224,10 @@ namespace {
 
 // 1.5D: replica `rep` computes the stages of the column blocks j with j mod c == rep
 inline bool in_set(const mggcn_model_s* m, int rep, int j) { return m->c == 1 || j % m->c == rep; }
+// 1.5D: the replica of row block i that broadcasts it (i mod c) is its ROOT; only the root
+// needs the block's GEMM products (HW, the input gradient) and contributes W_G, the loss and
+// |T|; the other replica only adds its partial SpMM stages (every rank is a root in 1D)
+inline bool is_root(const mggcn_model_s* m, const Rank& r) { return in_set(m, r.rep, r.rank); }
 
 // ---------------------------------------------------------------- profiling
 cudaEvent_t prof_event(mggcn_model_s* m) {
@@ -1002,11 +1006,14 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
                 if (j != r.rank) m->w_bcast_bytes += 4.0 * (double)width * (double)t.ncols;
             }
     };
+    int64_t root_rows = 0;                           // 1.5D: GEMM products only on the root replica
+    for (auto& r : m->ranks)
+        if (is_root(m, r)) root_rows += r.rows;
     for (int l = 0; l < L; ++l) {
         const int64_t w = m->order[l] == G_ORDER ? m->d[l + 1] : m->d[l];
         if (!(l == 0 && (flags & MGGCN_F_CACHE_L0))) spmm_work(0, w);   // steady state: T0 cached
-        const double gf = 2.0 * (double)m->n_local * (double)m->d[l] * (double)m->d[l + 1];
-        m->w_gemm_flops += gf;                       // forward
+        const double gf = 2.0 * (double)root_rows * (double)m->d[l] * (double)m->d[l + 1];
+        m->w_gemm_flops += m->order[l] == G_ORDER ? gf : gf * (double)m->n_local / (double)std::max<int64_t>(root_rows, 1);
         m->w_gemm_flops += gf;                       // W_G
         if (l > 0) m->w_gemm_flops += gf;            // H_G
         if (m->order[l] == G_ORDER) spmm_work(1, m->d[l + 1]);   // backward SpMM (Eq. 9)
@@ -1395,7 +1402,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
         layer_ids[l] = l;
         if (m->order[l] == G_ORDER) {
             for (auto& r : m->ranks)
-                if (r.has_fwd[l]) {
+                if (r.has_fwd[l] && is_root(m, r)) {
                     ProfScope ps(m, PC_GEMM, m->cs);
                     CK(gemm_launch(r.g_fwd[l], m->cs));                                  // Eq. 5 -> HWB (Eq. 16)
                 }
@@ -1419,7 +1426,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
     if (m->ipc && m->sc_seq) RC(ipc_wait_peers(m, m->cs, 5, m->sc_seq));   // peers read my last scalars
     for (auto& r : m->ranks) {
         CK(launch_count_labelled(r.y, r.rows, reinterpret_cast<int64_t*>(r.ce_partial), r.ntrain_local, m->cs));
-        if (r.rep) CK(cudaMemsetAsync(r.ntrain_local, 0, 8, m->cs));   // 1.5D: counted once (replica 0)
+        if (!is_root(m, r)) CK(cudaMemsetAsync(r.ntrain_local, 0, 8, m->cs));   // 1.5D: counted once (root)
     }
     RC(reduce_all(m, true));
     if (logits) {
@@ -1435,7 +1442,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
                              prescale ? r.inv_deg : nullptr, (m->flags & MGGCN_F_RELU_LAST) ? 1 : 0, r.ce_partial,
                              m->cs));
         CK(launch_sum_partials(r.ce_partial, kCeBlocks, r.loss_local, m->cs));
-        if (r.rep) CK(cudaMemsetAsync(r.loss_local, 0, 8, m->cs));
+        if (!is_root(m, r)) CK(cudaMemsetAsync(r.loss_local, 0, 8, m->cs));
     }
     RC(reduce_all(m, false));
     if (loss) {
@@ -1534,7 +1541,7 @@ static int wgrad_reduce(mggcn_model_s* m, int l) {
         float* dst = (m->nlocal > 1 ? r.WG_local : m->ipc ? m->WGp : m->WG) + m->woff[l];
         if (m->ipc && m->wg_seq >= (uint32_t)m->L)
             RC(ipc_wait_peers(m, m->cs, 3, m->wg_seq + 1 - m->L));   // peers finished reading this slice
-        if (r.has_wgrad[l] && r.rep == 0) {      // 1.5D: replica 0 contributes W_G (replica 1: zeros)
+        if (r.has_wgrad[l] && is_root(m, r)) {   // 1.5D: the root replica contributes W_G (the other: zeros)
             {
                 ProfScope ps(m, PC_GEMM, m->cs);
                 CK(gemm_launch(r.g_wgrad[l], m->cs));
@@ -1592,7 +1599,7 @@ static int backward_impl(mggcn_model_s* m) {
             RC(wgrad_reduce(m, l));                                           // Eq. 10
             if (l > 0)
                 for (auto& r : m->ranks)
-                    if (r.has_igrad[l]) {
+                    if (r.has_igrad[l] && is_root(m, r)) {
                         ProfScope ps(m, PC_GEMM, m->cs);
                         CK(gemm_launch(r.g_igrad[l], m->cs));                 // Eq. 11 + Eq. 8 mask -> AHWB_{l-1}
                     }

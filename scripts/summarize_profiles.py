@@ -71,10 +71,11 @@ def main():
             if hdr and len(r) == len(hdr):
                 d = dict(zip(hdr, r))
                 launches.append((int(d["ID"]), d["Kernel Name"], float(d["Metric Value"])))
-        # second epoch only (after the warm-up epoch): from the 2nd adam launch boundary
+        # the timed epoch (the second of the bench's model, after one warm-up epoch): the launches
+        # after the first Adam's weight re-split up to and including the second Adam's
         adam_ids = [i for i, n, _ in launches if "adam_kernel" in n]
         if len(adam_ids) >= 2:
-            ep = [(i, n, t) for i, n, t in launches if adam_ids[-2] < i <= adam_ids[-1] + 3]
+            ep = [(i, n, t) for i, n, t in launches if adam_ids[0] + 3 < i <= adam_ids[1] + 3]
         else:
             ep = launches
         tot = sum(t for _, _, t in ep)

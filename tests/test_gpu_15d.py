@@ -114,8 +114,11 @@ def test_15d_broadcast_volume(mg):
     for P in (4, 8):
         g15 = GCN(w.n, rp, col, None, w.dims, P=P, perm_seed=w.perm_seed, loopback=True, replicas=2)
         g1 = GCN(w.n, rp, col, None, w.dims, P=P, perm_seed=w.perm_seed, loopback=True)
+        gb = GCN(w.n, rp, col, None, w.dims, P=P // 2, perm_seed=w.perm_seed, loopback=True)
         b15, b1 = g15.epoch_work()["bcast_bytes"], g1.epoch_work()["bcast_bytes"]
-        g15.close()
-        g1.close()
+        # GEMM work: only the root replica of a block multiplies -> the 1D work at P' row blocks
+        assert g15.epoch_work()["gemm_flops"] == gb.epoch_work()["gemm_flops"]
+        for gm in (g15, g1, gb):
+            gm.close()
         Pb = P // 2
         assert abs(b15 / b1 - (Pb - 1) / (P - 1)) < 1e-9, (P, b15, b1)

@@ -1,24 +1,27 @@
 """Small end-to-end run for compute-sanitizer: loopback P=2 Cora-shaped epoch,
-an SpMM-first config, and the three GEMM ops (ragged shapes)."""
+an SpMM-first config (112 classes: the 32-lane CE row groups), a 1.5D loopback
+epoch (MGGCN_F_REPL2, P = 4), and the three GEMM ops (ragged shapes)."""
 import os, sys
 import numpy as np, torch
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import gen
 import paper_conf_icpp_balinsc22_b200 as mg
 from paper_conf_icpp_balinsc22_b200 import GCN
-for dims, P, n, m in (((1433, 16, 7), 2, 2708, 10556), ((8, 32, 24, 5), 1, 3001, 60000)):
+for dims, P, n, m, c in (((1433, 16, 7), 2, 2708, 10556, 1), ((8, 128, 128, 112), 1, 3001, 60000, 1),
+                         ((100, 64, 47), 4, 3001, 60000, 2)):
     rp, col = gen.rmat_csr(n, m, 5)
     X = gen.features(n, dims[0], 6); y = gen.labels(n, dims[-1], 7, 100)
     Ws = [gen.glorot(dims[l], dims[l + 1], 8 + l) for l in range(len(dims) - 1)]
-    gm = GCN(n, rp, col, None, dims, P=P, perm_seed=9, loopback=P > 1, flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE)
+    gm = GCN(n, rp, col, None, dims, P=P, perm_seed=9, loopback=P > 1, flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE,
+             replicas=c)
     gm.set_weights(Ws)
     for host in (False, True):
         Xl, yl = gm.permute_rows(X), gm.permute_rows(y)
         Xin = Xl if host else torch.from_numpy(Xl).cuda()
         yin = yl if host else torch.from_numpy(yl).cuda()
-        loss = gm.forward(Xin, yin, logits=torch.empty((n, dims[-1]), device="cuda"))
+        loss = gm.forward(Xin, yin, logits=torch.empty((c * n, dims[-1]), device="cuda"))
         gm.backward(); gm.step()
-    print("epoch ok", dims, P, loss, flush=True)
+    print("epoch ok", dims, P, c, loss, flush=True)
     gm.close()
 for op, (M, N, K) in ((0, (300, 41, 602)), (1, (257, 256, 41)), (2, (602, 47, 1000))):
     rng = np.random.default_rng(op)

@@ -101,6 +101,29 @@ int main() {
     CK(cudaFuncSetAttribute(gather_mixed<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     CK(cudaFuncSetAttribute(gather_mixed<1>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     int* didx; CK(cudaMalloc(&didx, n_idx * 4));
+    // ---- SM scaling of plain LDG gathers (mode 0, no hot rows) from an L2-resident table:
+    // linear in the number of SMs => a per-SM (L1 fill) limit; flat => a shared L2 limit
+    if (getenv("SM_SWEEP")) {
+        const size_t rows = 60000;
+        float4* tab; CK(cudaMalloc(&tab, rows * kRowBytes)); CK(cudaMemset(tab, 0, rows * kRowBytes));
+        uint64_t s = 88172645463325252ull;
+        for (size_t i = 0; i < n_idx; ++i) { s ^= s << 13; s ^= s >> 7; s ^= s << 17; h[i] = (int)(s % rows); }
+        CK(cudaMemcpy(didx, h.data(), n_idx * 4, cudaMemcpyHostToDevice));
+        for (int g : {18, 37, 74, 111, 148}) {
+            gather_mixed<0><<<g, kThreads, smem>>>(tab, didx, n_idx, H, out);
+            CK(cudaDeviceSynchronize());
+            CK(cudaEventRecord(a));
+            for (int r = 0; r < 3; ++r) gather_mixed<0><<<g, kThreads, smem>>>(tab, didx, n_idx, H, out);
+            CK(cudaEventRecord(b)); CK(cudaEventSynchronize(b));
+            float ms; CK(cudaEventElapsedTime(&ms, a, b));
+            const double gbs = n_idx * (double)kRowBytes * 3 / (ms * 1e-3) / 1e9;
+            printf("{\"sm_sweep\": %d, \"table_MB\": %.1f, \"GBps\": %.1f, \"GBps_per_sm\": %.1f, \"B_per_clk_per_sm_at_1965\": %.1f}\n",
+                   g, rows * kRowBytes / 1048576.0, gbs, gbs / g, gbs / g / 1.965);
+            fflush(stdout);
+        }
+        CK(cudaFree(tab));
+        return 0;
+    }
     for (size_t rows : {60000ul, 232965ul}) {
         float4* tab; CK(cudaMalloc(&tab, rows * kRowBytes)); CK(cudaMemset(tab, 0, rows * kRowBytes));
         for (int C : {1, 2, 4, 8, 16}) {

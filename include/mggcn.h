@@ -187,6 +187,9 @@ int mggcn_get_weights(mggcn_model m, int32_t layer, float* W);
  *            stride is the library's padded ld (d_0 rounded up to 8) and that
  *            is 16-B aligned is read IN PLACE (no copy): it must then stay valid
  *            and unchanged until this epoch's mggcn_backward has completed.
+ *            A host X with the padded stride is copied with one contiguous
+ *            copy (fastest end-to-end path); any other stride goes through
+ *            a device staging chunk.  Padding columns are never read as data.
  *            NULL: use the inputs of the pending mggcn_prefetch.
  *   y_local  int32 labels of the same rows (host or device); -1 = unlabelled.
  *   loss     host out: global mean CE over labelled vertices (reading C5), or

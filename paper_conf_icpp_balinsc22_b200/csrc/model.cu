@@ -538,6 +538,10 @@ int copy_inputs(mggcn_model_s* m, int k, const float* X, int64_t ldx, const int3
                 CK(cudaMemcpy2DAsync(dst + r0 * m->ld[0], m->ld[0] * 4, stage, ldx * 4, m->d[0] * 4, nr,
                                      cudaMemcpyDeviceToDevice, s));
             }
+        } else if (ldx == m->ld[0]) {
+            // already in the padded layout (host or device): one contiguous copy; the padding
+            // columns are copied too and never read as data (GEMM tensor maps stop at d_0)
+            CK(cudaMemcpyAsync(dst, X + r.row_off * ldx, sizeof(float) * r.rows * ldx, cudaMemcpyDefault, s));
         } else {
             CK(cudaMemcpy2DAsync(dst, m->ld[0] * 4, X + r.row_off * ldx, ldx * 4, m->d[0] * 4, r.rows,
                                  cudaMemcpyDefault, s));

@@ -303,3 +303,41 @@ def test_state_errors(mg):
     with pytest.raises(mg.MggcnError) as e:
         GCN(200, rp, col, None, (8, 4, 16, 2))      # SpMM-first at l = 1
     assert e.value.code == mg.MGGCN_EUNSUPPORTED
+
+
+@pytest.mark.parametrize("dims", [(1433, 16, 7), (100, 256, 47)])
+def test_padded_host_inputs_with_nan_padding(mg, dims):
+    """Host X in the library's padded row layout (one contiguous H2D, mggcn.h) whose
+    padding columns hold NaN: padding is never read as data (GEMM tensor maps stop at
+    d_0; the SpMM-first T0 padding is ignored), so the epoch still matches the oracle.
+    Also through mggcn_prefetch (the e2e path of bench.py)."""
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    n, m = 2708, 10556
+    rp, col = gen.rmat_csr(n, m, 31)
+    X = gen.features(n, dims[0], 32)
+    y = gen.labels(n, dims[-1], 33)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 34 + l) for l in range(len(dims) - 1)]
+    pg = oracle.permute_graph(n, rp, col, None, seed=35)
+    ref = oracle.epoch(pg, X, y, Ws)
+    for P, use_prefetch in ((1, False), (2, True)):
+        gm = GCN(n, rp, col, None, dims, P=P, perm_seed=35, flags=mg.MGGCN_F_OVERLAP, loopback=P > 1)
+        gm.set_weights(Ws)
+        Xl, yl = gm.permute_rows(X), gm.permute_rows(y)
+        Xh = np.full((Xl.shape[0], gm.ld0), np.nan, dtype=np.float32)
+        Xh[:, :dims[0]] = Xl
+        Xh = torch.from_numpy(Xh).pin_memory()
+        yh = torch.from_numpy(yl).pin_memory()
+        logits = torch.empty((n, dims[-1]), dtype=torch.float32, device="cuda")
+        if use_prefetch:
+            gm.prefetch(Xh, yh)
+            loss = gm.forward(None, None, want_loss=True, logits=logits)
+        else:
+            loss = gm.forward(Xh, yh, want_loss=True, logits=logits)
+        gm.backward()
+        lib = {"perm": gm.perm, "logits": logits.cpu().numpy(), "loss": loss, "WG": gm.grads()}
+        gm.step()
+        lib["W"] = gm.get_weights()
+        lib["adam"] = [gm.adam_state(l) for l in range(len(Ws))]
+        gm.close()
+        assert np.isfinite(lib["logits"]).all()
+        compare(lib, ref, dims)

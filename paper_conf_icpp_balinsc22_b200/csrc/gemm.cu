@@ -32,8 +32,15 @@ namespace {
 constexpr int BM = 128;          // UMMA_M (cta_group::1)
 constexpr int BK = 32;           // 32 fp32 = 128 B = one SWIZZLE_128B row
 constexpr int kMaxBN = 128;
-constexpr int kThreads = 320;
-constexpr int kXfWarp0 = 4, kTmaWarp = 8, kMmaWarp = 9;
+#ifndef MGGCN_ROW_RAWB
+#define MGGCN_ROW_RAWB 0          // 1: B_lo recomputed in smem from the raw W tile; 0: B_lo loaded by TMA (faster: profiles/r01_row_gemm_sweep.log)
+#endif
+#ifndef MGGCN_ROW_XF_WARPS
+#define MGGCN_ROW_XF_WARPS 4
+#endif
+constexpr int kXfWarps = MGGCN_ROW_XF_WARPS;      // transform (lo split) warps of the row GEMM
+constexpr int kXfWarp0 = 4, kTmaWarp = 4 + kXfWarps, kMmaWarp = 5 + kXfWarps;
+constexpr int kThreads = (6 + kXfWarps) * 32;
 constexpr int kTmemCols = 256;   // 2 accumulators x 128 columns
 
 // shared-memory map (bytes from a 1024-B aligned base)
@@ -638,7 +645,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     if (threadIdx.x == 0) {
         for (int s = 0; s < NS; ++s) {
             mbar_init(full + s, 1);
-            mbar_init(xf + s, 128);
+            mbar_init(xf + s, kXfWarps * 32);
             mbar_init(empty + s, 1);
         }
         for (int s = 0; s < 2; ++s) {
@@ -662,7 +669,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
 
     if (warp == kTmaWarp) {
         if (lane == 0) {
-            const uint32_t bytes = (uint32_t)(BM * kRowBK * 4 + BN * kRowBK * 4 * (x1 ? 1 : 2));
+            const uint32_t bytes = (uint32_t)(BM * kRowBK * 4 + BN * kRowBK * 4 * (MGGCN_ROW_RAWB || x1 ? 1 : 2));
             int s = 0;
             uint32_t ph = 0;
             for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
@@ -673,26 +680,31 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                     mbar_expect_tx(full + s, bytes);
                     tma_load_2d(st, &tmA, kb * kRowBK, mt * BM, full + s);
                     tma_load_2d(st + 16384, &tmBh, kb * kRowBK, nt * BN, full + s);
-                    if (!x1) tma_load_2d(st + kBlo, &tmBl, kb * kRowBK, nt * BN, full + s);
+                    if (!MGGCN_ROW_RAWB && !x1) tma_load_2d(st + kBlo, &tmBl, kb * kRowBK, nt * BN, full + s);
                     if (++s == NS) { s = 0; ph ^= 1; }
                 }
             }
         }
-    } else if (warp >= kXfWarp0 && warp < kXfWarp0 + 4) {
+    } else if (warp >= kXfWarp0 && warp < kXfWarp0 + kXfWarps) {
         const int t = threadIdx.x - kXfWarp0 * 32;
         int s = 0;
         uint32_t ph = 0;
         for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
             for (int kb = 0; kb < nkb; ++kb) {
                 float4* a = reinterpret_cast<float4*>(smem + kRowStage0 + s * SB);
-                float4* al = reinterpret_cast<float4*>(smem + kRowStage0 + s * SB + 8192);
                 mbar_wait(full + s, ph);
-#pragma unroll
-                for (int c = t; c < BM * 4; c += 128) {
-                    float4 v = a[c], h, l;
+                // raw A [0, 512) -> lo at +512; raw B [1024, 1024 + 4 BN) -> lo at +4 BN (float4
+                // units, same swizzled offsets).  3xTF32: the MMA reads a raw x as hi = x &
+                // 0xFFFFE000 itself, so only lo = x - hi is written (B's lo is recomputed per
+                // tile instead of loaded: 40 -> 24 KB of TMA per k block at BN = 256).
+                const int nA = BM * 4, nT = nA + (MGGCN_ROW_RAWB ? BN * 4 : 0);
+                for (int c = t; c < nT; c += kXfWarps * 32) {
+                    const int src = c < nA ? c : 1024 + (c - nA);
+                    const int dst = src + (c < nA ? nA : BN * 4);
+                    float4 v = a[src], h, l;
                     split4(v, h, l, x1);
-                    if (x1) a[c] = h;      // 3xTF32: the MMA reads x as hi = x & 0xFFFFE000 itself
-                    else al[c] = l;
+                    if (x1) a[src] = h;    // 1xTF32: round to nearest in place
+                    else a[dst] = l;
                 }
                 fence_proxy_async();
                 mbar_arrive(xf + s);
@@ -816,7 +828,9 @@ __global__ void split_weights_kernel(const float* __restrict__ W, int din, int d
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
         const int c = (int)(i / dout), k = (int)(i % dout);
         float hi, lo;
-        split_tf32(W[c * ldw + k], hi, lo, x1 != 0);
+        const float w = W[c * ldw + k];
+        split_tf32(w, hi, lo, x1 != 0);
+        if (!x1) hi = w;   // the raw value: the MMA reads it as tf32 by truncation (= the hi part)
         if (t_hi) {
             t_hi[(int64_t)k * ldt + c] = hi;
             t_lo[(int64_t)k * ldt + c] = lo;

@@ -136,15 +136,26 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
         qc[ch] = q < w4 ? q : 0;      // clamped: always a valid address, result unused
     }
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    // persistent warps: static stride over the work items (hub segments first)
-    for (int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; wi < n_items; wi += nwarps) {
-        const int4 it = __ldg(items + wi);
+    // Persistent warps: static stride over the work items (hub segments first).
+    // Software-pipelined across items: the descriptor of the item two strides
+    // ahead and the first index chunk of the next item are loaded while the
+    // current item gathers, so a short row (Products-shaped: ~50 entries, 1-2
+    // chunks) does not pay item -> index -> gather as three serial latencies.
+    const int4 kNone = make_int4(0, 0, 0, -1);
+    int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    int4 it = wi < n_items ? __ldg(items + wi) : kNone;
+    int4 itn = wi + nwarps < n_items ? __ldg(items + wi + nwarps) : kNone;
+    int cur_c = (it.y + lane < it.z) ? ld_stream_i32(col + it.y + lane) : 0;
+    float cur_v = 0.f;
+    if (VALS) cur_v = (it.y + lane < it.z) ? ld_stream_f32(val + it.y + lane) : 0.f;
+    for (; wi < n_items; wi += nwarps) {
+        const int4 it2 = wi + 2 * nwarps < n_items ? __ldg(items + wi + 2 * nwarps) : kNone;
+        const float scale = (rowscale && it.w < 0) ? __ldg(rowscale + it.x) : 1.f;
         float4 acc[CH];
 #pragma unroll
         for (int c = 0; c < CH; ++c) acc[c] = make_float4(0.f, 0.f, 0.f, 0.f);
-        int nxt_c = (it.y + lane < it.z) ? ld_stream_i32(col + it.y + lane) : 0;
-        float nxt_v = 0.f;
-        if (VALS) nxt_v = (it.y + lane < it.z) ? ld_stream_f32(val + it.y + lane) : 0.f;
+        int nxt_c = cur_c;
+        float nxt_v = cur_v;
         for (int base = it.y; base < it.z; base += 32) {
             const int cnt = min(32, it.z - base);
             const int my_c = nxt_c;
@@ -153,6 +164,10 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 const int e = base + 32 + lane;
                 nxt_c = e < it.z ? ld_stream_i32(col + e) : 0;
                 if (VALS) nxt_v = e < it.z ? ld_stream_f32(val + e) : 0.f;
+            } else {                      // ... or the next item's first chunk
+                const int e = itn.y + lane;
+                nxt_c = e < itn.z ? ld_stream_i32(col + e) : 0;
+                if (VALS) nxt_v = e < itn.z ? ld_stream_f32(val + e) : 0.f;
             }
             int k0 = 0;
             for (; k0 + U * S <= cnt; k0 += U * S) {
@@ -192,6 +207,11 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                     for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_fma(a[u], x[u][ch], acc[ch]);
             }
         }
+        if (it.z <= it.y) {               // empty row: still fetch the next item's first chunk
+            const int e = itn.y + lane;
+            nxt_c = e < itn.z ? ld_stream_i32(col + e) : 0;
+            if (VALS) nxt_v = e < itn.z ? ld_stream_f32(val + e) : 0.f;
+        }
         // combine the S slots (fixed xor tree => deterministic)
 #pragma unroll
         for (int off = G; off < 32; off <<= 1)
@@ -207,7 +227,6 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 }
             } else {
                 float4* orow = out + (int64_t)it.x * ldo4;
-                const float scale = rowscale ? __ldg(rowscale + it.x) : 1.f;
 #pragma unroll
                 for (int ch = 0; ch < CH; ++ch) {
                     const int q = cl + ch * G;
@@ -215,6 +234,10 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 }
             }
         }
+        cur_c = nxt_c;
+        cur_v = nxt_v;
+        it = itn;
+        itn = it2;
     }
 }
 

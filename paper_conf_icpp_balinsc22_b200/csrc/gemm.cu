@@ -35,6 +35,9 @@ constexpr int kMaxBN = 128;
 #ifndef MGGCN_ROW_RAWB
 #define MGGCN_ROW_RAWB 0          // 1: B_lo recomputed in smem from the raw W tile; 0: B_lo loaded by TMA (faster: profiles/r01_row_gemm_sweep.log)
 #endif
+#ifndef MGGCN_ROW_PF
+#define MGGCN_ROW_PF 0            // row GEMM: L2 prefetch of the A box this many k blocks ahead (0 = off)
+#endif
 #ifndef MGGCN_ROW_XF_WARPS
 #define MGGCN_ROW_XF_WARPS 4
 #endif
@@ -94,6 +97,12 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* tm, in
             smem_u32(dst)),
         "l"((uint64_t)tm), "r"(c0), "r"(c1), "r"(smem_u32(bar))
         : "memory");
+}
+
+// L2 prefetch of a tensor box (no shared-memory destination, no completion)
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* tm, int c0, int c1) {
+    asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"((uint64_t)tm), "r"(c0), "r"(c1)
+                 : "memory");
 }
 
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
@@ -676,6 +685,12 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
                 for (int kb = 0; kb < nkb; ++kb) {
                     uint8_t* st = smem + kRowStage0 + s * SB;
+                    if (MGGCN_ROW_PF > 0) {   // A streams from DRAM: warm L2 ahead of the ring
+                        const int kp = kb + MGGCN_ROW_PF;
+                        if (kp < nkb) tma_prefetch_2d(&tmA, kp * kRowBK, mt * BM);
+                        else if (tile + (int)gridDim.x < total_tiles)
+                            tma_prefetch_2d(&tmA, (kp - nkb) * kRowBK, ((tile + gridDim.x) / p.n_tiles) * BM);
+                    }
                     mbar_wait(empty + s, ph ^ 1);
                     mbar_expect_tx(full + s, bytes);
                     tma_load_2d(st, &tmA, kb * kRowBK, mt * BM, full + s);

@@ -38,6 +38,9 @@ constexpr int kMaxBN = 128;
 #ifndef MGGCN_ROW_PF
 #define MGGCN_ROW_PF 0            // row GEMM: L2 prefetch of the A box this many k blocks ahead (0 = off)
 #endif
+#ifndef MGGCN_ROW_DBG
+#define MGGCN_ROW_DBG 0           // TIMING EXPERIMENTS ONLY (results invalid): 1 no MMAs, 2 no lo split, 4 no TMA loads
+#endif
 #ifndef MGGCN_ROW_XF_WARPS
 #define MGGCN_ROW_XF_WARPS 4
 #endif
@@ -627,9 +630,62 @@ __device__ __forceinline__ void bulk_wait_read() {
 }
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 
+// ---- CTA-pair (cta_group::2) helpers
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// arrive on the barrier at the same shared-memory offset in CTA `rank` of the cluster
+__device__ __forceinline__ void mbar_arrive_cluster(uint64_t* bar, uint32_t rank) {
+    uint32_t ra;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(bar)), "r"(rank));
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred P1;\n"
+        "WAITC_%=:\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P1, [%0], %1;\n\t"
+        "@!P1 bra WAITC_%=;\n}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void mma_tf32_pair(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                              uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+        : "memory");
+}
+// completion of the pair's MMAs arrives on the barrier at this offset in BOTH CTAs
+__device__ __forceinline__ void mma_commit_pair(uint64_t* bar) {
+    asm volatile(
+        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+            smem_u32(bar)),
+        "h"((unsigned short)3)
+        : "memory");
+}
+
 // byte offset of (row r, 16-B chunk q) in a [128][32 fp32] SWIZZLE_128B tile
 __device__ __forceinline__ int sw128_off(int r, int q) { return r * 128 + ((q ^ (r & 7)) << 4); }
 
+// PAIR (opt-in, MGGCN_ROW_PAIR=1): a cluster of two CTAs on one TPC computes a
+// 256 x BN tile with tcgen05.mma.cta_group::2 (M = 256): each CTA stages its
+// own 128 rows of A and HALF of B (BN/2 rows of W^T), so the per-SM TMA feed
+// per k block drops from A 8K + B 2 x 16K to A 8K + B 2 x 8K at BN = 256 (the
+// feed, not the MMA rate, bounds the single-CTA kernel:
+// profiles/r01_row_gemm_components.log).  Only CTA 0 issues MMAs; CTA 1's
+// transform / epilogue warps sync locally and one thread arrives on CTA 0's
+// xf / tmem_empty barrier; MMA completion is multicast to both CTAs.  It is
+// correct but slower for 3xTF32 (each k step reads the peer's B half three
+// times across SMs), so the single-CTA kernel stays the default.
+template <bool PAIR>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBh,
                  const __grid_constant__ CUtensorMap tmBl, const __grid_constant__ CUtensorMap tmC, const KParams p) {
@@ -647,55 +703,73 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     const bool x1 = (p.flags & GEMM_TF32X1) != 0;
     const bool mask = (p.flags & GEMM_MASK) != 0;
     const int BN = p.BN;
+    const int BNH = PAIR ? BN / 2 : BN;         // rows of W^T staged by this CTA
     const uint32_t tcols = BN > 128 ? 512u : 256u;
-    const int NS = row_stages(BN), SB = row_stage_bytes(BN);
-    const int kBlo = 16384 + BN * 64;            // B_lo offset within a stage
+    const int NS = row_stages(BNH), SB = row_stage_bytes(BNH);
+    const int kBlo = 16384 + BNH * 64;           // B_lo offset within a stage
+    const uint32_t crank = PAIR ? cluster_rank() : 0u;
+    const int nunits = PAIR ? (int)(gridDim.x / 2) : (int)gridDim.x;    // tile workers (CTA pairs or CTAs)
+    const int unit = PAIR ? (int)(blockIdx.x / 2) : (int)blockIdx.x;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < NS; ++s) {
             mbar_init(full + s, 1);
-            mbar_init(xf + s, kXfWarps * 32);
+            mbar_init(xf + s, kXfWarps * 32 + (PAIR ? 1 : 0));   // PAIR: + one arrival from CTA 1
             mbar_init(empty + s, 1);
         }
         for (int s = 0; s < 2; ++s) {
             mbar_init(tmem_full + s, 1);
-            mbar_init(tmem_empty + s, 128);
+            mbar_init(tmem_empty + s, 128 + (PAIR ? 1 : 0));
             mbar_init(old_full + s, 1);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == kMmaWarp) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "r"(tcols));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        if (PAIR) {
+            asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                             smem_u32(tmem_slot)),
+                         "r"(tcols));
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+        } else {
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                             smem_u32(tmem_slot)),
+                         "r"(tcols));
+            asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+        }
     }
     tc_fence_before();
     __syncthreads();
+    if (PAIR) cluster_sync_all();                // both CTAs' barriers exist before any remote arrive
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
-    const int total_tiles = p.m_tiles * p.n_tiles;
+    const int total_tiles = (PAIR ? (p.m_tiles + 1) / 2 : p.m_tiles) * p.n_tiles;
     const int nkb = (p.K + kRowBK - 1) / kRowBK;
 
     if (warp == kTmaWarp) {
         if (lane == 0) {
-            const uint32_t bytes = (uint32_t)(BM * kRowBK * 4 + BN * kRowBK * 4 * (MGGCN_ROW_RAWB || x1 ? 1 : 2));
+            const uint32_t bytes = (uint32_t)(BM * kRowBK * 4 + BNH * kRowBK * 4 * (MGGCN_ROW_RAWB || x1 ? 1 : 2));
             int s = 0;
             uint32_t ph = 0;
-            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
-                const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
+            for (int tile = unit; tile < total_tiles; tile += nunits) {
+                const int nt = tile % p.n_tiles, mt = PAIR ? (tile / p.n_tiles) * 2 + (int)crank : tile / p.n_tiles;
+                const int nb = nt * BN + (int)crank * BNH;   // first W^T row staged here
                 for (int kb = 0; kb < nkb; ++kb) {
                     uint8_t* st = smem + kRowStage0 + s * SB;
-                    if (MGGCN_ROW_PF > 0) {   // A streams from DRAM: warm L2 ahead of the ring
+                    if (!PAIR && MGGCN_ROW_PF > 0) {   // A streams from DRAM: warm L2 ahead of the ring
                         const int kp = kb + MGGCN_ROW_PF;
                         if (kp < nkb) tma_prefetch_2d(&tmA, kp * kRowBK, mt * BM);
                         else if (tile + (int)gridDim.x < total_tiles)
                             tma_prefetch_2d(&tmA, (kp - nkb) * kRowBK, ((tile + gridDim.x) / p.n_tiles) * BM);
                     }
                     mbar_wait(empty + s, ph ^ 1);
-                    mbar_expect_tx(full + s, bytes);
-                    tma_load_2d(st, &tmA, kb * kRowBK, mt * BM, full + s);
-                    tma_load_2d(st + 16384, &tmBh, kb * kRowBK, nt * BN, full + s);
-                    if (!MGGCN_ROW_RAWB && !x1) tma_load_2d(st + kBlo, &tmBl, kb * kRowBK, nt * BN, full + s);
+                    if (MGGCN_ROW_DBG & 4) {
+                        mbar_arrive(full + s);
+                    } else {
+                        mbar_expect_tx(full + s, bytes);
+                        tma_load_2d(st, &tmA, kb * kRowBK, mt * BM, full + s);
+                        tma_load_2d(st + 16384, &tmBh, kb * kRowBK, nb, full + s);
+                        if (!MGGCN_ROW_RAWB && !x1) tma_load_2d(st + kBlo, &tmBl, kb * kRowBK, nb, full + s);
+                    }
                     if (++s == NS) { s = 0; ph ^= 1; }
                 }
             }
@@ -704,7 +778,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         const int t = threadIdx.x - kXfWarp0 * 32;
         int s = 0;
         uint32_t ph = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+        for (int tile = unit; tile < total_tiles; tile += nunits) {
             for (int kb = 0; kb < nkb; ++kb) {
                 float4* a = reinterpret_cast<float4*>(smem + kRowStage0 + s * SB);
                 mbar_wait(full + s, ph);
@@ -712,42 +786,57 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 // units, same swizzled offsets).  3xTF32: the MMA reads a raw x as hi = x &
                 // 0xFFFFE000 itself, so only lo = x - hi is written (B's lo is recomputed per
                 // tile instead of loaded: 40 -> 24 KB of TMA per k block at BN = 256).
-                const int nA = BM * 4, nT = nA + (MGGCN_ROW_RAWB ? BN * 4 : 0);
-                for (int c = t; c < nT; c += kXfWarps * 32) {
+                const int nA = BM * 4, nT = nA + (MGGCN_ROW_RAWB ? BNH * 4 : 0);
+                for (int c = t; c < ((MGGCN_ROW_DBG & 2) ? 0 : nT); c += kXfWarps * 32) {
                     const int src = c < nA ? c : 1024 + (c - nA);
-                    const int dst = src + (c < nA ? nA : BN * 4);
+                    const int dst = src + (c < nA ? nA : BNH * 4);
                     float4 v = a[src], h, l;
                     split4(v, h, l, x1);
                     if (x1) a[src] = h;    // 1xTF32: round to nearest in place
                     else a[dst] = l;
                 }
                 fence_proxy_async();
-                mbar_arrive(xf + s);
+                if (PAIR && crank != 0) {   // CTA 1: one release.cluster arrival on CTA 0's barrier
+                    asm volatile("bar.sync 2, %0;" ::"n"(kXfWarps * 32) : "memory");
+                    if (t == 0) mbar_arrive_cluster(xf + s, 0);
+                } else {
+                    mbar_arrive(xf + s);
+                }
                 if (++s == NS) { s = 0; ph ^= 1; }
             }
         }
     } else if (warp == kMmaWarp) {
-        if (lane == 0) {
+        if (lane == 0 && crank == 0) {
             const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) |
-                                   ((uint32_t)(BM >> 4) << 24);
+                                   ((uint32_t)((PAIR ? 2 * BM : BM) >> 4) << 24);
             int s = 0;
             uint32_t ph = 0, tc = 0;
-            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
+            for (int tile = unit; tile < total_tiles; tile += nunits, ++tc) {
                 const int acc = tc & 1;
                 const uint32_t aph = (tc >> 1) & 1;
-                mbar_wait(tmem_empty + acc, aph ^ 1);
+                if (PAIR) mbar_wait_cluster(tmem_empty + acc, aph ^ 1);
+                else mbar_wait(tmem_empty + acc, aph ^ 1);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
                 for (int kb = 0; kb < nkb; ++kb) {
-                    mbar_wait(xf + s, ph);
+                    if (PAIR) mbar_wait_cluster(xf + s, ph);
+                    else mbar_wait(xf + s, ph);
                     tc_fence_after();
                     const uint32_t base = smem_u32(smem + kRowStage0 + s * SB);
                     const uint64_t ah = sw64_desc(base), al = sw64_desc(base + 8192);
                     const uint64_t bh = sw64_desc(base + 16384), bl = sw64_desc(base + kBlo);
 #pragma unroll
-                    for (int kk = 0; kk < kRowBK / 8; ++kk) {
+                    for (int kk = 0; kk < ((MGGCN_ROW_DBG & 1) ? 0 : kRowBK / 8); ++kk) {
                         const uint64_t adv = (uint64_t)((kk * 8 * 4) >> 4);
-                        if (!x1) {   // small products first
+                        if (PAIR) {
+                            if (!x1) {
+                                mma_tf32_pair(d_tmem, al + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
+                                mma_tf32_pair(d_tmem, ah + adv, bl + adv, idesc, 1u);
+                                mma_tf32_pair(d_tmem, ah + adv, bh + adv, idesc, 1u);
+                            } else {
+                                mma_tf32_pair(d_tmem, ah + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
+                            }
+                        } else if (!x1) {   // small products first
                             mma_tf32(d_tmem, al + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
                             mma_tf32(d_tmem, ah + adv, bl + adv, idesc, 1u);
                             mma_tf32(d_tmem, ah + adv, bh + adv, idesc, 1u);
@@ -755,10 +844,12 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                             mma_tf32(d_tmem, ah + adv, bh + adv, idesc, (kb | kk) ? 1u : 0u);
                         }
                     }
-                    mma_commit(empty + s);
+                    if (PAIR) mma_commit_pair(empty + s);
+                    else mma_commit(empty + s);
                     if (++s == NS) { s = 0; ph ^= 1; }
                 }
-                mma_commit(tmem_full + acc);
+                if (PAIR) mma_commit_pair(tmem_full + acc);
+                else mma_commit(tmem_full + acc);
             }
         }
     } else {
@@ -767,8 +858,8 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         const bool leader = threadIdx.x == 0;
         uint32_t tc = 0, chunk_ctr = 0;
         const int nch = (BN + 31) / 32;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++tc) {
-            const int nt = tile % p.n_tiles, mt = tile / p.n_tiles;
+        for (int tile = unit; tile < total_tiles; tile += nunits, ++tc) {
+            const int nt = tile % p.n_tiles, mt = PAIR ? (tile / p.n_tiles) * 2 + (int)crank : tile / p.n_tiles;
             const int acc = tc & 1;
             const uint32_t aph = (tc >> 1) & 1;
             const int row = mt * BM + r;
@@ -822,14 +913,23 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 }
             }
             tc_fence_before();
-            mbar_arrive(tmem_empty + acc);
+            if (PAIR && crank != 0) {       // CTA 1: one arrival on CTA 0's barrier
+                epi_bar();
+                if (leader) mbar_arrive_cluster(tmem_empty + acc, 0);
+            } else {
+                mbar_arrive(tmem_empty + acc);
+            }
         }
         if (leader) bulk_wait_read<0>();
     }
     __syncthreads();
+    if (PAIR) cluster_sync_all();                // the peer's MMAs / arrivals are done
     if (warp == kMmaWarp) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
+        if (PAIR)
+            asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
+        else
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(tcols));
     }
 }
 
@@ -963,11 +1063,31 @@ cudaError_t launch_wgrad_mn(const GemmPlan& g, const KParams& kp, cudaStream_t s
 cudaError_t launch_rows(const GemmPlan& g, const KParams& kp, cudaStream_t s) {
     static bool attr_set = false;
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(gemm_rows_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kRowSmem);
+        cudaError_t e = cudaFuncSetAttribute(gemm_rows_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             kRowSmem);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(gemm_rows_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kRowSmem);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    gemm_rows_kernel<<<g.grid, kThreads, kRowSmem, s>>>(g.tmA, g.tmB, g.tmB2, g.tmC, kp);
+    if (g.variant == 2) {   // CTA pairs (cluster of 2, tcgen05 cta_group::2)
+        cudaLaunchConfig_t cfg = {};
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = 2;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.gridDim = dim3((unsigned)g.grid);
+        cfg.blockDim = dim3(kThreads);
+        cfg.dynamicSmemBytes = kRowSmem;
+        cfg.stream = s;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaError_t e = cudaLaunchKernelEx(&cfg, gemm_rows_kernel<true>, g.tmA, g.tmB, g.tmB2, g.tmC, kp);
+        count_launches(1);
+        return e != cudaSuccess ? e : cudaGetLastError();
+    }
+    gemm_rows_kernel<false><<<g.grid, kThreads, kRowSmem, s>>>(g.tmA, g.tmB, g.tmB2, g.tmC, kp);
     count_launches(1);
     return cudaGetLastError();
 }
@@ -994,13 +1114,31 @@ int gemm_plan_rows(GemmPlan& g, int64_t M, int64_t N, int64_t K, const float* A,
     g.k_chunks = 1;
     g.k_chunk_len = (K + BK - 1) / BK * BK;
     if ((ldc & 3) || (reinterpret_cast<uintptr_t>(C) & 15)) return -1;
+    // CTA pairs (cta_group::2, M = 256) when B is wide: each CTA of a pair stages half of B
+    static int pair_env = -1;
+    if (pair_env < 0) {
+        // default off: correct, but 1.5-1.8x SLOWER for 3xTF32 -- the pair's MMAs read the peer
+        // CTA's half of B three times per k step (hi, lo, hi) over the SM-to-SM path
+        // (profiles/r01_row_gemm_pair.log)
+        const char* e = getenv("MGGCN_ROW_PAIR");
+        pair_env = e ? atoi(e) : 0;
+    }
+    const bool pair = pair_env != 0 && g.BN >= 128 && g.m_tiles >= 2;
+    g.variant = pair ? 2 : 0;
+    const int bbox = pair ? g.BN / 2 : g.BN;
     int rc = encode2d_sw(&g.tmA, A, K, M, lda, 16, BM, 64);
-    if (!rc) rc = encode2d_sw(&g.tmB, Bhi, K, N, ldb, 16, g.BN, 64);
-    if (!rc) rc = encode2d_sw(&g.tmB2, Blo, K, N, ldb, 16, g.BN, 64);
+    if (!rc) rc = encode2d_sw(&g.tmB, Bhi, K, N, ldb, 16, bbox, 64);
+    if (!rc) rc = encode2d_sw(&g.tmB2, Blo, K, N, ldb, 16, bbox, 64);
     if (!rc) rc = encode2d_sw(&g.tmC, C, N, M, ldc, 32, BM, 128);   // epilogue store / old-value load
     if (rc) return rc;
-    const int total = g.m_tiles * g.n_tiles;
-    g.grid = total < num_sms() ? total : num_sms();
+    if (pair) {
+        const int total = ((g.m_tiles + 1) / 2) * g.n_tiles;      // 256-row pair tiles
+        const int pairs = num_sms() / 2;
+        g.grid = 2 * (total < pairs ? total : pairs);
+    } else {
+        const int total = g.m_tiles * g.n_tiles;
+        g.grid = total < num_sms() ? total : num_sms();
+    }
     return 0;
 }
 

@@ -191,3 +191,21 @@ def test_spmm_column_windows(win):
                        capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
     assert " passed" in r.stdout
+
+
+def test_gemm_cta_pair_variant():
+    """The opt-in CTA-pair row GEMM (MGGCN_ROW_PAIR=1: cluster of 2, tcgen05.mma.cta_group::2,
+    each CTA stages half of B) passes the same integer-exact and random GEMM cases in a
+    fresh process (shapes with >= 2 M tiles and BN >= 128 take the pair path)."""
+    import os
+    import subprocess
+    import sys
+    if os.environ.get("MGGCN_ROW_PAIR"):
+        pytest.skip("already inside a forced-variant run")
+    here = os.path.dirname(os.path.abspath(__file__))
+    env = dict(os.environ, MGGCN_ROW_PAIR="1")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", os.path.join(here, "test_gpu_kernels.py"),
+                        "-k", "gemm_integer_exact or gemm_random"], env=env, cwd=os.path.dirname(here),
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout

@@ -117,8 +117,16 @@ __device__ __forceinline__ float4 epilogue(float4 acc, const float4* out_row, in
 template <int CH>
 __host__ __device__ constexpr int unroll_for() { return CH == 1 ? 16 : CH == 2 ? MGGCN_SPMM_U2 : CH == 3 ? 5 : 4; }
 
+#ifndef MGGCN_SPMM_MINB_NARROW
+#define MGGCN_SPMM_MINB_NARROW MGGCN_SPMM_MINB
+#endif
+// narrow rows (G * CH <= 16 float4, <= 64 floats per window): short gathers, latency-bound on
+// short rows -> optionally more resident warps (fewer registers)
+template <int G, int CH>
+__host__ __device__ constexpr int minb_for() { return G * CH <= 16 ? MGGCN_SPMM_MINB_NARROW : MGGCN_SPMM_MINB; }
+
 template <int G, int CH, bool VALS>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, MGGCN_SPMM_MINB)
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, minb_for<G, CH>())
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const float4* __restrict__ B, int64_t ldb4,
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,

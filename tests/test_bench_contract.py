@@ -1,0 +1,43 @@
+"""bench.py host-side contract (CPU only): the epoch's SpMM widths and the
+L2-line model behind roofline.l2_gather, and the reference arm (the CPU oracle
+on a bounded sample) printing one JSON line with the driver's keys."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def test_spmm_widths_follow_the_order_rule():
+    import bench
+    # Reddit-shaped: every layer GeMM-first (d_l >= d_{l+1}, C10): forward + backward SpMM per layer
+    assert sorted(bench.spmm_widths([602, 256, 256, 41])) == [41, 41, 256, 256, 256, 256]
+    # Products / Proteins-shaped: SpMM-first layer 0 (forward T0 only, backward skipped, C11)
+    assert sorted(bench.spmm_widths([100, 256, 256, 47])) == [47, 47, 100, 256, 256]
+    assert sorted(bench.spmm_widths([8, 128, 128, 112])) == [8, 112, 112, 128, 128]
+
+
+@pytest.mark.parametrize("width,lines", [(256, 8), (128, 4), (41, 2), (48, 2), (100, 4), (8, 1), (602, 19)])
+def test_line_bytes(width, lines):
+    import bench
+    assert bench.line_bytes(width) == pytest.approx(128 * lines, rel=0.2)
+
+
+def test_reference_arm_json_line():
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--workload", "cora",
+                        "--steps", "2", "--warmup", "1", "--oracle-rows", "300"],
+                       capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "impl", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+              "config", "cpu_baseline", "e2e"):
+        assert k in d, k
+    assert d["impl"] == "reference" and d["higher_is_better"] is False and d["value"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]

@@ -69,23 +69,26 @@ __device__ __forceinline__ uint64_t l2_policy_last() {
     return pol;
 }
 
-__device__ __forceinline__ int ld_stream_i32(const int32_t* p) {
+// the L2 policies are created once per thread (a createpolicy per load would cost an issue slot per gather)
+__device__ __forceinline__ int ld_stream_i32(const int32_t* p, uint64_t pol) {
     int v;
 #if MGGCN_SPMM_HINT >= 1
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(l2_policy_first()));
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
 #else
+    (void)pol;
     asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
 #endif
     return v;
 }
 
-__device__ __forceinline__ float4 ld_gather(const float4* p) {
+__device__ __forceinline__ float4 ld_gather(const float4* p, uint64_t pol) {
 #if MGGCN_SPMM_HINT >= 2
     float4 v;
     asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
-                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(l2_policy_last()));
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
     return v;
 #else
+    (void)pol;
     return __ldg(p);
 #endif
 }
@@ -137,6 +140,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
     const int lane = threadIdx.x & 31;
     const int slot = lane / G, cl = lane % G;
     const uint32_t ldb = (uint32_t)ldb4;
+    const uint64_t pf = MGGCN_SPMM_HINT >= 1 ? l2_policy_first() : 0, pl = MGGCN_SPMM_HINT >= 2 ? l2_policy_last() : 0;
     int qc[CH];
 #pragma unroll
     for (int ch = 0; ch < CH; ++ch) {
@@ -153,7 +157,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
     int64_t wi = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     int4 it = wi < n_items ? __ldg(items + wi) : kNone;
     int4 itn = wi + nwarps < n_items ? __ldg(items + wi + nwarps) : kNone;
-    int cur_c = (it.y + lane < it.z) ? ld_stream_i32(col + it.y + lane) : 0;
+    int cur_c = (it.y + lane < it.z) ? ld_stream_i32(col + it.y + lane, pf) : 0;
     float cur_v = 0.f;
     if (VALS) cur_v = (it.y + lane < it.z) ? ld_stream_f32(val + it.y + lane) : 0.f;
     for (; wi < n_items; wi += nwarps) {
@@ -170,11 +174,11 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
             const float my_v = nxt_v;
             if (base + 32 < it.z) {       // prefetch the next chunk's indices
                 const int e = base + 32 + lane;
-                nxt_c = e < it.z ? ld_stream_i32(col + e) : 0;
+                nxt_c = e < it.z ? ld_stream_i32(col + e, pf) : 0;
                 if (VALS) nxt_v = e < it.z ? ld_stream_f32(val + e) : 0.f;
             } else {                      // ... or the next item's first chunk
                 const int e = itn.y + lane;
-                nxt_c = e < itn.z ? ld_stream_i32(col + e) : 0;
+                nxt_c = e < itn.z ? ld_stream_i32(col + e, pf) : 0;
                 if (VALS) nxt_v = e < itn.z ? ld_stream_f32(val + e) : 0.f;
             }
             int k0 = 0;
@@ -188,7 +192,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                     a[u] = VALS ? __shfl_sync(0xffffffffu, my_v, k) : 1.f;
                     const float4* brow = B + c * ldb;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch]);
+                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch], pl);
                 }
 #pragma unroll
                 for (int u = 0; u < U; ++u)
@@ -207,7 +211,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                     a[u] = k < cnt ? v : 0.f;
                     const float4* brow = B + c * ldb;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch]);
+                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch], pl);
                 }
 #pragma unroll
                 for (int u = 0; u < U; ++u)
@@ -217,7 +221,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
         }
         if (it.z <= it.y) {               // empty row: still fetch the next item's first chunk
             const int e = itn.y + lane;
-            nxt_c = e < itn.z ? ld_stream_i32(col + e) : 0;
+            nxt_c = e < itn.z ? ld_stream_i32(col + e, pf) : 0;
             if (VALS) nxt_v = e < itn.z ? ld_stream_f32(val + e) : 0.f;
         }
         // combine the S slots (fixed xor tree => deterministic)

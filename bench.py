@@ -234,7 +234,7 @@ def run_reference(args):
     sample = f"{R} random output rows of every SpMM/GEMM/CE op of one epoch (n = {w.n}), scaled by n/R; Adam full"
     line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": statistics.median(walls) * 1e3,
-            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f32 storage, f64 accumulate",
+            "higher_is_better": False, "scaling": "strong", "vs_baseline": None, "dtype": "f32 storage, f64 accumulate",
             "data": "synthetic", "config": workload_desc(w, 1),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}

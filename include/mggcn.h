@@ -212,6 +212,29 @@ int mggcn_prefetch(mggcn_model m, const float* X_local, int64_t ldx, const int32
 int mggcn_reset_cache(mggcn_model m);
 int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps);
 
+/* ------------------------------------------------------- captured epochs
+ * mggcn_epoch_capture — records ONE whole epoch (mggcn_forward with loss =
+ *   NULL and no logits -> mggcn_backward -> mggcn_step(lr, beta1, beta2, eps))
+ *   on the compute stream into a CUDA graph; nothing executes.  The epoch is
+ *   Fig. 1's forward / loss / backward / Adam sequence with the
+ *   same kernels, streams and events as the eager calls; the comm stream is
+ *   forked and joined inside the graph.  X_local / y_local: DEVICE pointers
+ *   (same meaning as in mggcn_forward) whose addresses the graph bakes in:
+ *   each replay reads whatever they hold then, so the caller keeps them valid
+ *   and may refill them between replays.  Only between epochs (ESTATE after
+ *   a forward/backward without step or with a prefetch pending); EINVAL for
+ *   host pointers; EUNSUPPORTED with MGGCN_F_IPC or MGGCN_F_CACHE_L0, or if
+ *   the stream cannot be captured.  A new capture replaces the old graph;
+ *   mggcn_model_free releases it.
+ * mggcn_epoch_replay — launches the captured epoch `epochs` times on the
+ *   compute stream (asynchronous).  Adam's step count advances per replay
+ *   (its bias corrections are re-set in the graph before each launch), so N
+ *   replays are bitwise the same as N eager epochs.  mggcn_get_loss reads the
+ *   last replay's loss.  ESTATE without a capture or mid-epoch. */
+int mggcn_epoch_capture(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float lr,
+                        float beta1, float beta2, float eps);
+int mggcn_epoch_replay(mggcn_model m, int32_t epochs);
+
 /* Synchronising getters / checkpoint. */
 int mggcn_get_loss(mggcn_model m, float* loss);                 /* loss of the last forward */
 int mggcn_get_grad(mggcn_model m, int32_t layer, float* WG);    /* reduced W_G of the last backward */

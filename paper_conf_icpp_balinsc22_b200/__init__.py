@@ -36,7 +36,8 @@ EXPORTS = (
     "mggcn_backward", "mggcn_step", "mggcn_get_loss", "mggcn_get_grad", "mggcn_get_adam", "mggcn_set_adam",
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
-    "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer",
+    "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
+    "mggcn_epoch_replay",
 )
 
 
@@ -91,6 +92,8 @@ def _load():
         "mggcn_kernel_launch_count": ([], ctypes.c_int64),
         "mggcn_reset_cache": ([P], ctypes.c_int),
         "mggcn_prefetch": ([P, P, i64, P], ctypes.c_int),
+        "mggcn_epoch_capture": ([P, P, i64, P, f32, f32, f32, f32], ctypes.c_int),
+        "mggcn_epoch_replay": ([P, i32], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(lib, name)
@@ -258,6 +261,14 @@ def mggcn_reset_cache(m):
 
 def mggcn_step(m, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8):
     _check(_lib.mggcn_step(m, lr, beta1, beta2, eps))
+
+
+def mggcn_epoch_capture(m, X, ldx, y, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8):
+    _check(_lib.mggcn_epoch_capture(m, _ptr(X), ldx, _ptr(y), lr, beta1, beta2, eps))
+
+
+def mggcn_epoch_replay(m, epochs=1):
+    _check(_lib.mggcn_epoch_replay(m, epochs))
 
 
 def mggcn_get_loss(m):

@@ -100,6 +100,11 @@ cudaError_t launch_sum_partials(const double* partial, int count, double* out, c
 cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* scratch, int64_t* out, cudaStream_t s);
 cudaError_t launch_adam(float* W, const float* g, float* m, float* v, int64_t count, double lr, double b1,
                         double b2, double eps, int64_t t, cudaStream_t s);
+// CUDA-graph epochs: the Adam kernel's address, and a re-set of a captured Adam node's
+// arguments (bias corrections for step t) in an instantiated graph.
+const void* adam_kernel_func();
+cudaError_t graph_set_adam(cudaGraphExec_t ex, cudaGraphNode_t node, float* W, const float* g, float* m, float* v,
+                           int64_t count, double lr, double b1, double b2, double eps, int64_t t);
 // out[i] = sum_r in[r][i] in r order (loopback "all-reduce").
 cudaError_t launch_sum_buffers(const float* const* in, int nin, float* out, int64_t count, cudaStream_t s);
 cudaError_t launch_sum_i64(const int64_t* in, int nin, int64_t* out, cudaStream_t s);

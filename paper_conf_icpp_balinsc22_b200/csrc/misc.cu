@@ -342,15 +342,38 @@ cudaError_t launch_count_labelled(const int32_t* y, int64_t n, int64_t* scratch,
     return cudaGetLastError();
 }
 
-cudaError_t launch_adam(float* W, const float* g, float* m, float* v, int64_t count, double lr, double b1, double b2,
-                        double eps, int64_t t, cudaStream_t s) {
-    const double c1 = 1.0 - std::pow(b1, (double)t), c2 = 1.0 - std::pow(b2, (double)t);
+static int adam_blocks(int64_t count) {
     int blocks = (int)((count + 255) / 256);
     if (blocks > 1184) blocks = 1184;
     if (blocks < 1) blocks = 1;
-    adam_kernel<<<blocks, 256, 0, s>>>(W, g, m, v, count, lr, b1, b2, eps, c1, c2);
+    return blocks;
+}
+
+cudaError_t launch_adam(float* W, const float* g, float* m, float* v, int64_t count, double lr, double b1, double b2,
+                        double eps, int64_t t, cudaStream_t s) {
+    const double c1 = 1.0 - std::pow(b1, (double)t), c2 = 1.0 - std::pow(b2, (double)t);
+    adam_kernel<<<adam_blocks(count), 256, 0, s>>>(W, g, m, v, count, lr, b1, b2, eps, c1, c2);
     count_launches(1);
     return cudaGetLastError();
+}
+
+// Captured epochs (mggcn_epoch_capture): Adam's bias corrections depend on the
+// step count t, a kernel argument, so every replay re-sets the Adam node's
+// arguments for its own t before the graph is launched.
+const void* adam_kernel_func() { return reinterpret_cast<const void*>(&adam_kernel); }
+
+cudaError_t graph_set_adam(cudaGraphExec_t ex, cudaGraphNode_t node, float* W, const float* g, float* m, float* v,
+                           int64_t count, double lr, double b1, double b2, double eps, int64_t t) {
+    double c1 = 1.0 - std::pow(b1, (double)t), c2 = 1.0 - std::pow(b2, (double)t);
+    void* args[] = {&W, &g, &m, &v, &count, &lr, &b1, &b2, &eps, &c1, &c2};
+    cudaKernelNodeParams p = {};
+    p.func = const_cast<void*>(adam_kernel_func());
+    p.gridDim = dim3((unsigned)adam_blocks(count));
+    p.blockDim = dim3(256);
+    p.sharedMemBytes = 0;
+    p.kernelParams = args;
+    p.extra = nullptr;
+    return cudaGraphExecKernelNodeSetParams(ex, node, &p);
 }
 
 cudaError_t launch_sum_buffers(const float* const* in, int nin, float* out, int64_t count, cudaStream_t s) {

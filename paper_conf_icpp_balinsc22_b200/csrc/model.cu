@@ -194,6 +194,14 @@ struct mggcn_model_s {
     int64_t xstage_floats = 0;
     cudaEvent_t ev_pref = nullptr, ev_xfree[2] = {nullptr, nullptr};
     int xcur = 0, pref_buf = -1;
+    // captured epoch (mggcn_epoch_capture / mggcn_epoch_replay): forward -> backward -> step
+    // as one CUDA graph; the Adam node's arguments are re-set per replay (step count t)
+    bool capturing = false;
+    cudaGraph_t eg = nullptr;
+    cudaGraphExec_t ege = nullptr;
+    cudaGraphNode_t eg_adam = nullptr;
+    int64_t eg_kernels = 0;
+    double eg_lr = 0, eg_b1 = 0, eg_b2 = 0, eg_eps = 0;
 };
 
 namespace {
@@ -247,7 +255,7 @@ struct ProfScope {
     cudaStream_t s;
     cudaEvent_t a = nullptr;
     ProfScope(mggcn_model_s* m_, int c, cudaStream_t s_) : m(m_), cls(c), s(s_) {
-        if (m->flags & MGGCN_F_PROFILE) {
+        if ((m->flags & MGGCN_F_PROFILE) && !m->capturing) {   // a captured epoch is timed as a whole
             a = prof_event(m);
             cudaEventRecord(a, s);
         }
@@ -1075,6 +1083,8 @@ static void destroy(mggcn_model_s* m) {
         cudaEventDestroy(std::get<2>(rec));
     }
     for (auto e : m->prof_pool) cudaEventDestroy(e);
+    if (m->ege) cudaGraphExecDestroy(m->ege);
+    if (m->eg) cudaGraphDestroy(m->eg);
     if (m->comm_bc) ncclCommDestroy(m->comm_bc);
     if (m->comm_pair) ncclCommDestroy(m->comm_pair);
     if (m->comm) ncclCommDestroy(m->comm);
@@ -1627,27 +1637,166 @@ extern "C" int mggcn_backward(mggcn_model m) {
     return poison(m, rc);
 }
 
+static bool bad_hyper(float lr, float beta1, float beta2, float eps) {
+    return !(lr > 0) || !(beta1 >= 0 && beta1 < 1) || !(beta2 >= 0 && beta2 < 1) || !(eps > 0);
+}
+
+static int step_impl(mggcn_model_s* m, float lr, float beta1, float beta2, float eps) {
+    RC(wait_wg(m));
+    m->t += 1;
+    ProfScope ps(m, PC_ADAM, m->cs);
+    CK(launch_adam(m->W, m->WG, m->Mom, m->Vel, m->wtotal, lr, beta1, beta2, eps, m->t, m->cs));
+    RC(refresh_weight_splits(m));
+    return MGGCN_OK;
+}
+
 extern "C" int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps) {
     MODEL_GUARD(m);
     if (m->state != ST_BWD) {
         set_error("step: needs a preceding backward");
         return MGGCN_ESTATE;
     }
-    if (!(lr > 0) || !(beta1 >= 0 && beta1 < 1) || !(beta2 >= 0 && beta2 < 1) || !(eps > 0)) {
+    if (bad_hyper(lr, beta1, beta2, eps)) {
         set_error("step: bad hyper-parameters");
         return MGGCN_EINVAL;
     }
-    auto body = [&]() -> int {
-        RC(wait_wg(m));
-        m->t += 1;
-        ProfScope ps(m, PC_ADAM, m->cs);
-        CK(launch_adam(m->W, m->WG, m->Mom, m->Vel, m->wtotal, lr, beta1, beta2, eps, m->t, m->cs));
-        RC(refresh_weight_splits(m));
-        return MGGCN_OK;
-    };
-    int rc = body();
+    int rc = step_impl(m, lr, beta1, beta2, eps);
     if (rc == MGGCN_OK) m->state = ST_READY;
     return poison(m, rc);
+}
+
+// ------------------------------------------------------- captured epochs
+// The whole epoch (forward with no host loss read -> backward -> step) is
+// captured once on the compute stream into a CUDA graph, with the comm stream
+// forked and joined through the same events as the eager path; a replay is one
+// cudaGraphLaunch, so the ~40 kernel launches of an epoch leave no host gaps.
+// The graph bakes in every pointer (X, y, the workspace) and the launch plan;
+// only Adam's step count changes between replays, and its node is re-set.
+static void drop_epoch_graph(mggcn_model_s* m) {
+    if (m->ege) cudaGraphExecDestroy(m->ege);
+    if (m->eg) cudaGraphDestroy(m->eg);
+    m->ege = nullptr;
+    m->eg = nullptr;
+    m->eg_adam = nullptr;
+    m->eg_kernels = 0;
+}
+
+static bool is_device_ptr(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+extern "C" int mggcn_epoch_capture(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float lr,
+                                   float beta1, float beta2, float eps) {
+    MODEL_GUARD(m);
+    if (!X_local || !y_local || ldx < m->d[0] || bad_hyper(lr, beta1, beta2, eps)) {
+        set_error("epoch_capture: NULL X/y, ldx < d_0 or bad hyper-parameters");
+        return MGGCN_EINVAL;
+    }
+    if (!is_device_ptr(X_local) || !is_device_ptr(y_local)) {
+        set_error("epoch_capture: X and y must be device memory (the graph bakes in their addresses)");
+        return MGGCN_EINVAL;
+    }
+    if (m->state != ST_READY || m->pref_buf >= 0) {
+        set_error("epoch_capture: only between epochs, with no prefetch pending");
+        return MGGCN_ESTATE;
+    }
+    if (m->ipc || (m->flags & MGGCN_F_CACHE_L0)) {
+        set_error("epoch_capture: not with MGGCN_F_IPC (host-side sequence numbers) or MGGCN_F_CACHE_L0 "
+                  "(first-epoch-only work)");
+        return MGGCN_EUNSUPPORTED;
+    }
+    drop_epoch_graph(m);
+    RC(poison(m, wait_wg(m)));
+    const int64_t t_saved = m->t, launches0 = mggcn_kernel_launch_count();
+    if (cudaStreamBeginCapture(m->cs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+        set_error("epoch_capture: cudaStreamBeginCapture failed on the compute stream");
+        cudaGetLastError();
+        return MGGCN_EUNSUPPORTED;
+    }
+    m->capturing = true;
+    int rc = forward_impl(m, X_local, ldx, y_local, nullptr, nullptr);
+    if (rc == MGGCN_OK && cudaEventRecord(m->ev_xfree[m->xcur], m->cs) != cudaSuccess) rc = MGGCN_ECUDA;
+    if (rc == MGGCN_OK) rc = backward_impl(m);
+    if (rc == MGGCN_OK && cudaEventRecord(m->ev_xfree[m->xcur], m->cs) != cudaSuccess) rc = MGGCN_ECUDA;
+    if (rc == MGGCN_OK) rc = step_impl(m, lr, beta1, beta2, eps);
+    cudaGraph_t g = nullptr;
+    const cudaError_t ec = cudaStreamEndCapture(m->cs, &g);
+    m->capturing = false;
+    m->t = t_saved;                 // nothing ran: the replays advance t
+    m->state = ST_READY;
+    m->need_wg_wait = false;        // the graph joins the comm stream back into the compute stream
+    count_launches((int)(launches0 - mggcn_kernel_launch_count()));
+    // events recorded during the capture became graph edges; re-record them on the
+    // (no longer capturing) compute stream so that eager calls may wait on them again
+    for (cudaEvent_t e : {m->ev_begin, m->ev_comm_end, m->ev_tmp, m->ev_wg, m->ev_comm_done, m->ev_xfree[0],
+                          m->ev_xfree[1]})
+        if (e) cudaEventRecord(e, m->cs);
+    for (auto& r : m->ranks)
+        for (int k = 0; k < 2; ++k) {
+            if (r.ev_bc[k]) cudaEventRecord(r.ev_bc[k], m->cs);
+            if (r.ev_free[k]) cudaEventRecord(r.ev_free[k], m->cs);
+        }
+    if (rc != MGGCN_OK || ec != cudaSuccess || !g) {
+        if (g) cudaGraphDestroy(g);
+        cudaGetLastError();
+        if (rc == MGGCN_OK) set_error(std::string("epoch_capture: ") + cudaGetErrorString(ec));
+        return rc == MGGCN_ENCCL ? MGGCN_ENCCL : MGGCN_EUNSUPPORTED;
+    }
+    size_t nn = 0;
+    cudaGraphGetNodes(g, nullptr, &nn);
+    std::vector<cudaGraphNode_t> nodes(nn);
+    if (nn) cudaGraphGetNodes(g, nodes.data(), &nn);
+    for (cudaGraphNode_t nd : nodes) {
+        cudaGraphNodeType ty;
+        if (cudaGraphNodeGetType(nd, &ty) != cudaSuccess || ty != cudaGraphNodeTypeKernel) continue;
+        ++m->eg_kernels;
+        cudaKernelNodeParams kp;
+        if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess && kp.func == adam_kernel_func()) m->eg_adam = nd;
+    }
+    cudaGetLastError();
+    m->eg = g;
+    if (!m->eg_adam || cudaGraphInstantiate(&m->ege, g, 0) != cudaSuccess) {
+        cudaGetLastError();
+        drop_epoch_graph(m);
+        set_error("epoch_capture: Adam node not found or cudaGraphInstantiate failed");
+        return MGGCN_EUNSUPPORTED;
+    }
+    m->eg_lr = lr;
+    m->eg_b1 = beta1;
+    m->eg_b2 = beta2;
+    m->eg_eps = eps;
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_epoch_replay(mggcn_model m, int32_t epochs) {
+    MODEL_GUARD(m);
+    if (!m->ege) {
+        set_error("epoch_replay: no captured epoch (mggcn_epoch_capture)");
+        return MGGCN_ESTATE;
+    }
+    if (m->state != ST_READY || m->pref_buf >= 0 || epochs < 1) {
+        set_error("epoch_replay: only between epochs, epochs >= 1");
+        return m->state != ST_READY || m->pref_buf >= 0 ? MGGCN_ESTATE : MGGCN_EINVAL;
+    }
+    auto body = [&]() -> int {
+        RC(wait_wg(m));
+        for (int e = 0; e < epochs; ++e) {
+            m->t += 1;
+            CK(graph_set_adam(m->ege, m->eg_adam, m->W, m->WG, m->Mom, m->Vel, m->wtotal, m->eg_lr, m->eg_b1,
+                              m->eg_b2, m->eg_eps, m->t));
+            CK(cudaGraphLaunch(m->ege, m->cs));
+            count_launches((int)m->eg_kernels);
+        }
+        // a later mggcn_prefetch refills an input buffer only after the replays
+        for (cudaEvent_t e : m->ev_xfree) CK(cudaEventRecord(e, m->cs));
+        return MGGCN_OK;
+    };
+    return poison(m, body());
 }
 
 // -------------------------------------------------------------- profiling

@@ -7,8 +7,8 @@ from __future__ import annotations
 
 import numpy as np
 
-from . import (MGGCN_F_IPC, MGGCN_F_OVERLAP, MGGCN_F_REPL2, MGGCN_F_REPLICA1, mggcn_backward, mggcn_epoch_work,
-               mggcn_forward, mggcn_get_adam, mggcn_get_grad, mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free,
+from . import (MGGCN_F_IPC, MGGCN_F_OVERLAP, MGGCN_F_REPL2, MGGCN_F_REPLICA1, mggcn_backward, mggcn_epoch_capture,
+               mggcn_epoch_replay, mggcn_epoch_work, mggcn_forward, mggcn_get_adam, mggcn_get_grad, mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free,
                mggcn_ipc_connect, mggcn_ipc_export, mggcn_load_csr, mggcn_model_create, mggcn_model_free,
                mggcn_part_free, mggcn_part_info, mggcn_partition, mggcn_prefetch, mggcn_set_adam,
                mggcn_set_weights, mggcn_step, mggcn_workspace_bytes)
@@ -136,6 +136,19 @@ class GCN:
 
     def step(self, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8):
         mggcn_step(self.m, lr, beta1, beta2, eps)
+
+    def capture_epoch(self, X_local, y_local, lr=0.01, beta1=0.9, beta2=0.999, eps=1e-8):
+        """Record one forward -> backward -> step epoch as a CUDA graph (device X/y, whose
+        addresses the graph keeps: refill them in place between replays)."""
+        torch = self.torch
+        self.cs.wait_stream(torch.cuda.current_stream(self.device))
+        self._graph_inputs = (X_local, y_local)   # keep the baked-in buffers alive
+        ldx = X_local.shape[1] if X_local.ndim == 2 else self.dims[0]
+        mggcn_epoch_capture(self.m, X_local, ldx, y_local, lr, beta1, beta2, eps)
+
+    def replay_epoch(self, epochs=1):
+        """Launch the captured epoch `epochs` times (asynchronous, on the compute stream)."""
+        mggcn_epoch_replay(self.m, epochs)
 
     def loss(self):
         return mggcn_get_loss(self.m)

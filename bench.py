@@ -55,6 +55,9 @@ def parse():
     ap.add_argument("--no-cache-l0", action="store_true",
                     help="skip the extra MGGCN_F_CACHE_L0 timing (reported under 'cache_l0', never the headline)")
     ap.add_argument("--oracle-rows", type=int, default=0, help="row sample of the oracle leg (0 = auto)")
+    ap.add_argument("--graph", action="store_true",
+                    help="N > 1: also take the headline from captured-epoch replays (NCCL collectives inside the "
+                         "graph; default for N = 1 only, since multi-GPU capture is unverified on one-GPU boxes)")
     ap.add_argument("--eager", action="store_true",
                     help="headline from eager forward/backward/step calls instead of replays of the captured "
                          "epoch (mggcn_epoch_capture); the eager loop is timed either way (profile breakdown)")
@@ -337,7 +340,7 @@ def main():
     # kernels and stream order, no per-kernel host launch gaps; the headline unless --eager.
     # The graph is captured without the profiling events, so this loop has no per-op events.
     gtime = None
-    if not args.eager and args.comm != "ipc":
+    if not args.eager and args.comm != "ipc" and (world == 1 or args.graph):
         gm.capture_epoch(Xd, yd, lr=0.01)
         gm.replay_epoch(args.warmup)
         gm.synchronize()

@@ -28,7 +28,24 @@ struct SpmmTile {
     const int32_t* col = nullptr;
     const float* val = nullptr;    // nullptr => pattern-only (value 1)
     int64_t nnz = 0, nrows = 0, ncols = 0;
+    // L2 priority classes: when set, col[e] = (cls << 24) | column, where cls
+    // is the 1/8-octave class of the column's rank by reuse count in this tile
+    // (hot_class_of); launch_spmm gathers the rows of the classes that fit its
+    // L2 budget with evict_last and the rest with evict_first.
+    bool hot_enc = false;
 };
+
+// default evict_last budget of the L2 priority classes (MGGCN_SPMM_HOT_MB overrides)
+constexpr int kHotDefaultMB = 0;
+
+// 1/8-octave class of rank r (0 = most reused column): 8*floor(log2(r+1)) + the
+// next 3 bits of r+1; monotone in r, < 200 for r < 2^24.
+inline int hot_class_of(int64_t r) {
+    const uint64_t x = (uint64_t)r + 1;
+    int e = 63 - __builtin_clzll(x);
+    const int f = e >= 3 ? (int)((x >> (e - 3)) & 7) : (int)((x << (3 - e)) & 7);
+    return 8 * e + f;
+}
 
 enum SpmmFlags : int { SPMM_ACCUM = 1, SPMM_LAST = 2, SPMM_RELU = 4 };
 

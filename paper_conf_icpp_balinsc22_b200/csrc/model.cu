@@ -98,6 +98,39 @@ void coalesce(const HostTile& t, HostTile& o) {
     }
 }
 
+// L2 priority classes of a tile's columns (SpmmTile::hot_enc): the columns are
+// ranked by reuse (entries per column, descending; ties by column id) and the
+// device copy of the index carries hot_class_of(rank) in bits 24..31.  Used
+// only for blocks whose 128-float slice exceeds the L2 (R-MAT hubs are reused
+// across the whole tile; the rest of the block streams through).
+bool want_hot_classes(const HostTile& ht) {
+    static int env = -1;
+    static int64_t l2 = 0;
+    if (env < 0) {
+        const char* e = getenv("MGGCN_SPMM_HOTCLS");
+        env = e ? atoi(e) : 0;   // opt-in: no gain on Products-shaped blocks (profiles/r01_hot_sweep.log)
+        int dev = 0, v = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&v, cudaDevAttrL2CacheSize, dev);
+        l2 = v;
+    }
+    if (env == 0 || ht.ncols > ((int64_t)1 << 24)) return false;
+    return env == 2 || (l2 > 0 && ht.ncols * 512 > l2);   // 2: always (tests)
+}
+
+std::vector<int32_t> encode_hot_classes(const HostTile& ht) {
+    std::vector<int64_t> cnt(ht.ncols, 0);
+    for (int32_t c : ht.col) ++cnt[c];
+    std::vector<int32_t> ord(ht.ncols);
+    for (int64_t c = 0; c < ht.ncols; ++c) ord[c] = (int32_t)c;
+    std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return cnt[a] > cnt[b]; });
+    std::vector<uint32_t> cls(ht.ncols);
+    for (int64_t r = 0; r < ht.ncols; ++r) cls[ord[r]] = (uint32_t)std::min(255, hot_class_of(r));
+    std::vector<int32_t> out(ht.col.size());
+    for (size_t e = 0; e < ht.col.size(); ++e) out[e] = (int32_t)((cls[ht.col[e]] << 24) | (uint32_t)ht.col[e]);
+    return out;
+}
+
 struct Rank {
     const mggcn_part_s* part = nullptr;
     int rank = 0;
@@ -349,6 +382,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                 t.items = b.take<int4>(hi.items.size());
                 t.splits = b.take<int4>(hi.splits.size());
                 t.col = b.take<int32_t>(ht.col.size());
+                t.hot_enc = want_hot_classes(ht);
                 t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
             }
         }
@@ -392,9 +426,13 @@ int upload_static(mggcn_model_s* m) {
                 if (!hi.splits.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.splits), hi.splits.data(),
                                        sizeof(int4) * hi.splits.size(), cudaMemcpyHostToDevice, m->cs));
-                if (!ht.col.empty())
-                    CK(cudaMemcpyAsync(const_cast<int32_t*>(t.col), ht.col.data(), sizeof(int32_t) * ht.col.size(),
-                                       cudaMemcpyHostToDevice, m->cs));
+                if (!ht.col.empty()) {
+                    std::vector<int32_t> enc;
+                    if (t.hot_enc) enc = encode_hot_classes(ht);
+                    CK(cudaMemcpyAsync(const_cast<int32_t*>(t.col), t.hot_enc ? enc.data() : ht.col.data(),
+                                       sizeof(int32_t) * ht.col.size(), cudaMemcpyHostToDevice, m->cs));
+                    if (t.hot_enc) CK(cudaStreamSynchronize(m->cs));   // enc is a temporary
+                }
                 if (t.val && !ht.val.empty())
                     CK(cudaMemcpyAsync(const_cast<float*>(t.val), ht.val.data(), sizeof(float) * ht.val.size(),
                                        cudaMemcpyHostToDevice, m->cs));

@@ -63,6 +63,11 @@ __device__ __forceinline__ uint64_t l2_policy_first() {
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
     return pol;
 }
+__device__ __forceinline__ uint64_t l2_policy_normal() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
 __device__ __forceinline__ uint64_t l2_policy_last() {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
@@ -91,6 +96,14 @@ __device__ __forceinline__ float4 ld_gather(const float4* p, uint64_t pol) {
     (void)pol;
     return __ldg(p);
 #endif
+}
+
+// gather with a per-load L2 policy (degree-ranked priority classes)
+__device__ __forceinline__ float4 ld_gather_pol(const float4* p, uint64_t pol) {
+    float4 v;
+    asm volatile("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
+    return v;
 }
 
 __device__ __forceinline__ float ld_stream_f32(const float* p) {
@@ -128,12 +141,15 @@ __host__ __device__ constexpr int unroll_for() { return CH == 1 ? 16 : CH == 2 ?
 template <int G, int CH>
 __host__ __device__ constexpr int minb_for() { return G * CH <= 16 ? MGGCN_SPMM_MINB_NARROW : MGGCN_SPMM_MINB; }
 
-template <int G, int CH, bool VALS>
+// HOT: the column indices carry L2 priority classes in bits 24..31 (SpmmTile::hot_enc);
+// rows of class < hot_T are gathered with evict_last, the others with evict_first,
+// so the most reused rows of a block larger than the L2 stay resident.
+template <int G, int CH, bool VALS, bool HOT>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, minb_for<G, CH>())
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const float4* __restrict__ B, int64_t ldb4,
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,
-                  const float* __restrict__ rowscale, int w4, int flags) {
+                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T) {
     constexpr int S = 32 / G;
     // U entries per slot per group; U * S <= 32 so a group fits a 32-entry chunk
     constexpr int U = unroll_for<CH>() < G ? unroll_for<CH>() : G;
@@ -141,6 +157,11 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
     const int slot = lane / G, cl = lane % G;
     const uint32_t ldb = (uint32_t)ldb4;
     const uint64_t pf = MGGCN_SPMM_HINT >= 1 ? l2_policy_first() : 0, pl = MGGCN_SPMM_HINT >= 2 ? l2_policy_last() : 0;
+    uint64_t ph = 0, pc = 0;
+    if (HOT) {
+        ph = hot_T > 0 ? l2_policy_last() : l2_policy_normal();
+        pc = hot_T > 0 ? l2_policy_first() : l2_policy_normal();
+    }
     int qc[CH];
 #pragma unroll
     for (int ch = 0; ch < CH; ++ch) {
@@ -188,11 +209,18 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     const int k = k0 + u * S + slot;
-                    const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, my_c, k);
+                    const uint32_t raw = (uint32_t)__shfl_sync(0xffffffffu, my_c, k);
                     a[u] = VALS ? __shfl_sync(0xffffffffu, my_v, k) : 1.f;
-                    const float4* brow = B + c * ldb;
+                    if (HOT) {
+                        const float4* brow = B + (raw & 0xFFFFFFu) * ldb;
+                        const uint64_t pol = (raw >> 24) < hot_T ? ph : pc;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch], pl);
+                        for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather_pol(brow + qc[ch], pol);
+                    } else {
+                        const float4* brow = B + raw * ldb;
+#pragma unroll
+                        for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch], pl);
+                    }
                 }
 #pragma unroll
                 for (int u = 0; u < U; ++u)
@@ -206,12 +234,19 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 for (int u = 0; u < U; ++u) {
                     const int k = k0 + u * S + slot;
                     const int kc = k < cnt ? k : cnt - 1;
-                    const uint32_t c = (uint32_t)__shfl_sync(0xffffffffu, my_c, kc);
+                    const uint32_t raw = (uint32_t)__shfl_sync(0xffffffffu, my_c, kc);
                     const float v = VALS ? __shfl_sync(0xffffffffu, my_v, kc) : 1.f;
                     a[u] = k < cnt ? v : 0.f;
-                    const float4* brow = B + c * ldb;
+                    if (HOT) {
+                        const float4* brow = B + (raw & 0xFFFFFFu) * ldb;
+                        const uint64_t pol = (raw >> 24) < hot_T ? ph : pc;
 #pragma unroll
-                    for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch], pl);
+                        for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather_pol(brow + qc[ch], pol);
+                    } else {
+                        const float4* brow = B + raw * ldb;
+#pragma unroll
+                        for (int ch = 0; ch < CH; ++ch) x[u][ch] = ld_gather(brow + qc[ch], pl);
+                    }
                 }
 #pragma unroll
                 for (int u = 0; u < U; ++u)
@@ -282,14 +317,14 @@ int sm_count() {
     return n;
 }
 
-template <int G, int CH, bool V>
+template <int G, int CH, bool V, bool H>
 int64_t persistent_blocks(int64_t n_items) {
     static int per_sm = 0;
     if (per_sm == 0) {
         const char* co = getenv("MGGCN_SPMM_CARVEOUT");
-        if (co) cudaFuncSetAttribute(spmm_stage_kernel<G, CH, V>, cudaFuncAttributePreferredSharedMemoryCarveout,
+        if (co) cudaFuncSetAttribute(spmm_stage_kernel<G, CH, V, H>, cudaFuncAttributePreferredSharedMemoryCarveout,
                                      atoi(co));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmm_stage_kernel<G, CH, V>, kWarpsPerBlock * 32, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spmm_stage_kernel<G, CH, V, H>, kWarpsPerBlock * 32, 0);
         if (per_sm <= 0) per_sm = 1;
     }
     const int64_t need = (n_items + kWarpsPerBlock - 1) / kWarpsPerBlock;
@@ -297,16 +332,24 @@ int64_t persistent_blocks(int64_t n_items) {
     return need < cap ? need : cap;
 }
 
+template <int G, int CH, bool V, bool H>
+void launch_one(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, int64_t ldo4, float4* partial,
+                int64_t ldp4, const float* rowscale, int w4, int flags, uint32_t hot_T, cudaStream_t s) {
+    const int64_t blocks = persistent_blocks<G, CH, V, H>(t.n_items);
+    spmm_stage_kernel<G, CH, V, H><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
+        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T);
+}
+
 template <int G, int CH>
 cudaError_t launch_gc(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, int64_t ldo4, float4* partial,
-                      int64_t ldp4, const float* rowscale, int w4, int flags, cudaStream_t s) {
-    const int64_t blocks = t.val ? persistent_blocks<G, CH, true>(t.n_items) : persistent_blocks<G, CH, false>(t.n_items);
-    if (t.val)
-        spmm_stage_kernel<G, CH, true><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
-            t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags);
-    else
-        spmm_stage_kernel<G, CH, false><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
-            t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags);
+                      int64_t ldp4, const float* rowscale, int w4, int flags, uint32_t hot_T, cudaStream_t s) {
+    if (t.val) {
+        if (t.hot_enc) launch_one<G, CH, true, true>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, s);
+        else launch_one<G, CH, true, false>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, s);
+    } else {
+        if (t.hot_enc) launch_one<G, CH, false, true>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, s);
+        else launch_one<G, CH, false, false>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, s);
+    }
     count_launches(1);
     return cudaGetLastError();
 }
@@ -318,7 +361,7 @@ cudaError_t launch_gc(const SpmmTile& t, const float4* B, int64_t ldb4, float4* 
     X(4, 3) X(8, 3) X(16, 3) X(32, 3) X(8, 4) X(16, 4) X(32, 4)
 
 cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, int64_t ldo4,
-                        float4* partial, int64_t ldp4, const float* rowscale, int flags, cudaStream_t s) {
+                        float4* partial, int64_t ldp4, const float* rowscale, int flags, uint32_t hot_T, cudaStream_t s) {
     int bg = 0, bc = 0;
     double best = 1e9;
 #define MGGCN_PICK(g, c)                                                         \
@@ -337,7 +380,7 @@ cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4
         if (fg > 0 && fg * fc >= w4) { bg = fg; bc = fc; }
     }
 #define MGGCN_CALL(g, c) \
-    if (bg == g && bc == c) return launch_gc<g, c>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, s);
+    if (bg == g && bc == c) return launch_gc<g, c>(t, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, s);
     MGGCN_SPMM_SHAPES(MGGCN_CALL)
 #undef MGGCN_CALL
     return cudaErrorInvalidValue;
@@ -369,16 +412,43 @@ cudaError_t launch_spmm(const SpmmTile& t, const float* B, int64_t ldb, float* o
         const int64_t full = t.ncols * (int64_t)width * 4, w128 = t.ncols * 128 * 4;
         win = (width > 128 && 2 * full > (int64_t)l2_bytes && w128 <= (int64_t)l2_bytes) ? 128 : 512;
     }
+    // L2 priority classes (tiles with hot_enc): when the gathered window does not
+    // fit the L2, the rows of the most reused columns, up to hot_bytes of them,
+    // are gathered with evict_last and the rest with evict_first (0 = normal).
+    static int64_t hot_bytes = -1;
+    static bool hot_force = false;   // MGGCN_SPMM_HOTCLS=2 (tests): classes even for blocks that fit
+    if (hot_bytes < 0) {
+        const char* hc = getenv("MGGCN_SPMM_HOTCLS");
+        hot_force = hc && atoi(hc) == 2;
+        const char* e = getenv("MGGCN_SPMM_HOT_MB");
+        hot_bytes = (int64_t)((e ? atof(e) : (double)kHotDefaultMB) * 1048576.0);
+        if (const char* pm = getenv("MGGCN_L2_PERSIST_MB")) {   // experiment hook: persisting set-aside
+            int dev = 0, mx = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev);
+            size_t want = (size_t)(atof(pm) * 1048576.0);
+            if (want > (size_t)mx) want = (size_t)mx;
+            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
+            size_t got = 0;
+            cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize);
+            fprintf(stderr, "[mggcn] persisting L2 set-aside %zu B (max %d B)\n", got, mx);
+        }
+    }
     for (int c0 = 0; c0 < width; c0 += win) {
         const int w = width - c0 < win ? width - c0 : win;
         const int w4 = (w + 3) / 4;
+        uint32_t hot_T = 0;
+        if (t.hot_enc && hot_bytes > 0 && (hot_force || t.ncols * (int64_t)w4 * 16 > (int64_t)l2_bytes)) {
+            const int64_t H = hot_bytes / ((int64_t)w4 * 16);
+            hot_T = (uint32_t)hot_class_of(H < t.ncols ? H : t.ncols);
+        }
         const float4* Bw = reinterpret_cast<const float4*>(B + c0);
         float4* Ow = reinterpret_cast<float4*>(out + c0);
         float4* Pw = reinterpret_cast<float4*>(partial);
         const int64_t ldb4 = ldb / 4, ldo4 = ldo / 4, ldp4 = w4;
         cudaError_t e;
         if (t.n_items > 0) {
-            e = dispatch_gc(w4, t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, flags, s);
+            e = dispatch_gc(w4, t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, flags, hot_T, s);
             if (e != cudaSuccess) return e;
         }
         if (t.n_splits > 0) {

@@ -193,6 +193,26 @@ def test_spmm_column_windows(win):
     assert " passed" in r.stdout
 
 
+@pytest.mark.parametrize("hot_mb", ["0", "0.25", "64"])
+def test_spmm_hot_classes(hot_mb):
+    """L2 priority classes (column indices carry the reuse-rank class in bits 24..31,
+    rows of the hottest classes gathered evict_last): forced on for every tile
+    (MGGCN_SPMM_HOTCLS=2) with an evict_last budget of none, a few hub rows, or all
+    rows, the R-MAT hub and integer-exact cases match the oracle in a fresh process."""
+    import os
+    import subprocess
+    import sys
+    if os.environ.get("MGGCN_SPMM_HOTCLS"):
+        pytest.skip("already inside a forced-class run")
+    here = os.path.dirname(os.path.abspath(__file__))
+    env = dict(os.environ, MGGCN_SPMM_HOTCLS="2", MGGCN_SPMM_HOT_MB=hot_mb)
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", os.path.join(here, "test_gpu_kernels.py"),
+                        "-k", "rmat_hubs or exactness_graph or weighted_directed or power_law"], env=env,
+                       cwd=os.path.dirname(here), capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout
+
+
 def test_gemm_cta_pair_variant():
     """The opt-in CTA-pair row GEMM (MGGCN_ROW_PAIR=1: cluster of 2, tcgen05.mma.cta_group::2,
     each CTA stages half of B) passes the same integer-exact and random GEMM cases in a

@@ -152,6 +152,9 @@ int mggcn_part_inv_deg(mggcn_part part, float* inv_deg);
  * workspace: device memory, caller-owned, >= mggcn_workspace_bytes, 256-B
  * aligned; it must outlive the model.  compute_stream / comm_stream:
  * cudaStream_t values (streams 0 and 1 of P:929-933); 0 = legacy default.
+ * With NCCL (P > 1) and MGGCN_F_OVERLAP the SpMM launches oversubscribed grids
+ * whose blocks retire throughout the launch, so NCCL's kernels can take SMs
+ * mid-stage: give comm_stream the higher priority (cudaStreamCreateWithPriority).
  * EUNSUPPORTED: an SpMM-first layer (d_l < d_{l+1}) at l > 0. */
 int mggcn_workspace_bytes(const mggcn_part* parts, int32_t nlocal, int32_t L, const int32_t* dims, uint32_t flags,
                           size_t* bytes);

@@ -47,7 +47,12 @@ inline int hot_class_of(int64_t r) {
     return 8 * e + f;
 }
 
-enum SpmmFlags : int { SPMM_ACCUM = 1, SPMM_LAST = 2, SPMM_RELU = 4 };
+// SPMM_YIELD (host-side only): oversubscribe the grid (kYieldBlocks x the resident
+// blocks) so blocks retire throughout the launch and a collective kernel on a
+// higher-priority stream (NCCL broadcast / all-reduce) gets SMs within a few
+// microseconds instead of waiting for a persistent grid to drain.
+enum SpmmFlags : int { SPMM_ACCUM = 1, SPMM_LAST = 2, SPMM_RELU = 4, SPMM_YIELD = 8 };
+constexpr int kYieldBlocks = 4;
 
 // width: columns to compute (multiple of 4, <= ldb, <= ldo); B and out 16-B aligned.
 // rowscale (nullable): multiplies the finished row on the LAST stage.

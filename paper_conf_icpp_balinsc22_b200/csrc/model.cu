@@ -645,6 +645,8 @@ int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const flo
     const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
     float* out = job.dst(m, r, job.ctx);
     ProfScope ps(m, PC_SPMM, m->cs);
+    // NCCL collectives run as kernels on the comm stream: let them in while the SpMM runs
+    if (m->comm && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
     CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
                    (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
     return MGGCN_OK;

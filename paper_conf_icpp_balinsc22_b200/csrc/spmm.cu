@@ -318,7 +318,7 @@ int sm_count() {
 }
 
 template <int G, int CH, bool V, bool H>
-int64_t persistent_blocks(int64_t n_items) {
+int64_t persistent_blocks(int64_t n_items, int over) {
     static int per_sm = 0;
     if (per_sm == 0) {
         const char* co = getenv("MGGCN_SPMM_CARVEOUT");
@@ -328,14 +328,23 @@ int64_t persistent_blocks(int64_t n_items) {
         if (per_sm <= 0) per_sm = 1;
     }
     const int64_t need = (n_items + kWarpsPerBlock - 1) / kWarpsPerBlock;
-    const int64_t cap = (int64_t)per_sm * sm_count();
+    const int64_t cap = (int64_t)per_sm * sm_count() * over;
     return need < cap ? need : cap;
 }
 
 template <int G, int CH, bool V, bool H>
 void launch_one(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, int64_t ldo4, float4* partial,
                 int64_t ldp4, const float* rowscale, int w4, int flags, uint32_t hot_T, cudaStream_t s) {
-    const int64_t blocks = persistent_blocks<G, CH, V, H>(t.n_items);
+    // SPMM_YIELD: blocks retire throughout the launch (see kernels.cuh); MGGCN_SPMM_YIELD=k
+    // overrides the factor (and with k > 1 applies it to every launch, for measurement)
+    static int yenv = -1;
+    if (yenv < 0) {
+        const char* e = getenv("MGGCN_SPMM_YIELD");
+        yenv = e ? atoi(e) : 0;
+        if (yenv < 0) yenv = 0;
+    }
+    const int over = yenv > 1 ? yenv : ((flags & SPMM_YIELD) ? (yenv == 1 ? 1 : kYieldBlocks) : 1);
+    const int64_t blocks = persistent_blocks<G, CH, V, H>(t.n_items, over);
     spmm_stage_kernel<G, CH, V, H><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
         t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T);
 }

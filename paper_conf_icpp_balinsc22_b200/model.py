@@ -65,7 +65,8 @@ class GCN:
         self.ws_bytes = mggcn_workspace_bytes(self.parts, self.dims, flags)
         self.workspace = torch.empty(self.ws_bytes, dtype=torch.uint8, device=self.device)
         self.cs = torch.cuda.Stream(device=self.device)
-        self.ms = torch.cuda.Stream(device=self.device)
+        # the comm stream outranks compute: NCCL's kernels take SMs as the SpMM's blocks retire (SPMM_YIELD)
+        self.ms = torch.cuda.Stream(device=self.device, priority=-1)
         self.m = mggcn_model_create(self.parts, self.dims, flags, nccl_id, self.workspace.data_ptr(), self.ws_bytes,
                                     self.cs.cuda_stream, self.ms.cuda_stream)
         if self.comm == "ipc":

@@ -57,7 +57,11 @@ enum {
     MGGCN_F_RELU_LAST = 2u,   /* ReLU on the last layer too (literal Eq. 4, reading C4) */
     MGGCN_F_TF32X1 = 4u,      /* 1xTF32 GEMMs (faster, ~1e-3 rel. error); default is
                                  3xTF32 (hi/lo split, ~fp32 accuracy)                  */
-    MGGCN_F_NO_BCAST = 16u,   /* TIMING ONLY: skip broadcasts; results invalid         */
+    MGGCN_F_NO_BCAST = 16u,   /* TIMING ONLY: skip broadcasts; results invalid.  With
+                                 P > 1, nlocal = 1, nccl_id128 = NULL and no IPC it is
+                                 the SOLO mode: one rank of a P-way run alone, every
+                                 collective skipped (per-rank compute time of a
+                                 partition too large for loopback). */
     MGGCN_F_PROFILE = 32u,    /* record per-op CUDA events (see mggcn_get_profile)     */
     MGGCN_F_NO_COALESCE = 64u,/* keep duplicate entries as separate gathers (default:
                                  merged on the device copy, value = multiplicity)       */

@@ -219,6 +219,10 @@ struct mggcn_model_s {
     void* ipc_alloc = nullptr;
     size_t ipc_alloc_off = 0;
     bool ipc = false, ipc_connected = false;
+    // SOLO timing mode (MGGCN_F_NO_BCAST, P > 1, nlocal = 1, no NCCL id, no IPC): one rank of a
+    // P-way run on its own, every collective skipped; per-rank compute time of a partition
+    // too large for loopback (Papers-shaped at P = 8).  Results are invalid by construction.
+    bool solo = false;
     size_t ws_bytes = 0;             // planned workspace bytes
     size_t sym_bytes = 0;            // symmetric region [0, sym_bytes) (IPC peers must agree)
     uint32_t spmm_seq = 0, wg_seq = 0, sc_seq = 0;
@@ -646,7 +650,7 @@ int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const flo
     float* out = job.dst(m, r, job.ctx);
     ProfScope ps(m, PC_SPMM, m->cs);
     // NCCL collectives run as kernels on the comm stream: let them in while the SpMM runs
-    if (m->comm && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
+    if ((m->comm || m->solo) && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
     CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
                    (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
     return MGGCN_OK;
@@ -721,7 +725,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
         const int rq = q % c;                            // the replica group that needs block q
         {
             ProfScope ps(m, PC_BCAST, m->ms);
-            if (m->comm) {
+            if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
                 Rank& r = m->ranks[0];
                 if (r.rep == rq) {
                     const size_t count = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width;
@@ -812,7 +816,7 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
         // ---- broadcast of block q (comm stream)
         {
             ProfScope ps(m, PC_BCAST, m->ms);
-            if (m->comm) {
+            if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
                 Rank& r = m->ranks[0];
                 const size_t count = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width;
                 if (q == r.rank) {
@@ -1168,8 +1172,10 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
         delete m;
         return MGGCN_EUNSUPPORTED;
     }
-    if (m->P > 1 && nlocal == 1 && !nccl_id128 && !m->ipc) {
-        set_error("model_create: P > 1 with nlocal = 1 needs an NCCL unique id (or MGGCN_F_IPC)");
+    m->solo = m->P > 1 && nlocal == 1 && !nccl_id128 && !m->ipc && (flags & MGGCN_F_NO_BCAST) && m->c == 1;
+    if (m->P > 1 && nlocal == 1 && !nccl_id128 && !m->ipc && !m->solo) {
+        set_error("model_create: P > 1 with nlocal = 1 needs an NCCL unique id (or MGGCN_F_IPC, or the "
+                  "MGGCN_F_NO_BCAST solo timing mode)");
         delete m;
         return MGGCN_EINVAL;
     }
@@ -1212,7 +1218,7 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
     if (rc != MGGCN_OK) return fail(rc);
     rc = plan_gemms(m);
     if (rc != MGGCN_OK) return fail(rc);
-    if (m->P > 1 && nlocal == 1 && !m->ipc) {
+    if (m->P > 1 && nlocal == 1 && !m->ipc && !m->solo) {
         ncclUniqueId id;
         std::memcpy(&id, nccl_id128, 128);
         ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;

@@ -341,3 +341,47 @@ def test_padded_host_inputs_with_nan_padding(mg, dims):
         gm.close()
         assert np.isfinite(lib["logits"]).all()
         compare(lib, ref, dims)
+
+
+@pytest.mark.parametrize("dims", [(24, 16, 5), (8, 32, 32, 6)])
+def test_solo_timing_mode_on_disconnected_halves(mg, dims):
+    """SOLO timing mode (MGGCN_F_NO_BCAST, P = 2, nlocal = 1, no NCCL id): one rank of a 2-way run
+    alone, every collective skipped.  On a graph made of two disconnected copies of an R-MAT
+    graph with the identity permutation, the off-diagonal tiles are empty, so the skipped
+    broadcasts and reductions carry nothing and rank r's epoch is exactly the oracle epoch of
+    component r (its own |T|, its own W_G).  Without NO_BCAST the same call is EINVAL."""
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    n0 = 700
+    rp0, col0 = gen.rmat_csr(n0, 12000, 31)
+    rp = np.concatenate([rp0, rp0[1:] + rp0[-1]]).astype(np.int64)
+    col = np.concatenate([col0, col0 + n0]).astype(np.int32)
+    n = 2 * n0
+    X = gen.features(n, dims[0], 32)
+    y = gen.labels(n, dims[-1], 33)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 34 + l) for l in range(len(dims) - 1)]
+    flags = mg.MGGCN_F_OVERLAP | mg.MGGCN_F_NO_BCAST
+    for rank in (0, 1):
+        gm = GCN(n, rp, col, None, dims, P=2, rank=rank, perm_seed=0, flags=flags)
+        assert gm.rows == n0 and gm.row0 == rank * n0
+        gm.set_weights(Ws)
+        sl = slice(rank * n0, (rank + 1) * n0)
+        logits = torch.empty((n0, dims[-1]), dtype=torch.float32, device="cuda")
+        loss = gm.forward(torch.from_numpy(X[sl].copy()).cuda(), torch.from_numpy(y[sl].copy()).cuda(),
+                          want_loss=True, logits=logits)
+        gm.backward()
+        WG = gm.grads()
+        gm.step(lr=0.01)
+        W1 = gm.get_weights()
+        gm.close()
+        ref = oracle.epoch(oracle.permute_graph(n0, rp0, col0, None, seed=0), X[sl], y[sl], Ws)
+        assert rel(logits.cpu().numpy(), ref.logits) < REL_TOL
+        assert abs(loss - ref.loss) / abs(ref.loss) < REL_TOL
+        for a, b in zip(WG, ref.WG):
+            assert rel(a, b) < REL_TOL
+        for l in range(len(Ws)):
+            g = ref.WG[l]
+            mask = np.abs(g) > 1e-3 * np.abs(g).max()
+            np.testing.assert_allclose(W1[l][mask], ref.W[l][mask], rtol=0, atol=1e-5)
+    with pytest.raises(mg.MggcnError) as e:
+        GCN(n, rp, col, None, dims, P=2, rank=0, perm_seed=0, flags=mg.MGGCN_F_OVERLAP)
+    assert e.value.code == mg.MGGCN_EINVAL

@@ -51,6 +51,7 @@ def parse():
                          "ranks that split the broadcast stages and sum their partials; N must be a multiple of 4")
     ap.add_argument("--tf32x1", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-exposed", action="store_true", help="skip the N > 1 NO_BCAST exposed-comm ablation")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cache-l0", action="store_true",
                     help="skip the extra MGGCN_F_CACHE_L0 timing (reported under 'cache_l0', never the headline)")
@@ -436,6 +437,44 @@ def main():
                             "W_G0 = T0^T Z_G0 (exact by associativity); removes both layer-0 SpMMs per epoch. "
                             "Opt-in; not the headline value."}
         gm = gc
+
+    # ---- N > 1: exposed communication by ablation (SURVEY §8(d) "How to time it"): the same eager
+    # epochs with MGGCN_F_NO_BCAST (timing only: broadcasts skipped, results invalid; the W_G and
+    # loss all-reduces still run) give the compute-only time T_c; exposed = (T - T_c) / T.
+    exposed = None
+    if world > 1 and not args.no_exposed:
+        Ws_now = gm.get_weights()
+        gm.close()
+        del gm
+        torch.cuda.empty_cache()
+        gn = GCN(w.n, rp, col, None, w.dims, P=P, rank=rank, perm_seed=w.perm_seed,
+                 flags=flags | mg.MGGCN_F_NO_BCAST, graph=graph, replicas=args.replicas, **comm_kw())
+        gn.set_weights(Ws_now)
+        for _ in range(args.warmup):
+            gn.forward(Xd, yd, want_loss=False)
+            gn.backward()
+            gn.step(lr=0.01)
+        gn.synchronize()
+        dist.barrier()
+        torch.cuda.synchronize()
+        n0, n1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n0.record(gn.cs)
+        for _ in range(args.steps):
+            gn.forward(Xd, yd, want_loss=False)
+            gn.backward()
+            gn.step(lr=0.01)
+        n1.record(gn.cs)
+        n1.synchronize()
+        gn.synchronize()
+        dist.barrier()
+        t_c = max_over_ranks(dist, n0.elapsed_time(n1) / args.steps)
+        exposed = {"compute_only_ms": t_c, "eager_ms": ms_eager,
+                   "frac": max(0.0, (ms_eager - t_c) / ms_eager) if ms_eager > 0 else None,
+                   "bcast_bytes_per_rank_per_epoch": work["bcast_bytes"],
+                   "nvlink_bound_ms": work["bcast_bytes"] / 900e9 * 1e3,
+                   "how": "(eager epoch ms - the same epochs with MGGCN_F_NO_BCAST) / eager epoch ms, max over ranks; "
+                          "target < 0.15 (north_star)"}
+        gm = gn
     mg.mggcn_graph_free(graph)
 
     if rank != 0:
@@ -500,6 +539,7 @@ def main():
                  "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps},
         "loss_after": loss_now,
         "cache_l0": cache_l0,
+        "exposed_comm": exposed,
         "setup_s": {"generate": t_gen, "load_csr+partition+upload": t_setup},
     }
     # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1 only)

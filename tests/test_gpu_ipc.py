@@ -81,3 +81,26 @@ def test_ipc_two_ranks_vs_oracle(tmp_path, reference, mode):
     # lr * sign(g) of near-zero gradients legitimately differs, so only its loss is compared
     for l in range(L):
         assert rel(res[0][f"WG0_{l}"], r1.WG[l]) < REL_TOL, l
+
+
+def test_bench_two_ranks_ipc_exposed_comm():
+    """bench.py's multi-process path end to end (torchrun, 2 ranks, IPC backend; both ranks on
+    this GPU, so the times are time-sliced, not scaling numbers): one JSON line from rank 0 with
+    n_gpus = 2, the NO_BCAST exposed-communication ablation and a finite loss."""
+    import json
+    ROOT = os.path.dirname(HERE)
+    port = free_port()
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES=os.environ.get("CUDA_VISIBLE_DEVICES", "0"))
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
+                        "--gpus", "2", "--comm", "ipc", "--workload", "cora", "--steps", "3", "--warmup", "3",
+                        "--no-e2e", "--no-cpu-baseline", "--no-cache-l0"],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and np.isfinite(d["loss_after"])
+    ex = d["exposed_comm"]
+    assert ex is not None and ex["compute_only_ms"] > 0 and 0.0 <= ex["frac"] <= 1.0
+    assert ex["bcast_bytes_per_rank_per_epoch"] > 0

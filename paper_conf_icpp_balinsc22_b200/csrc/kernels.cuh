@@ -22,6 +22,7 @@ constexpr int kSplit = 2048;
 struct SpmmTile {
     const int4* items = nullptr;   // {row, beg, end, slot}
     int64_t n_items = 0;
+    int64_t n_items_nz = 0;        // items[0, n_items_nz) are hub segments and non-empty rows, the rest empty rows
     const int4* splits = nullptr;  // {row, first_slot, nslots, 0}
     int64_t n_splits = 0;
     int64_t n_slots = 0;

@@ -43,6 +43,7 @@ struct Bump {
 struct HostItems {
     std::vector<int4> items, splits;
     int64_t nslots = 0;
+    int64_t n_nonempty = 0;   // items[0, n_nonempty): hub segments and non-empty rows; then empty rows
 };
 
 // Work items of one tile: hub rows (> kSplit entries) are cut into segments
@@ -64,10 +65,15 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
             h.nslots += nseg;
         }
     }
+    // Empty rows go last: an accumulating middle stage skips them (adding an empty row's zero
+    // sum is a no-op), which saves their output read-modify-write (SpmmTile::n_items_nz).
     for (int32_t r : order) {
         const int64_t len = rp[r + 1] - rp[r];
-        if (len <= kSplit) h.items.push_back(make_int4(r, rp[r], rp[r + 1], -1));
+        if (len > 0 && len <= kSplit) h.items.push_back(make_int4(r, rp[r], rp[r + 1], -1));
     }
+    h.n_nonempty = (int64_t)h.items.size();
+    for (int32_t r : order)
+        if (rp[r + 1] == rp[r]) h.items.push_back(make_int4(r, rp[r], rp[r + 1], -1));
 }
 
 // Duplicate entries (multi-edges, reading C19) are adjacent within a row
@@ -381,6 +387,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                 t.ncols = ht.ncols;
                 t.nnz = ht.rowptr.back();
                 t.n_items = (int64_t)hi.items.size();
+                t.n_items_nz = hi.n_nonempty;
                 t.n_splits = (int64_t)hi.splits.size();
                 t.n_slots = hi.nslots;
                 t.items = b.take<int4>(hi.items.size());

@@ -397,9 +397,14 @@ cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4
 
 }  // namespace
 
-cudaError_t launch_spmm(const SpmmTile& t, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
+cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
                         const float* rowscale, int width, int flags, cudaStream_t s) {
-    if (t.nrows == 0) return cudaSuccess;
+    if (tile.nrows == 0) return cudaSuccess;
+    // a middle stage (accumulating, not the last) skips the tile's empty rows: their sum is
+    // zero, so their output read-modify-write is a no-op (the first stage writes every row,
+    // the last applies the row scale / ReLU to every row)
+    SpmmTile t = tile;
+    if ((flags & SPMM_ACCUM) && !(flags & SPMM_LAST)) t.n_items = t.n_items_nz;
     // Column windows of at most `win` floats.  The gathers are bound by the
     // SMs' L2 line rate; when the gathered block B_j is larger
     // than half the L2, a 128-float window that fits it (n_j * 512 B <= L2) keeps the

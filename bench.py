@@ -72,6 +72,29 @@ def workload_desc(w, P):
             "l2": "no flush: every epoch streams inputs larger than L2 (features, CSR, activations)"}
 
 
+def graph_stats(n, rp, col, perm):
+    """Realised power-law stress of the synthetic graph: degree max / mean, and the
+    spread of non-zeros over the P x P tiles of the permuted 1D partition (max / mean) at P = 2, 4, 8."""
+    deg = np.diff(rp)
+    out = {"deg_max": int(deg.max()), "deg_mean": float(deg.mean()),
+           "deg_max_over_mean": float(deg.max() / max(deg.mean(), 1e-30)), "tile_nnz_max_over_mean": {}}
+    pu = np.repeat(perm, deg)               # new id of each entry's row
+    pv = perm[col]                          # new id of each entry's column
+    for P in (2, 4, 8):
+        if n < P:
+            continue
+        bu = (pu * P) // n                  # block of new id x: largest i with floor(i n / P) <= x
+        bv = (pv * P) // n
+        # p(i) = floor(i n / P): x is in block i iff p(i) <= x < p(i+1); (x P) // n can be one low
+        # when i n / P is fractional, so correct it against the exact boundaries
+        bnd = (np.arange(P + 1, dtype=np.int64) * n) // P
+        bu = np.where(pu >= bnd[np.minimum(bu + 1, P)], bu + 1, bu)
+        bv = np.where(pv >= bnd[np.minimum(bv + 1, P)], bv + 1, bv)
+        cnt = np.bincount(bu * P + bv, minlength=P * P)
+        out["tile_nnz_max_over_mean"][P] = float(cnt.max() / max(cnt.mean(), 1e-30))
+    return out
+
+
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
     FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
@@ -476,6 +499,7 @@ def main():
                           "target < 0.15 (north_star)"}
         gm = gn
     mg.mggcn_graph_free(graph)
+    gstats = graph_stats(w.n, rp, col, np.asarray(gm.perm, dtype=np.int64)) if rank == 0 else None
 
     if rank != 0:
         gm.close()
@@ -540,6 +564,7 @@ def main():
         "loss_after": loss_now,
         "cache_l0": cache_l0,
         "exposed_comm": exposed,
+        "graph_stats": gstats,
         "setup_s": {"generate": t_gen, "load_csr+partition+upload": t_setup},
     }
     # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1 only)

@@ -41,3 +41,24 @@ def test_reference_arm_json_line():
     assert d["impl"] == "reference" and d["higher_is_better"] is False and d["value"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+
+
+def test_graph_stats_tile_spread_matches_brute_force():
+    """bench.graph_stats: the P x P tile histogram of the permuted partition p(i) = floor(i n / P)
+    equals a brute-force assignment by searching the partition boundaries."""
+    import numpy as np
+    import bench
+    import gen
+    n = 1003
+    rp, col = gen.rmat_csr(n, 20000, 7)
+    perm = np.random.default_rng(1).permutation(n).astype(np.int64)
+    st = bench.graph_stats(n, rp, col, perm)
+    deg = np.diff(rp)
+    assert st["deg_max"] == deg.max() and abs(st["deg_mean"] - deg.mean()) < 1e-12
+    pu, pv = np.repeat(perm, deg), perm[col]
+    for P in (2, 4, 8):
+        bnd = (np.arange(P + 1) * n) // P
+        bu = np.searchsorted(bnd, pu, side="right") - 1
+        bv = np.searchsorted(bnd, pv, side="right") - 1
+        c = np.bincount(bu * P + bv, minlength=P * P)
+        assert abs(st["tile_nnz_max_over_mean"][P] - c.max() / c.mean()) < 1e-12

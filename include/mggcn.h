@@ -290,6 +290,13 @@ int mggcn_debug_gemm(int32_t op, int64_t M, int64_t N, int64_t K, const float* A
  * (Eq. 8 / 21), pre-scaled row-wise by inv_deg when layer l is GeMM-first (its
  * backward SpMM then runs on the pattern, reading C20).  EINVAL: bad layer/ld. */
 int mggcn_debug_layer(mggcn_model m, int32_t layer, float* dst, int64_t ld);
+/* mggcn_debug_comm_delay: delay injection for the stage/overlap rule.
+ * With max_us > 0, every later broadcast (all backends) and every SpMM stage is
+ * preceded by a spin kernel of a pseudo-random 0..max_us microseconds on the
+ * comm or the compute stream (splitmix64 of seed and a counter), so the two
+ * streams interleave differently from run to run; results must not change.
+ * max_us = 0 turns it off.  EINVAL: max_us outside [0, 10000]. */
+int mggcn_debug_comm_delay(mggcn_model m, uint64_t seed, int32_t max_us);
 
 #ifdef __cplusplus
 }

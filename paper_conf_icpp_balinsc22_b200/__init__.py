@@ -37,7 +37,7 @@ EXPORTS = (
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
     "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
-    "mggcn_epoch_replay",
+    "mggcn_epoch_replay", "mggcn_debug_comm_delay",
 )
 
 
@@ -88,6 +88,7 @@ def _load():
         "mggcn_model_free": ([P], None),
         "mggcn_debug_spmm": ([P, i32, P, i64, i32, P, i64], ctypes.c_int),
         "mggcn_debug_layer": ([P, i32, P, i64], ctypes.c_int),
+        "mggcn_debug_comm_delay": ([P, ctypes.c_uint64, i32], ctypes.c_int),
         "mggcn_debug_gemm": ([i32, i64, i64, i64, P, i64, P, i64, P, i64, u32, up], ctypes.c_int),
         "mggcn_kernel_launch_count": ([], ctypes.c_int64),
         "mggcn_reset_cache": ([P], ctypes.c_int),
@@ -328,6 +329,10 @@ def mggcn_model_free(m):
 
 def mggcn_debug_spmm(m, direction, B, ldb, width, out, ldo):
     _check(_lib.mggcn_debug_spmm(m, direction, _ptr(B), ldb, width, _ptr(out), ldo))
+
+
+def mggcn_debug_comm_delay(m, seed, max_us):
+    _check(_lib.mggcn_debug_comm_delay(m, seed, max_us))
 
 
 def mggcn_debug_layer(m, layer, shape):

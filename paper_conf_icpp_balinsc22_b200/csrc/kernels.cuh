@@ -9,6 +9,8 @@ namespace mggcn {
 
 // process-wide count of kernel launches issued by this library
 void count_launches(int n);
+// test hook (mggcn_debug_comm_delay): one thread spinning on %globaltimer for ns nanoseconds
+cudaError_t launch_spin(uint64_t ns, cudaStream_t s);
 
 // ------------------------------------------------------------------ SpMM
 // One stage of the staged SpMM: out_i (+)= T_ij · B_j for one

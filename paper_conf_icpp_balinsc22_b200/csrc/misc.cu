@@ -328,6 +328,20 @@ cudaError_t launch_softmax_ce(float* Z, int64_t n, int C, int64_t ld, const int3
     return cudaGetLastError();
 }
 
+__global__ void spin_kernel(uint64_t ns) {
+    uint64_t t0, t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+    do {
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    } while (t - t0 < ns);
+}
+
+cudaError_t launch_spin(uint64_t ns, cudaStream_t s) {
+    spin_kernel<<<1, 1, 0, s>>>(ns);
+    count_launches(1);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_sum_partials(const double* partial, int count, double* out, cudaStream_t s) {
     sum_partials_kernel<<<1, 32, 0, s>>>(partial, count, out);
     count_launches(1);

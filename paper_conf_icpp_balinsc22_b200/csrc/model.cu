@@ -229,6 +229,9 @@ struct mggcn_model_s {
     // P-way run on its own, every collective skipped; per-rank compute time of a partition
     // too large for loopback (Papers-shaped at P = 8).  Results are invalid by construction.
     bool solo = false;
+    // delay injection (mggcn_debug_comm_delay): spin kernels of pseudo-random length
+    uint64_t delay_seed = 0, delay_ctr = 0;
+    int32_t delay_max_us = 0;
     size_t ws_bytes = 0;             // planned workspace bytes
     size_t sym_bytes = 0;            // symmetric region [0, sym_bytes) (IPC peers must agree)
     uint32_t spmm_seq = 0, wg_seq = 0, sc_seq = 0;
@@ -652,7 +655,19 @@ struct SpmmJob {
     const void* ctx;
 };
 
+// delay injection: a spin of 0..delay_max_us on stream s (test hook, P:929-941 rule check)
+int inject_delay(mggcn_model_s* m, cudaStream_t s) {
+    if (m->delay_max_us <= 0) return MGGCN_OK;
+    uint64_t z = m->delay_seed + 0x9E3779B97F4A7C15ull * (++m->delay_ctr);
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    CK(launch_spin((z % ((uint64_t)m->delay_max_us + 1)) * 1000ull, s));
+    return MGGCN_OK;
+}
+
 int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags) {
+    RC(inject_delay(m, m->cs));
     const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
     float* out = job.dst(m, r, job.ctx);
     ProfScope ps(m, PC_SPMM, m->cs);
@@ -683,6 +698,7 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
         const int q = (me + st) % P, k = st - 1, slot = k & 1;
         {
             ProfScope ps(m, PC_BCAST, m->ms);
+            RC(inject_delay(m, m->ms));
             if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
             CK(stream_wait_u32(m->ms, peer_ptr(m, q, m->flags_dev) + 0, seq));   // block q is ready
             const size_t bytes = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width * sizeof(float);
@@ -732,6 +748,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
         const int rq = q % c;                            // the replica group that needs block q
         {
             ProfScope ps(m, PC_BCAST, m->ms);
+            RC(inject_delay(m, m->ms));
             if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
                 Rank& r = m->ranks[0];
                 if (r.rep == rq) {
@@ -823,6 +840,7 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
         // ---- broadcast of block q (comm stream)
         {
             ProfScope ps(m, PC_BCAST, m->ms);
+            RC(inject_delay(m, m->ms));
             if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
                 Rank& r = m->ranks[0];
                 const size_t count = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width;
@@ -1892,6 +1910,18 @@ extern "C" int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* gathe
 }
 
 // ------------------------------------------------------------- test hooks
+extern "C" int mggcn_debug_comm_delay(mggcn_model m, uint64_t seed, int32_t max_us) {
+    MODEL_GUARD(m);
+    if (max_us < 0 || max_us > 10000) {
+        set_error("debug_comm_delay: max_us must be in [0, 10000]");
+        return MGGCN_EINVAL;
+    }
+    m->delay_seed = seed;
+    m->delay_ctr = 0;
+    m->delay_max_us = max_us;
+    return MGGCN_OK;
+}
+
 extern "C" int mggcn_debug_layer(mggcn_model m, int32_t layer, float* dst, int64_t ld) {
     MODEL_GUARD(m);
     RC(check_layer(m, layer));

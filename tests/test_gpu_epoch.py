@@ -26,9 +26,12 @@ def mg():
     return mg
 
 
-def run_library(mg, n, rp, col, vals, X, y, Ws, dims, P, seed, flags, host_inputs=False, steps=1, lr=0.01):
+def run_library(mg, n, rp, col, vals, X, y, Ws, dims, P, seed, flags, host_inputs=False, steps=1, lr=0.01,
+                delay=None, replicas=1):
     from paper_conf_icpp_balinsc22_b200 import GCN
-    gm = GCN(n, rp, col, vals, dims, P=P, perm_seed=seed, flags=flags, loopback=P > 1)
+    gm = GCN(n, rp, col, vals, dims, P=P, perm_seed=seed, flags=flags, loopback=P > 1, replicas=replicas)
+    if delay is not None:                       # (seed, max_us): spin kernels on both streams
+        mg.mggcn_debug_comm_delay(gm.m, *delay)
     gm.set_weights(Ws)
     Xl = gm.permute_rows(X)
     yl = gm.permute_rows(y)
@@ -36,7 +39,7 @@ def run_library(mg, n, rp, col, vals, X, y, Ws, dims, P, seed, flags, host_input
         Xin, yin = Xl, yl
     else:
         Xin, yin = torch.from_numpy(Xl).cuda(), torch.from_numpy(yl).cuda()
-    logits = torch.empty((n, dims[-1]), dtype=torch.float32, device="cuda")
+    logits = torch.empty((replicas * n, dims[-1]), dtype=torch.float32, device="cuda")
     out = {}
     for s in range(steps):
         out["loss"] = gm.forward(Xin, yin, want_loss=True, logits=logits if s == 0 else None)
@@ -385,3 +388,33 @@ def test_solo_timing_mode_on_disconnected_halves(mg, dims):
     with pytest.raises(mg.MggcnError) as e:
         GCN(n, rp, col, None, dims, P=2, rank=0, perm_seed=0, flags=mg.MGGCN_F_OVERLAP)
     assert e.value.code == mg.MGGCN_EINVAL
+
+
+@pytest.mark.parametrize("P,replicas", [(3, 1), (4, 1), (4, 2)])
+def test_delay_injection_keeps_results_bitwise(mg, P, replicas):
+    """SURVEY §4 pipeline-logic test: spin kernels of pseudo-random length (0..200 us) before
+    every broadcast (comm stream) and every SpMM stage (compute stream) reshuffle how the
+    two streams interleave; the P:929-941 event rule must keep logits, loss, W_G and the
+    updated W bitwise equal to the undelayed run, for several seeds, 1D and 1.5D."""
+    n, m = 1500, 30000
+    rp, col = gen.rmat_csr(n, m, 71)
+    dims = (24, 48, 9)
+    X = gen.features(n, dims[0], 72)
+    y = gen.labels(n, dims[-1], 73)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 74 + l) for l in range(2)]
+    base = run_library(mg, n, rp, col, None, X, y, Ws, dims, P, 75, mg.MGGCN_F_OVERLAP, steps=2, replicas=replicas)
+    for seed in (1, 2, 3):
+        d = run_library(mg, n, rp, col, None, X, y, Ws, dims, P, 75, mg.MGGCN_F_OVERLAP, steps=2,
+                        delay=(seed, 200), replicas=replicas)
+        assert np.array_equal(base["logits"], d["logits"])
+        assert base["loss"] == d["loss"]
+        for a, b in zip(base["WG"], d["WG"]):
+            assert np.array_equal(a, b)
+        for a, b in zip(base["W"], d["W"]):
+            assert np.array_equal(a, b)
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    gm = GCN(n, rp, col, None, dims, P=1, perm_seed=75)
+    with pytest.raises(mg.MggcnError) as e:
+        mg.mggcn_debug_comm_delay(gm.m, 0, 20000)
+    assert e.value.code == mg.MGGCN_EINVAL
+    gm.close()

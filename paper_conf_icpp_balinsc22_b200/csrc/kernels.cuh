@@ -19,7 +19,18 @@ cudaError_t launch_spin(uint64_t ns, cudaStream_t s);
 // directly (slot = -1); longer rows (R-MAT hubs) are cut into kSplit-entry
 // segments whose partial sums go to `partial[slot]` and are combined in
 // segment order by a fix-up kernel (deterministic, no float atomics).
-constexpr int kSplit = 2048;
+constexpr int kSplit = 2048;      // longest segment
+constexpr int kSplitMin = 128;    // shortest segment (small tiles, e.g. Reddit-shaped at P = 8)
+
+// Segment length of a tile with nnz entries: the longest work item is one warp
+// walking a segment, so a short stage (a small tile) needs short segments or
+// its hub segments become the stage's critical path; ~nnz / (4 x 2368 warps),
+// a power of two in [kSplitMin, kSplit].  MGGCN_SPMM_SPLIT overrides.
+inline int split_for(int64_t nnz) {
+    int s = kSplit;
+    while (s > kSplitMin && (int64_t)s * 4 * 2368 > nnz) s >>= 1;
+    return s;
+}
 
 struct SpmmTile {
     const int4* items = nullptr;   // {row, beg, end, slot}

@@ -53,6 +53,13 @@ struct HostItems {
 // consecutive items reuse gathered rows in L1/L2; numbering is unchanged).
 void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& order) {
     const auto& rp = t.rowptr;
+    static int split_env = -1;
+    if (split_env < 0) {
+        const char* e = getenv("MGGCN_SPMM_SPLIT");
+        split_env = e ? atoi(e) : 0;
+        if (split_env != 0 && (split_env < 32 || split_env > 65536)) split_env = 0;
+    }
+    const int64_t kSplit = split_env ? split_env : split_for(rp.back());
     for (int64_t r = 0; r < t.nrows; ++r) {
         const int64_t len = rp[r + 1] - rp[r];
         if (len > kSplit) {

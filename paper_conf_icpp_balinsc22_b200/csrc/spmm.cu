@@ -4,7 +4,7 @@
 //     C_i (+)= A_ij · H_j
 // with A_ij a CSR tile (Eq. 14-15) of Â'^T (forward, Eq. 6) or Â' (backward,
 // Eq. 9).  HBM/L2-bound gather: each non-zero pulls one dense feature row.
-//   - one warp per work item (a row, or a <= kSplit-entry segment of a hub
+//   - one warp per work item (a row, or a <= split_for(nnz)-entry segment of a hub
 //     row); the column indices of 32 entries are fetched by one coalesced
 //     128-B load and broadcast with shuffles;
 //   - lanes are split into S = 32/G slots x G lanes: each slot gathers one
@@ -288,20 +288,34 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
     }
 }
 
-// Hub rows: sum the segment partials in segment order, then the same epilogue.
-__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+// Hub rows: one block per split row.  Warp w sums segments w, w + 8, ... in order,
+// then warp 0 adds the 8 warp sums in warp order and applies the same epilogue
+// (a fixed order => deterministic, no float atomics).  w4 <= 128 (windows of at
+// most 512 floats).
+constexpr int kFixWarps = 8;
+__global__ void __launch_bounds__(kFixWarps * 32)
 spmm_fixup_kernel(const int4* __restrict__ splits, int64_t n_splits, const float4* __restrict__ partial,
                   int64_t ldp4, float4* __restrict__ out, int64_t ldo4, const float* __restrict__ rowscale, int w4,
                   int flags) {
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int lane = threadIdx.x & 31;
-    if (warp >= n_splits) return;
-    const int4 sp = __ldg(splits + warp);
+    __shared__ float4 red[kFixWarps][128];
+    const int64_t sid = blockIdx.x;
+    if (sid >= n_splits) return;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int4 sp = __ldg(splits + sid);
+    for (int q = lane; q < w4; q += 32) {
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll 4
+        for (int s = warp; s < sp.z; s += kFixWarps) acc = f4_add(acc, partial[(int64_t)(sp.y + s) * ldp4 + q]);
+        red[warp][q] = acc;
+    }
+    __syncthreads();
+    if (warp != 0) return;
     float4* orow = out + (int64_t)sp.x * ldo4;
     const float scale = rowscale ? __ldg(rowscale + sp.x) : 1.f;
     for (int q = lane; q < w4; q += 32) {
-        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int s = 0; s < sp.z; ++s) acc = f4_add(acc, partial[(int64_t)(sp.y + s) * ldp4 + q]);
+        float4 acc = red[0][q];
+#pragma unroll
+        for (int w = 1; w < kFixWarps; ++w) acc = f4_add(acc, red[w][q]);
         orow[q] = epilogue(acc, orow, q, flags, scale);
     }
 }
@@ -466,9 +480,8 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
             if (e != cudaSuccess) return e;
         }
         if (t.n_splits > 0) {
-            const int64_t blocks = (t.n_splits + kWarpsPerBlock - 1) / kWarpsPerBlock;
-            spmm_fixup_kernel<<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4, Ow,
-                                                                                ldo4, rowscale, w4, flags);
+            spmm_fixup_kernel<<<(unsigned)t.n_splits, kFixWarps * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4, Ow,
+                                                                               ldo4, rowscale, w4, flags);
             count_launches(1);
             e = cudaGetLastError();
             if (e != cudaSuccess) return e;

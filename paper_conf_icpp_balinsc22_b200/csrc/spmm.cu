@@ -288,7 +288,25 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
     }
 }
 
-// Hub rows: one block per split row.  Warp w sums segments w, w + 8, ... in order,
+// Hub rows with few segments: one warp per split row sums the partials in segment order.
+__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+spmm_fixup_warp_kernel(const int4* __restrict__ splits, int64_t n_splits, const float4* __restrict__ partial,
+                       int64_t ldp4, float4* __restrict__ out, int64_t ldo4, const float* __restrict__ rowscale,
+                       int w4, int flags) {
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (warp >= n_splits) return;
+    const int4 sp = __ldg(splits + warp);
+    float4* orow = out + (int64_t)sp.x * ldo4;
+    const float scale = rowscale ? __ldg(rowscale + sp.x) : 1.f;
+    for (int q = lane; q < w4; q += 32) {
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int s = 0; s < sp.z; ++s) acc = f4_add(acc, partial[(int64_t)(sp.y + s) * ldp4 + q]);
+        orow[q] = epilogue(acc, orow, q, flags, scale);
+    }
+}
+
+// Hub rows with many segments (short segments of small tiles): one block per split row.  Warp w sums segments w, w + 8, ... in order,
 // then warp 0 adds the 8 warp sums in warp order and applies the same epilogue
 // (a fixed order => deterministic, no float atomics).  w4 <= 128 (windows of at
 // most 512 floats).
@@ -480,9 +498,18 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
             if (e != cudaSuccess) return e;
         }
         if (t.n_splits > 0) {
-            spmm_fixup_kernel<<<(unsigned)t.n_splits, kFixWarps * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4, Ow,
-                                                                               ldo4, rowscale, w4, flags);
-            count_launches(1);
+            const int64_t few = t.n_splits_few, many = t.n_splits - t.n_splits_few;
+            if (few > 0) {
+                spmm_fixup_warp_kernel<<<(unsigned)((few + kWarpsPerBlock - 1) / kWarpsPerBlock),
+                                         kWarpsPerBlock * 32, 0, s>>>(t.splits, few, Pw, ldp4, Ow, ldo4, rowscale, w4,
+                                                                      flags);
+                count_launches(1);
+            }
+            if (many > 0) {
+                spmm_fixup_kernel<<<(unsigned)many, kFixWarps * 32, 0, s>>>(t.splits + few, many, Pw, ldp4, Ow, ldo4,
+                                                                            rowscale, w4, flags);
+                count_launches(1);
+            }
             e = cudaGetLastError();
             if (e != cudaSuccess) return e;
         }

@@ -20,8 +20,7 @@ cudaError_t launch_spin(uint64_t ns, cudaStream_t s);
 // segments whose partial sums go to `partial[slot]` and are combined in
 // segment order by a fix-up kernel (deterministic, no float atomics).
 constexpr int kSplit = 2048;      // longest segment
-constexpr int kSplitMin = 128;
-constexpr int kFixManySegs = 32;  // split rows with more segments get a whole block in the fix-up    // shortest segment (small tiles, e.g. Reddit-shaped at P = 8)
+constexpr int kSplitMin = 128;    // shortest segment (small tiles, e.g. Reddit-shaped at P = 8)
 
 // Segment length of a tile with nnz entries: the longest work item is one warp
 // walking a segment, so a short stage (a small tile) needs short segments or
@@ -40,9 +39,8 @@ struct SpmmTile {
     const int4* splits = nullptr;  // {row, first_slot, nslots, 0}
     int64_t n_splits = 0;
     int64_t n_slots = 0;
-    int64_t max_segs = 0;          // most segments of one split row
-    int64_t n_splits_few = 0;      // splits[0, n_splits_few): <= kFixManySegs segments (warp-per-row fix-up),
-                                   // the rest: block-per-row fix-up
+    int64_t split = kSplit;        // segment length of this tile (split_for); short segments
+                                   // (a small tile) => many per row => block-per-row fix-up
     const int32_t* col = nullptr;
     const float* val = nullptr;    // nullptr => pattern-only (value 1)
     int64_t nnz = 0, nrows = 0, ncols = 0;

@@ -44,8 +44,7 @@ struct HostItems {
     std::vector<int4> items, splits;
     int64_t nslots = 0;
     int64_t n_nonempty = 0;   // items[0, n_nonempty): hub segments and non-empty rows; then empty rows
-    int64_t max_segs = 0;     // most segments of one split row
-    int64_t n_splits_few = 0; // splits[0, n_splits_few) have <= kFixManySegs segments
+    int64_t split = kSplit;   // segment length used for this tile
 };
 
 // Work items of one tile: hub rows (> kSplit entries) are cut into segments
@@ -67,7 +66,6 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
         if (len > kSplit) {
             const int64_t nseg = (len + kSplit - 1) / kSplit;
             h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
-            h.max_segs = std::max(h.max_segs, nseg);
             for (int64_t s = 0; s < nseg; ++s) {
                 const int64_t b = rp[r] + s * kSplit, e = std::min<int64_t>(rp[r + 1], b + kSplit);
                 h.items.push_back(make_int4((int)r, (int)b, (int)e, (int)(h.nslots + s)));
@@ -75,10 +73,7 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
             h.nslots += nseg;
         }
     }
-    // split rows with few segments first (warp-per-row fix-up), then those with many (block-per-row)
-    std::stable_partition(h.splits.begin(), h.splits.end(), [](const int4& sp) { return sp.z <= kFixManySegs; });
-    h.n_splits_few = 0;
-    for (const int4& sp : h.splits) h.n_splits_few += sp.z <= kFixManySegs;
+    h.split = kSplit;
     // Empty rows go last: an accumulating middle stage skips them (adding an empty row's zero
     // sum is a no-op), which saves their output read-modify-write (SpmmTile::n_items_nz).
     for (int32_t r : order) {
@@ -405,8 +400,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                 t.nnz = ht.rowptr.back();
                 t.n_items = (int64_t)hi.items.size();
                 t.n_items_nz = hi.n_nonempty;
-                t.max_segs = hi.max_segs;
-                t.n_splits_few = hi.n_splits_few;
+                t.split = hi.split;
                 t.n_splits = (int64_t)hi.splits.size();
                 t.n_slots = hi.nslots;
                 t.items = b.take<int4>(hi.items.size());

@@ -498,18 +498,23 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
             if (e != cudaSuccess) return e;
         }
         if (t.n_splits > 0) {
-            const int64_t few = t.n_splits_few, many = t.n_splits - t.n_splits_few;
-            if (few > 0) {
-                spmm_fixup_warp_kernel<<<(unsigned)((few + kWarpsPerBlock - 1) / kWarpsPerBlock),
-                                         kWarpsPerBlock * 32, 0, s>>>(t.splits, few, Pw, ldp4, Ow, ldo4, rowscale, w4,
-                                                                      flags);
-                count_launches(1);
+            // one fix-up launch per stage: a warp per split row for long segments (large tiles,
+            // few segments per row), a block per split row for short ones (small tiles: a hub row
+            // has hundreds of segments); same-box A/B in profiles/r01_split_sweep.log
+            static int fix_env = -1;
+            if (fix_env < 0) {
+                const char* fe = getenv("MGGCN_FIXUP_BLOCK");   // experiment hook: 0 warp, 1 block
+                fix_env = fe ? (atoi(fe) ? 1 : 0) : 2;
             }
-            if (many > 0) {
-                spmm_fixup_kernel<<<(unsigned)many, kFixWarps * 32, 0, s>>>(t.splits + few, many, Pw, ldp4, Ow, ldo4,
-                                                                            rowscale, w4, flags);
-                count_launches(1);
-            }
+            const bool block = fix_env == 2 ? t.split < kSplit : fix_env == 1;
+            if (block)
+                spmm_fixup_kernel<<<(unsigned)t.n_splits, kFixWarps * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4,
+                                                                                   Ow, ldo4, rowscale, w4, flags);
+            else
+                spmm_fixup_warp_kernel<<<(unsigned)((t.n_splits + kWarpsPerBlock - 1) / kWarpsPerBlock),
+                                         kWarpsPerBlock * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4, Ow, ldo4,
+                                                                      rowscale, w4, flags);
+            count_launches(1);
             e = cudaGetLastError();
             if (e != cudaSuccess) return e;
         }

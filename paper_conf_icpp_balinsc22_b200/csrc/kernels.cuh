@@ -17,8 +17,8 @@ cudaError_t launch_spin(uint64_t ns, cudaStream_t s);
 // tile T (CSR, local indices).  Work is pre-cut on the host into items
 // {row, beg, end, slot}: rows with <= kSplit entries are one item written
 // directly (slot = -1); longer rows (R-MAT hubs) are cut into kSplit-entry
-// segments whose partial sums go to `partial[slot]`; the warp that finishes a
-// row's last segment combines them in segment order (deterministic, no float atomics).
+// segments whose partial sums go to `partial[slot]` and are combined in
+// segment order by a fix-up kernel (deterministic, no float atomics).
 constexpr int kSplit = 2048;      // longest segment
 constexpr int kSplitMin = 128;    // shortest segment (small tiles, e.g. Reddit-shaped at P = 8)
 
@@ -37,8 +37,6 @@ struct SpmmTile {
     int64_t n_items = 0;
     int64_t n_items_nz = 0;        // items[0, n_items_nz) are hub segments and non-empty rows, the rest empty rows
     const int4* splits = nullptr;  // {row, first_slot, nslots, 0}
-    const int32_t* slot_split = nullptr;   // partial slot -> its split row's index in `splits`
-    uint32_t* split_cnt = nullptr;         // per split row: segments finished in the current launch (0 between launches)
     int64_t n_splits = 0;
     int64_t n_slots = 0;
     int64_t split = kSplit;        // segment length of this tile (split_for); short segments

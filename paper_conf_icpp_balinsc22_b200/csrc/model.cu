@@ -45,7 +45,6 @@ struct HostItems {
     int64_t nslots = 0;
     int64_t n_nonempty = 0;   // items[0, n_nonempty): hub segments and non-empty rows; then empty rows
     int64_t split = kSplit;   // segment length used for this tile
-    std::vector<int32_t> slot_split;   // partial slot -> split row index
 };
 
 // Work items of one tile: hub rows (> kSplit entries) are cut into segments
@@ -66,7 +65,6 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
         const int64_t len = rp[r + 1] - rp[r];
         if (len > kSplit) {
             const int64_t nseg = (len + kSplit - 1) / kSplit;
-            for (int64_t s = 0; s < nseg; ++s) h.slot_split.push_back((int32_t)h.splits.size());
             h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
             for (int64_t s = 0; s < nseg; ++s) {
                 const int64_t b = rp[r] + s * kSplit, e = std::min<int64_t>(rp[r + 1], b + kSplit);
@@ -407,8 +405,6 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                 t.n_slots = hi.nslots;
                 t.items = b.take<int4>(hi.items.size());
                 t.splits = b.take<int4>(hi.splits.size());
-                t.slot_split = b.take<int32_t>(hi.slot_split.size());
-                t.split_cnt = b.take<uint32_t>(hi.splits.size());
                 t.col = b.take<int32_t>(ht.col.size());
                 t.hot_enc = want_hot_classes(ht);
                 t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
@@ -451,13 +447,9 @@ int upload_static(mggcn_model_s* m) {
                 if (!hi.items.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.items), hi.items.data(), sizeof(int4) * hi.items.size(),
                                        cudaMemcpyHostToDevice, m->cs));
-                if (!hi.splits.empty()) {
+                if (!hi.splits.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.splits), hi.splits.data(),
                                        sizeof(int4) * hi.splits.size(), cudaMemcpyHostToDevice, m->cs));
-                    CK(cudaMemcpyAsync(const_cast<int32_t*>(t.slot_split), hi.slot_split.data(),
-                                       sizeof(int32_t) * hi.slot_split.size(), cudaMemcpyHostToDevice, m->cs));
-                    CK(cudaMemsetAsync(t.split_cnt, 0, sizeof(uint32_t) * hi.splits.size(), m->cs));
-                }
                 if (!ht.col.empty()) {
                     std::vector<int32_t> enc;
                     if (t.hot_enc) enc = encode_hot_classes(ht);

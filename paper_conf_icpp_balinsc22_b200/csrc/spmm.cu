@@ -149,9 +149,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, minb_for<G, CH>())
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const float4* __restrict__ B, int64_t ldb4,
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,
-                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T,
-                  const int4* __restrict__ splits, const int32_t* __restrict__ slot_split,
-                  uint32_t* __restrict__ split_cnt) {
+                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T) {
     constexpr int S = 32 / G;
     // U entries per slot per group; U * S <= 32 so a group fits a 32-entry chunk
     constexpr int U = unroll_for<CH>() < G ? unroll_for<CH>() : G;
@@ -283,34 +281,60 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 }
             }
         }
-        if (it.w >= 0) {
-            // Hub-row fix-up, fused: the warp that finishes a split row's LAST segment (an
-            // integer counter per split row) sums the row's partials in segment order and
-            // applies the epilogue, so the result does not depend on which warp that is.
-            __threadfence();                        // this segment's partial, visible device-wide
-            __syncwarp();
-            const int sidx = __ldg(slot_split + it.w);
-            uint32_t prev = 0;
-            if (lane == 0) prev = atomicAdd(split_cnt + sidx, 1u);
-            prev = __shfl_sync(0xffffffffu, prev, 0);
-            const int4 sp = __ldg(splits + sidx);
-            if (prev == (uint32_t)sp.z - 1u) {
-                __threadfence();                    // acquire the other segments' partials
-                const float sc = rowscale ? __ldg(rowscale + sp.x) : 1.f;
-                float4* orow = out + (int64_t)sp.x * ldo4;
-                for (int q = lane; q < w4; q += 32) {
-                    float4 a = make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll 8
-                    for (int s2 = 0; s2 < sp.z; ++s2) a = f4_add(a, __ldcg(partial + (int64_t)(sp.y + s2) * ldp4 + q));
-                    orow[q] = epilogue(a, orow, q, flags, sc);
-                }
-                if (lane == 0) split_cnt[sidx] = 0u;   // reset for the next launch (stream-ordered)
-            }
-        }
         cur_c = nxt_c;
         cur_v = nxt_v;
         it = itn;
         itn = it2;
+    }
+}
+
+// Hub rows with few segments: one warp per split row sums the partials in segment order.
+__global__ void __launch_bounds__(kWarpsPerBlock * 32)
+spmm_fixup_warp_kernel(const int4* __restrict__ splits, int64_t n_splits, const float4* __restrict__ partial,
+                       int64_t ldp4, float4* __restrict__ out, int64_t ldo4, const float* __restrict__ rowscale,
+                       int w4, int flags) {
+    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (warp >= n_splits) return;
+    const int4 sp = __ldg(splits + warp);
+    float4* orow = out + (int64_t)sp.x * ldo4;
+    const float scale = rowscale ? __ldg(rowscale + sp.x) : 1.f;
+    for (int q = lane; q < w4; q += 32) {
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int s = 0; s < sp.z; ++s) acc = f4_add(acc, partial[(int64_t)(sp.y + s) * ldp4 + q]);
+        orow[q] = epilogue(acc, orow, q, flags, scale);
+    }
+}
+
+// Hub rows with many segments (short segments of small tiles): one block per split row.  Warp w sums segments w, w + 8, ... in order,
+// then warp 0 adds the 8 warp sums in warp order and applies the same epilogue
+// (a fixed order => deterministic, no float atomics).  w4 <= 128 (windows of at
+// most 512 floats).
+constexpr int kFixWarps = 8;
+__global__ void __launch_bounds__(kFixWarps * 32)
+spmm_fixup_kernel(const int4* __restrict__ splits, int64_t n_splits, const float4* __restrict__ partial,
+                  int64_t ldp4, float4* __restrict__ out, int64_t ldo4, const float* __restrict__ rowscale, int w4,
+                  int flags) {
+    __shared__ float4 red[kFixWarps][128];
+    const int64_t sid = blockIdx.x;
+    if (sid >= n_splits) return;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int4 sp = __ldg(splits + sid);
+    for (int q = lane; q < w4; q += 32) {
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll 4
+        for (int s = warp; s < sp.z; s += kFixWarps) acc = f4_add(acc, partial[(int64_t)(sp.y + s) * ldp4 + q]);
+        red[warp][q] = acc;
+    }
+    __syncthreads();
+    if (warp != 0) return;
+    float4* orow = out + (int64_t)sp.x * ldo4;
+    const float scale = rowscale ? __ldg(rowscale + sp.x) : 1.f;
+    for (int q = lane; q < w4; q += 32) {
+        float4 acc = red[0][q];
+#pragma unroll
+        for (int w = 1; w < kFixWarps; ++w) acc = f4_add(acc, red[w][q]);
+        orow[q] = epilogue(acc, orow, q, flags, scale);
     }
 }
 
@@ -354,8 +378,7 @@ void launch_one(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, i
     const int over = yenv > 1 ? yenv : ((flags & SPMM_YIELD) ? (yenv == 1 ? 1 : kYieldBlocks) : 1);
     const int64_t blocks = persistent_blocks<G, CH, V, H>(t.n_items, over);
     spmm_stage_kernel<G, CH, V, H><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
-        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, t.splits,
-        t.slot_split, t.split_cnt);
+        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T);
 }
 
 template <int G, int CH>
@@ -472,6 +495,27 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
         cudaError_t e;
         if (t.n_items > 0) {
             e = dispatch_gc(w4, t, Bw, ldb4, Ow, ldo4, Pw, ldp4, rowscale, flags, hot_T, s);
+            if (e != cudaSuccess) return e;
+        }
+        if (t.n_splits > 0) {
+            // one fix-up launch per stage: a warp per split row for long segments (large tiles,
+            // few segments per row), a block per split row for short ones (small tiles: a hub row
+            // has hundreds of segments); same-box A/B in profiles/r01_split_sweep.log
+            static int fix_env = -1;
+            if (fix_env < 0) {
+                const char* fe = getenv("MGGCN_FIXUP_BLOCK");   // experiment hook: 0 warp, 1 block
+                fix_env = fe ? (atoi(fe) ? 1 : 0) : 2;
+            }
+            const bool block = fix_env == 2 ? t.split < kSplit : fix_env == 1;
+            if (block)
+                spmm_fixup_kernel<<<(unsigned)t.n_splits, kFixWarps * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4,
+                                                                                   Ow, ldo4, rowscale, w4, flags);
+            else
+                spmm_fixup_warp_kernel<<<(unsigned)((t.n_splits + kWarpsPerBlock - 1) / kWarpsPerBlock),
+                                         kWarpsPerBlock * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4, Ow, ldo4,
+                                                                      rowscale, w4, flags);
+            count_launches(1);
+            e = cudaGetLastError();
             if (e != cudaSuccess) return e;
         }
     }

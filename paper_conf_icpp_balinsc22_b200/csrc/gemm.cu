@@ -427,8 +427,14 @@ constexpr int kMnBK = 16;
 // (split -> MMA), sized from BN so narrow-N products keep more k blocks of
 // the streamed operands in flight (BN = 256: 6 raw + 2 lo stages of 24 KB;
 // BN = 64: 10 raw + 4 lo stages of 12 KB).
-constexpr int kMnBudget = 8 * 24576;
-constexpr int kMnMaxNR = 10, kMnMaxNL = 4;
+#ifndef MGGCN_MN_BUDGET
+#define MGGCN_MN_BUDGET (8 * 24576)
+#endif
+#ifndef MGGCN_MN_MAXNR
+#define MGGCN_MN_MAXNR 10
+#endif
+constexpr int kMnBudget = MGGCN_MN_BUDGET;
+constexpr int kMnMaxNR = MGGCN_MN_MAXNR, kMnMaxNL = 4;
 constexpr int kMnBars = kMnBudget;
 constexpr int kMnSmem = kMnBars + 512 + 1024;
 __host__ __device__ __forceinline__ int mn_stage_bytes(int BN) { return 8192 + (BN / 32) * 2048; }
@@ -604,17 +610,22 @@ constexpr int kRowBK = 16;
 // B_hi BN x 64 B | B_lo BN x 64 B, as many as fit the budget (3 for BN = 256,
 // 7 for BN = 48): narrow-N products are bound by the A stream, which needs
 // more k blocks in flight than the MMAs do.
+// Without the mask (forward F1, and B3 when no ReLU' applies) the old-C
+// chunks are never loaded, so the ring starts at kRowOld and gets their 32 KB
+// too (BN = 256: 3 -> 4 stages, BN = 48: 7 -> 8); MGGCN_ROW_RING=0 keeps the
+// short ring for A/B.
 constexpr int kRowOut = 0;
 constexpr int kRowOld = 2 * 16384;
 constexpr int kRowStage0 = 4 * 16384;
 constexpr int kRowStageBudget = 160 * 1024;
-constexpr int kRowMaxNS = 8;
+constexpr int kRowMaxNS = 10;
 constexpr int kRowBars = kRowStage0 + kRowStageBudget;
-constexpr int kRowSmem = kRowBars + 256 + 1024;
+constexpr int kRowSmem = kRowBars + 512 + 1024;
+constexpr int GEMM_ROW_LONGRING = 1 << 20;   // internal KParams flag: ring starts at kRowOld
 
 __host__ __device__ __forceinline__ int row_stage_bytes(int BN) { return (16384 + 2 * BN * 64 + 1023) / 1024 * 1024; }
-__host__ __device__ __forceinline__ int row_stages(int BN) {
-    const int ns = kRowStageBudget / row_stage_bytes(BN);
+__host__ __device__ __forceinline__ int row_stages(int BN, bool longring = false) {
+    const int ns = (kRowStageBudget + (longring ? kRowStage0 - kRowOld : 0)) / row_stage_bytes(BN);
     return ns < kRowMaxNS ? ns : kRowMaxNS;
 }
 
@@ -705,7 +716,9 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     const int BN = p.BN;
     const int BNH = PAIR ? BN / 2 : BN;         // rows of W^T staged by this CTA
     const uint32_t tcols = BN > 128 ? 512u : 256u;
-    const int NS = row_stages(BNH), SB = row_stage_bytes(BNH);
+    const bool longring = (p.flags & GEMM_ROW_LONGRING) != 0 && !mask;
+    const int NS = row_stages(BNH, longring), SB = row_stage_bytes(BNH);
+    uint8_t* const ring = smem + (longring ? kRowOld : kRowStage0);
     const int kBlo = 16384 + BNH * 64;           // B_lo offset within a stage
     const uint32_t crank = PAIR ? cluster_rank() : 0u;
     const int nunits = PAIR ? (int)(gridDim.x / 2) : (int)gridDim.x;    // tile workers (CTA pairs or CTAs)
@@ -754,7 +767,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                 const int nt = tile % p.n_tiles, mt = PAIR ? (tile / p.n_tiles) * 2 + (int)crank : tile / p.n_tiles;
                 const int nb = nt * BN + (int)crank * BNH;   // first W^T row staged here
                 for (int kb = 0; kb < nkb; ++kb) {
-                    uint8_t* st = smem + kRowStage0 + s * SB;
+                    uint8_t* st = ring + s * SB;
                     if (!PAIR && MGGCN_ROW_PF > 0) {   // A streams from DRAM: warm L2 ahead of the ring
                         const int kp = kb + MGGCN_ROW_PF;
                         if (kp < nkb) tma_prefetch_2d(&tmA, kp * kRowBK, mt * BM);
@@ -780,7 +793,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
         uint32_t ph = 0;
         for (int tile = unit; tile < total_tiles; tile += nunits) {
             for (int kb = 0; kb < nkb; ++kb) {
-                float4* a = reinterpret_cast<float4*>(smem + kRowStage0 + s * SB);
+                float4* a = reinterpret_cast<float4*>(ring + s * SB);
                 mbar_wait(full + s, ph);
                 // raw A [0, 512) -> lo at +512; raw B [1024, 1024 + 4 BN) -> lo at +4 BN (float4
                 // units, same swizzled offsets).  3xTF32: the MMA reads a raw x as hi = x &
@@ -822,7 +835,7 @@ gemm_rows_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
                     if (PAIR) mbar_wait_cluster(xf + s, ph);
                     else mbar_wait(xf + s, ph);
                     tc_fence_after();
-                    const uint32_t base = smem_u32(smem + kRowStage0 + s * SB);
+                    const uint32_t base = smem_u32(ring + s * SB);
                     const uint64_t ah = sw64_desc(base), al = sw64_desc(base + 8192);
                     const uint64_t bh = sw64_desc(base + 16384), bl = sw64_desc(base + kBlo);
 #pragma unroll
@@ -1212,6 +1225,11 @@ cudaError_t gemm_launch(const GemmPlan& g, cudaStream_t s) {
     kp.k_chunks = g.k_chunks; kp.k_chunk_len = (int)g.k_chunk_len;
     kp.C = g.C; kp.ldc = g.ldc; kp.partial = g.partial; kp.rowscale = g.rowscale;
     kp.flags = g.flags; kp.op2 = g.op == 2;
+    static const bool longring = [] {
+        const char* e = getenv("MGGCN_ROW_RING");
+        return !(e && atoi(e) == 0);
+    }();
+    if (g.op != 2 && g.variant != 2 && longring) kp.flags |= GEMM_ROW_LONGRING;
     for (int i = 0; i < 3; ++i) kp.desc_mn[i] = g.desc_mn[i];
 
     if (g.op == 2) return g.variant == 1 ? launch_wgrad_mn(g, kp, s) : launch_wgrad(g, kp, s);

@@ -146,6 +146,43 @@ class ClockSampler:
 _ORACLE_CACHE = {}
 
 
+def host_info():
+    """CPU model and core count of the host the oracle runs on (SURVEY §8(d) "Oracle timing")."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except Exception:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity_cores": len(os.sched_getaffinity(0))}
+
+
+class pinned_one_core:
+    """Run the oracle single-threaded on ONE core (os.sched_setaffinity), restoring the mask after."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.core = min(self.old)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.old)
+
+
+def oracle_calibration(workload):
+    """Full single-core oracle epoch vs the row-sampled estimate, measured once on one host by
+    scripts/calibrate_oracle.py (profiles/r02_oracle_calibration.json); None if absent."""
+    path = os.path.join(ROOT, "profiles", "r02_oracle_calibration.json")
+    try:
+        return json.load(open(path)).get(workload)
+    except Exception:
+        return None
+
+
 def oracle_epoch_sample(w, rp, col, rows_per_step, seed=0):
     """Time the CPU oracle's ops for ONE epoch of workload `w` restricted to a
     random sample of `rows_per_step` output rows (every SpMM, GEMM and the CE
@@ -202,6 +239,41 @@ def oracle_epoch_sample(w, rp, col, rows_per_step, seed=0):
 L2_GATHER_PEAK_GBPS = 19480.5
 
 
+def _git_blob_sha(path):
+    import hashlib
+    try:
+        data = open(path, "rb").read()
+    except Exception:
+        return None
+    return hashlib.sha1(b"blob %d\0" % len(data) + data).hexdigest()
+
+
+def library_sha256():
+    import hashlib
+    try:
+        return hashlib.sha256(open(os.path.join(ROOT, "paper_conf_icpp_balinsc22_b200", "libmggcn.so"),
+                                   "rb").read()).hexdigest()[:16]
+    except Exception:
+        return None
+
+
+def stored_traffic(workload, P):
+    """roofline.traffic: DRAM bytes per SpMM launch from one ncu --set full capture
+    (scripts/profile_round.sh + scripts/summarize_profiles.py), with the build it was taken on."""
+    path = os.path.join(ROOT, "profiles", f"spmm_traffic_{workload}_P{P}.json")
+    if not os.path.exists(path):
+        return None, None
+    try:
+        d = json.load(open(path))
+    except Exception:
+        return None, None
+    cur = library_sha256()
+    return d.get("dram_bytes_per_launch"), {
+        "file": os.path.relpath(path, ROOT), "tag": d.get("tag"), "git_sha": d.get("git_sha"),
+        "so_sha256": d.get("so_sha256"), "current_so_sha256": cur,
+        "same_build": (d.get("so_sha256") == cur) if d.get("so_sha256") else None}
+
+
 def spmm_widths(dims):
     """Widths of the SpMMs of one epoch (§4.4 order rule C10, first-layer skip C11)."""
     ws = []
@@ -237,7 +309,8 @@ def l2_gather_roofline(dims, work, spmm_ms_per_epoch, cache=False):
     return {"bound": "l2 (SM<-L2 line rate of random row gathers)", "achieved": ach, "peak": L2_GATHER_PEAK_GBPS,
             "unit": "GB/s", "frac": ach / L2_GATHER_PEAK_GBPS, "line_bytes_per_epoch": lb,
             "peak_source": "bench_micro/dsmem_gather.cu: uniform 512-B row gathers from an L2-resident table "
-                           "(profiles/r01_dsmem_gather.jsonl)"}
+                           "(profiles/r01_dsmem_gather.jsonl)",
+            "peak_source_blob_sha": _git_blob_sha(os.path.join(ROOT, "bench_micro", "dsmem_gather.cu"))}
 
 
 def auto_rows(w):
@@ -255,18 +328,25 @@ def run_reference(args):
     rp, col = gen.rmat_csr(w.n, w.m, w.seed_G)
     R = args.oracle_rows or auto_rows(w)
     vals, walls = [], []
-    for s in range(args.warmup + args.steps):
-        est, wall, _ = oracle_epoch_sample(w, rp, col, R, seed=s)
-        if s >= args.warmup:
-            vals.append(est)
-            walls.append(wall)
-    value = statistics.median(vals)
-    sample = f"{R} random output rows of every SpMM/GEMM/CE op of one epoch (n = {w.n}), scaled by n/R; Adam full"
+    with pinned_one_core():
+        for s in range(args.warmup + args.steps):
+            est, wall, _ = oracle_epoch_sample(w, rp, col, R, seed=s)
+            if s >= args.warmup:
+                vals.append(est)
+                walls.append(wall)
+    raw = statistics.median(vals)
+    cal = oracle_calibration(w.name)
+    value = raw * cal["ratio"] if cal else raw
+    sample = (f"{R} random output rows of every SpMM/GEMM/CE op of one epoch (n = {w.n}), scaled by n/R; Adam full; "
+              f"one pinned core" + ("; x calibration ratio full/sampled from profiles/r02_oracle_calibration.json"
+                                   if cal else "; uncalibrated"))
     line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": statistics.median(walls) * 1e3,
             "higher_is_better": False, "scaling": "strong", "vs_baseline": None, "dtype": "f32 storage, f64 accumulate",
             "data": "synthetic", "config": workload_desc(w, 1),
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             "estimated": True, "rows_sampled": R, "sampled_estimate_ms": raw, "calibration": cal,
+                             "host": host_info()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -358,6 +438,7 @@ def main():
     ms = ev0.elapsed_time(ev1) / args.steps
     prof = gm.profile(reset=True)
     work = gm.epoch_work()
+    work_detail = gm.epoch_work_detail()
     ms_eager = max_over_ranks(dist, ms)
 
     # ---- the same epochs as one CUDA graph each (mggcn_epoch_capture / _replay): identical
@@ -518,21 +599,44 @@ def main():
     spmm_ms, spmm_n = prof["spmm"]
     spmm_launch_ms = spmm_ms / max(spmm_n, 1)
     launches_per_epoch = spmm_n / args.steps
-    bytes_per_launch = work["spmm_bytes"] / max(launches_per_epoch, 1)
+    wd = work_detail
+    # SURVEY §8(d) compulsory bytes: 4 B per non-zero of the tiles as partitioned (pattern-only),
+    # rowptr, each gathered row once, each output row once
+    bytes_per_launch = wd["spmm_bytes"] / max(launches_per_epoch, 1)
+    struct_per_launch = wd["spmm_struct_bytes"] / max(launches_per_epoch, 1)
     achieved = bytes_per_launch / (spmm_launch_ms * 1e-3) / 1e9 if spmm_ms > 0 else 0.0
-    gather_gbs = (work["spmm_gather_bytes"] / max(launches_per_epoch, 1)) / (spmm_launch_ms * 1e-3) / 1e9 \
+    gather_gbs = (wd["spmm_gather_bytes"] / max(launches_per_epoch, 1)) / (spmm_launch_ms * 1e-3) / 1e9 \
         if spmm_ms > 0 else 0.0
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", f"spmm_traffic_{args.workload}_P{P}.json")
-    if os.path.exists(tpath):
-        try:
-            traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+    traffic, traffic_src = stored_traffic(args.workload, P)
     l2_gather = l2_gather_roofline(w.dims, work, spmm_ms / args.steps, cache=False)
     gemm_ms, gemm_n = prof["gemm"]
+    # dense TF32 peak = the measured bf16 peak x the nominal tf32 : bf16 ratio (1 : 2); the GEMMs are
+    # timed inside a long epoch, so the sustained figure is the denominator of their fraction
     tf32_peak = float(peaks.get("bf16_tflops_sustained", 1352.7)) / 2.0
-
+    tf32_burst = float(peaks.get("bf16_tflops", 1623.0)) / 2.0
+    gemm_tflops = wd["gemm_flops"] / (gemm_ms / args.steps * 1e-3) / 1e12 if gemm_ms else None
+    mma_passes = 1 if args.tf32x1 else 3            # 3xTF32 issues hi*hi + hi*lo + lo*hi
+    # per-epoch roofline (BASELINE.json metric; SURVEY §8(d) "Per-epoch bounds per GPU")
+    nvlink = 900.0
+    t_spmm = wd["spmm_bytes"] / (hbm * 1e9) * 1e3
+    t_gemm = wd["gemm_flops"] / (tf32_burst * 1e12) * 1e3
+    t_bc = wd["bcast_bytes"] / (nvlink * 1e9) * 1e3
+    hbm_all = wd["spmm_bytes"] + wd["gemm_bytes"] + wd["ce_bytes"] + wd["bcast_bytes"]
+    t_tight_hbm = hbm_all / (hbm * 1e9) * 1e3
+    official = max(t_spmm, t_gemm, t_bc)
+    tight = max(t_tight_hbm, t_gemm, t_bc)
+    epoch_roofline = {
+        "official_bound_ms": official, "official_frac": official / ms_max,
+        "tight_bound_ms": tight, "tight_frac": tight / ms_max,
+        "terms_ms": {"spmm_compulsory_over_hbm": t_spmm, "gemm_flops_over_tf32": t_gemm,
+                     "bcast_over_nvlink": t_bc, "all_compulsory_hbm_bytes_over_hbm": t_tight_hbm},
+        "bytes": {"spmm_compulsory": wd["spmm_bytes"], "gemm_operands": wd["gemm_bytes"], "ce": wd["ce_bytes"],
+                  "bcast_recv": wd["bcast_bytes"]},
+        "gemm_gflop": wd["gemm_flops"] / 1e9,
+        "peaks": {"hbm_GBps": hbm, "tf32_TFLOPs": tf32_burst, "nvlink_GBps": nvlink},
+        "how": "official = max(SpMM compulsory bytes / HBM, GEMM flops / dense TF32, broadcast bytes / NVLink) "
+               "(BASELINE.json north_star); tight = max(all compulsory HBM bytes incl. GEMM operands, CE and "
+               "broadcast writes / HBM, the other two); frac = bound / measured epoch ms (this line's value)"}
     line = {
         "metric": METRIC, "value": ms_max, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": False, "scaling": "strong",
@@ -550,17 +654,27 @@ def main():
         "clocks": clk,
         "roofline": {"bound": "hbm", "kernel": "spmm_stage (staged CSR SpMM, F2/B1)",
                      "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
-                     "traffic": traffic, "peak_source": peak_src,
+                     "traffic": traffic, "traffic_source": traffic_src, "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": bytes_per_launch,
+                     "struct_bytes_per_launch": struct_per_launch,
                      "launch_ms": spmm_launch_ms, "launches_per_epoch": launches_per_epoch,
                      "gather_model_GBps": gather_gbs,
-                     "note": "achieved = compulsory bytes (indices + rowptr + each input and output row once, "
-                             "SURVEY §8d) / measured launch time; gather_model_GBps = nnz*width*4 B / time; "
-                             "a launch = one SpMM stage (its column-window kernels + hub fix-up)",
+                     "note": "achieved = SURVEY §8(d) compulsory bytes (4 B per non-zero of the partitioned "
+                             "tiles, rowptr, each gathered and each output row once) / measured mean launch time "
+                             "(CUDA events on the compute stream); struct_bytes_per_launch = the same with the "
+                             "device tiles' coalesced (index + multiplicity) entries; gather_model_GBps = "
+                             "coalesced nnz * width * 4 B / time; a launch = one SpMM stage (its column-window "
+                             "kernels + hub fix-up)",
                      "l2_gather": l2_gather},
+        "epoch_roofline": epoch_roofline,
         "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
-        "gemm": {"tflops": work["gemm_flops"] / (gemm_ms / args.steps * 1e-3) / 1e12 if gemm_ms else None,
-                 "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps},
+        "gemm": {"tflops": gemm_tflops, "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps,
+                 "frac_model_flops": gemm_tflops / tf32_peak if gemm_tflops else None,
+                 "mma_passes": mma_passes,
+                 "tensor_frac": gemm_tflops * mma_passes / tf32_peak if gemm_tflops else None,
+                 "how": "model flops 2MNK per product / GEMM ms per epoch (CUDA events); tensor_frac counts the "
+                        "MMA work actually issued (3 TF32 passes for 3xTF32) against the sustained dense TF32 "
+                        "peak (MEASURED_PEAKS bf16 sustained / 2)"},
         "loss_after": loss_now,
         "cache_l0": cache_l0,
         "exposed_comm": exposed,
@@ -571,12 +685,19 @@ def main():
     if world == 1 and not args.no_cpu_baseline:
         R = args.oracle_rows or auto_rows(w)
         ests = []
-        for s in range(3):
-            est, _, _ = oracle_epoch_sample(w, rp, col, R, seed=s)
-            ests.append(est)
-        line["cpu_baseline"] = {"value": statistics.median(ests), "unit": UNIT, "cores": 1, "kind": "oracle",
+        with pinned_one_core():
+            for s in range(3):
+                est, _, _ = oracle_epoch_sample(w, rp, col, R, seed=s)
+                ests.append(est)
+        raw = statistics.median(ests)
+        cal = oracle_calibration(w.name)
+        line["cpu_baseline"] = {"value": raw * cal["ratio"] if cal else raw, "unit": UNIT, "cores": 1, "kind": "oracle",
                                 "sample": f"3 x {R} random output rows of every SpMM/GEMM/CE op of one epoch "
-                                          f"(n = {w.n}), scaled by n/R; Adam full; single thread"}
+                                          f"(n = {w.n}), scaled by n/R; Adam full; one pinned core" +
+                                          ("; x calibration ratio (full single-core oracle epoch / sampled estimate, "
+                                           "profiles/r02_oracle_calibration.json)" if cal else "; uncalibrated"),
+                                "estimated": True, "rows_sampled": R, "sampled_estimate_ms": raw,
+                                "calibration": cal, "host": host_info()}
     print(json.dumps(line), flush=True)
     gm.close()
     if world > 1:

@@ -95,7 +95,11 @@ enum {
                                  k / P').  NCCL: nlocal = 1, nccl id shared by all 2P'
                                  processes, MGGCN_F_REPLICA1 on the replica-1 processes.
                                  Not with MGGCN_F_IPC (EUNSUPPORTED). */
-    MGGCN_F_REPLICA1 = 1024u  /* with MGGCN_F_REPL2 and nlocal = 1: this process is replica 1 */
+    MGGCN_F_REPLICA1 = 1024u, /* with MGGCN_F_REPL2 and nlocal = 1: this process is replica 1 */
+    MGGCN_F_TIMELINE = 2048u  /* record one CUDA event pair per op on the stream it runs on,
+                                 tagged with the SpMM index and stage (the per-stage
+                                 comm / compute timelines of Fig. 6 / Fig. 8, P:1372-1403,
+                                 P:1545-1580); read with mggcn_get_timeline */
 };
 
 /* Size of one rank's IPC descriptor (mggcn_ipc_export). */
@@ -253,6 +257,16 @@ int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, const float* 
  * stream each op is launched on.  Classes: 0 spmm, 1 gemm, 2 loss, 3 adam,
  * 4 bcast, 5 allreduce, 6 other.  Synchronises. */
 int mggcn_get_profile(mggcn_model m, double* ms /*[7]*/, int64_t* launches /*[7]*/, int32_t reset);
+/* Per-stage timeline (MGGCN_F_TIMELINE; the paper's Fig. 6 / Fig. 8 stage
+ * timelines).  Copies up to `cap` records made
+ * since the last reset, in issue order: meta[5*i ..] = {op class (as in
+ * mggcn_get_profile), SpMM index within the epoch (-1 outside a SpMM), stage
+ * (-1 = local stage; k >= 0 = k-th remote block / broadcast), local rank
+ * index, stream (0 compute, 1 comm)}, t_ms[2*i ..] = {start, end} in device
+ * milliseconds relative to the first record's start.  *count = number of
+ * records available (may exceed cap).  Synchronises both streams.
+ * EINVAL: cap < 0, or cap > 0 with a NULL array. */
+int mggcn_get_timeline(mggcn_model m, int64_t cap, int32_t* meta, double* t_ms, int64_t* count, int32_t reset);
 /* Algorithmic work of one epoch of this model's rows for the roofline
  * (DESIGN.md §6): spmm_bytes = compulsory SpMM bytes
  * (indices + rowptr + each input row once + each output row once, summed over
@@ -261,6 +275,18 @@ int mggcn_get_profile(mggcn_model m, double* ms /*[7]*/, int64_t* launches /*[7]
  * broadcasts.  Any pointer may be NULL. */
 int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* spmm_gather_bytes, double* gemm_flops,
                      double* bcast_bytes);
+
+/* The same work model in more detail: writes min(n, 9) values into out and
+ * returns 9 (or a negative error): [0] spmm_bytes (SURVEY §8(d) compulsory:
+ * 4 B per non-zero of the partitioned tiles, +4 B if weighted, + rowptr + each
+ * gathered row once + each output row once), [1] the same with the device
+ * tiles' own structure (duplicates coalesced; index + multiplicity value per
+ * entry), [2] gather bytes of the coalesced tiles (nnz * width * 4), [3] gather
+ * bytes of the raw tiles, [4] gemm_flops, [5] gemm compulsory bytes
+ * (4(MK + KN + MN) per product, + MN for the B3 ReLU' mask), [6] bcast_bytes
+ * (received), [7] softmax-CE bytes (2 n C 4), [8] SpMM stage launches per epoch.
+ * EINVAL: NULL out, n < 0. */
+int mggcn_epoch_work_detail(mggcn_model m, double* out, int32_t n);
 
 /* Number of kernels this library has launched in this process (all models,
  * all debug hooks).  Read before and after a timed region to count them. */

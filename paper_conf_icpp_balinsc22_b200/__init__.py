@@ -26,6 +26,7 @@ MGGCN_F_CACHE_L0 = 128
 MGGCN_F_IPC = 256
 MGGCN_F_REPL2 = 512        # 1.5D, replication factor c = 2
 MGGCN_F_REPLICA1 = 1024    # with MGGCN_F_REPL2, nlocal = 1: this process is replica 1
+MGGCN_F_TIMELINE = 2048    # per-stage comm / compute event timeline (mggcn_get_timeline)
 MGGCN_IPC_BLOB_BYTES = 128
 PROFILE_CLASSES = ("spmm", "gemm", "loss", "adam", "bcast", "allreduce", "other")
 
@@ -37,7 +38,8 @@ EXPORTS = (
     "mggcn_get_profile", "mggcn_epoch_work", "mggcn_graph_free", "mggcn_part_free", "mggcn_model_free",
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
     "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
-    "mggcn_epoch_replay", "mggcn_debug_comm_delay",
+    "mggcn_epoch_replay", "mggcn_debug_comm_delay", "mggcn_get_timeline",
+    "mggcn_epoch_work_detail",
 )
 
 
@@ -82,7 +84,9 @@ def _load():
         "mggcn_get_adam": ([P, i32, P, P, P], ctypes.c_int),
         "mggcn_set_adam": ([P, i32, P, P, i64], ctypes.c_int),
         "mggcn_get_profile": ([P, P, P, i32], ctypes.c_int),
+        "mggcn_get_timeline": ([P, i64, P, P, P, i32], ctypes.c_int),
         "mggcn_epoch_work": ([P, P, P, P, P], ctypes.c_int),
+        "mggcn_epoch_work_detail": ([P, P, i32], ctypes.c_int),
         "mggcn_graph_free": ([P], None),
         "mggcn_part_free": ([P], None),
         "mggcn_model_free": ([P], None),
@@ -305,10 +309,35 @@ def mggcn_get_profile(m, reset=False):
     return {c: (ms[i], n[i]) for i, c in enumerate(PROFILE_CLASSES)}
 
 
+def mggcn_get_timeline(m, reset=True):
+    """Per-op records since the last reset (MGGCN_F_TIMELINE): a list of dicts
+    {cls, spmm, stage, rank, stream, t0, t1} (device ms from the first record)."""
+    cnt = ctypes.c_int64()
+    _check(_lib.mggcn_get_timeline(m, 0, None, None, ctypes.byref(cnt), 0))
+    n = cnt.value
+    meta = np.zeros((max(n, 1), 5), dtype=np.int32)
+    t = np.zeros((max(n, 1), 2), dtype=np.float64)
+    _check(_lib.mggcn_get_timeline(m, n, _ptr(meta), _ptr(t), ctypes.byref(cnt), 1 if reset else 0))
+    return [dict(cls=PROFILE_CLASSES[meta[i, 0]], spmm=int(meta[i, 1]), stage=int(meta[i, 2]), rank=int(meta[i, 3]),
+                 stream=int(meta[i, 4]), t0=float(t[i, 0]), t1=float(t[i, 1])) for i in range(n)]
+
+
 def mggcn_epoch_work(m):
     vals = [ctypes.c_double() for _ in range(4)]
     _check(_lib.mggcn_epoch_work(m, *[ctypes.byref(v) for v in vals]))
     return dict(zip(("spmm_bytes", "spmm_gather_bytes", "gemm_flops", "bcast_bytes"), [v.value for v in vals]))
+
+
+WORK_DETAIL_KEYS = ("spmm_bytes", "spmm_struct_bytes", "spmm_gather_bytes", "spmm_gather_raw_bytes", "gemm_flops",
+                    "gemm_bytes", "bcast_bytes", "ce_bytes", "spmm_stages")
+
+
+def mggcn_epoch_work_detail(m):
+    out = (ctypes.c_double * 16)()
+    k = _lib.mggcn_epoch_work_detail(m, out, 16)
+    if k < 0:
+        _check(k)
+    return {name: out[i] for i, name in enumerate(WORK_DETAIL_KEYS[:k])}
 
 
 def mggcn_kernel_launch_count() -> int:

@@ -208,6 +208,10 @@ struct mggcn_model_s {
     int64_t* ntrain = nullptr;
     cudaStream_t cs = nullptr, ms = nullptr;
     cudaEvent_t ev_begin = nullptr, ev_comm_end = nullptr, ev_tmp = nullptr, ev_wg = nullptr, ev_comm_done = nullptr;
+    // without MGGCN_F_OVERLAP: recorded on the compute stream after every SpMM stage launch
+    // (the local stage included); broadcast / pull k waits on it, so it starts only after
+    // the previous stage finished (strict bcast -> stage -> bcast alternation)
+    cudaEvent_t ev_stage = nullptr;
     ncclComm_t comm = nullptr;
     ncclComm_t comm_bc = nullptr, comm_pair = nullptr;   // 1.5D: replica group, row-block pair
     int state = ST_READY;
@@ -217,10 +221,16 @@ struct mggcn_model_s {
     // profiling
     std::vector<std::tuple<int, cudaEvent_t, cudaEvent_t>> prof_recs;
     std::vector<cudaEvent_t> prof_pool;
+    // per-stage timeline (MGGCN_F_TIMELINE): {class, spmm index, stage, local rank, stream}, events
+    struct TlRec { int32_t meta[5]; cudaEvent_t a, b; };
+    std::vector<TlRec> tl_recs;
+    int32_t tl_spmm = -1, tl_stage = -1, tl_rank = -1;   // context of the next ProfScope
+    int32_t tl_nspmm = 0;                                  // SpMMs issued since the last forward
     double prof_ms[PC_N] = {0};
     int64_t prof_n[PC_N] = {0};
     // epoch work
     double w_spmm_bytes = 0, w_gather_bytes = 0, w_gemm_flops = 0, w_bcast_bytes = 0;
+    double w_spmm_struct_bytes = 0, w_gemm_bytes = 0, w_ce_bytes = 0, w_gather_raw_bytes = 0, w_stages = 0;
     // X staging plan bookkeeping
     int layer_ids[64];
     bool t0_valid = false;          // MGGCN_F_CACHE_L0: T0 = Â'^T X computed
@@ -308,11 +318,23 @@ struct ProfScope {
     mggcn_model_s* m;
     int cls;
     cudaStream_t s;
-    cudaEvent_t a = nullptr;
+    cudaEvent_t a = nullptr;     // MGGCN_F_PROFILE pair (consumed by mggcn_get_profile)
+    cudaEvent_t ta = nullptr;    // MGGCN_F_TIMELINE pair (consumed by mggcn_get_timeline)
+    int32_t meta[5];
     ProfScope(mggcn_model_s* m_, int c, cudaStream_t s_) : m(m_), cls(c), s(s_) {
-        if ((m->flags & MGGCN_F_PROFILE) && !m->capturing) {   // a captured epoch is timed as a whole
+        if (m->capturing) return;   // a captured epoch is timed as a whole
+        if (m->flags & MGGCN_F_PROFILE) {
             a = prof_event(m);
             cudaEventRecord(a, s);
+        }
+        if (m->flags & MGGCN_F_TIMELINE) {
+            ta = prof_event(m);
+            cudaEventRecord(ta, s);
+            meta[0] = c;
+            meta[1] = m->tl_spmm;
+            meta[2] = m->tl_stage;
+            meta[3] = m->tl_rank;
+            meta[4] = s == m->cs ? 0 : 1;
         }
     }
     ~ProfScope() {
@@ -320,6 +342,15 @@ struct ProfScope {
             cudaEvent_t b = prof_event(m);
             cudaEventRecord(b, s);
             m->prof_recs.emplace_back(cls, a, b);
+        }
+        if (ta) {
+            cudaEvent_t tb = prof_event(m);
+            cudaEventRecord(tb, s);
+            mggcn_model_s::TlRec t;
+            for (int i = 0; i < 5; ++i) t.meta[i] = meta[i];
+            t.a = ta;
+            t.b = tb;
+            m->tl_recs.push_back(t);
         }
     }
 };
@@ -676,16 +707,35 @@ int inject_delay(mggcn_model_s* m, cudaStream_t s) {
     return MGGCN_OK;
 }
 
-int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags) {
+int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
     const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
     float* out = job.dst(m, r, job.ctx);
+    m->tl_stage = tl_k;
+    m->tl_rank = (int32_t)(&r - &m->ranks[0]);
     ProfScope ps(m, PC_SPMM, m->cs);
     // NCCL collectives run as kernels on the comm stream: let them in while the SpMM runs
     if ((m->comm || m->solo) && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
     CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
                    (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
     return MGGCN_OK;
+}
+
+// Without MGGCN_F_OVERLAP the exchange of block k may start only after the
+// previous SpMM stage (the local stage for k = 0) finished: mark_stage() after
+// every stage launch, serial_wait() before every broadcast / pull.
+int mark_stage(mggcn_model_s* m) {
+    if (!(m->flags & MGGCN_F_OVERLAP)) CK(cudaEventRecord(m->ev_stage, m->cs));
+    return MGGCN_OK;
+}
+int serial_wait(mggcn_model_s* m) {
+    if (!(m->flags & MGGCN_F_OVERLAP)) CK(cudaStreamWaitEvent(m->ms, m->ev_stage, 0));
+    return MGGCN_OK;
+}
+// timeline context of a broadcast / pull ProfScope
+void tl_comm(mggcn_model_s* m, int k, int rank_idx) {
+    m->tl_stage = k;
+    m->tl_rank = rank_idx;
 }
 
 int remote_index(int q, int self) { return q < self ? q : q - 1; }
@@ -703,10 +753,13 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
     CK(cudaEventRecord(m->ev_begin, m->cs));            // my source produced; BC slots free
     RC(ipc_signal(m, m->cs, 0, seq));                   // peers may pull my block
     CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
-    if (r.rows > 0) RC(launch_stage(m, r, job, me, mysrc, 0));
+    if (r.rows > 0) RC(launch_stage(m, r, job, me, mysrc, 0, -1));
+    RC(mark_stage(m));
     for (int st = 1; st < P; ++st) {
         const int q = (me + st) % P, k = st - 1, slot = k & 1;
         {
+            RC(serial_wait(m));
+            tl_comm(m, q, 0);
             ProfScope ps(m, PC_BCAST, m->ms);
             RC(inject_delay(m, m->ms));
             if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
@@ -716,8 +769,9 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
             CK(cudaEventRecord(r.ev_bc[slot], m->ms));
         }
         CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
-        if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], SPMM_ACCUM | (st == P - 1 ? SPMM_LAST : 0)));
+        if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], SPMM_ACCUM | (st == P - 1 ? SPMM_LAST : 0), q));
         CK(cudaEventRecord(r.ev_free[slot], m->cs));
+        RC(mark_stage(m));
     }
     RC(ipc_signal(m, m->ms, 1, seq));                   // I have read every peer's block
     CK(cudaEventRecord(m->ev_comm_end, m->ms));
@@ -744,19 +798,21 @@ int remote_index_15d(const mggcn_model_s* m, int q, const Rank& r) {
 int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
     const int P = m->P, c = m->c;
     const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
-    const bool overlap = (m->flags & MGGCN_F_OVERLAP) != 0;
     CK(cudaEventRecord(m->ev_begin, m->cs));
     CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
     std::vector<char> started(m->ranks.size(), 0);
     for (size_t k = 0; k < m->ranks.size(); ++k) {      // own block first
         Rank& r = m->ranks[k];
         if (!in_set(m, r.rep, r.rank)) continue;
-        if (r.rows > 0) RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), 0));
+        if (r.rows > 0) RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), 0, -1));
         started[k] = 1;
     }
+    RC(mark_stage(m));
     for (int q = 0; q < P; ++q) {
         const int rq = q % c;                            // the replica group that needs block q
         {
+            RC(serial_wait(m));
+            tl_comm(m, q, -1);
             ProfScope ps(m, PC_BCAST, m->ms);
             RC(inject_delay(m, m->ms));
             if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
@@ -768,7 +824,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
                         if (!nob && count) NK(ncclBroadcast(s, s, count, ncclFloat32, q, m->comm_bc, m->ms));
                     } else {
                         const int k = remote_index_15d(m, q, r), slot = k & 1;
-                        if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                        if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
                         if (!nob && count)
                             NK(ncclBroadcast(r.BC[slot], r.BC[slot], count, ncclFloat32, q, m->comm_bc, m->ms));
                         CK(cudaEventRecord(r.ev_bc[slot], m->ms));
@@ -780,7 +836,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
                 for (auto& r : m->ranks) {
                     if (r.rep != rq || r.rank == q) continue;
                     const int k = remote_index_15d(m, q, r), slot = k & 1;
-                    if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
                     if (!nob && bytes)
                         CK(cudaMemcpyAsync(r.BC[slot], job.src(m, root, job.ctx), bytes, cudaMemcpyDeviceToDevice,
                                            m->ms));
@@ -793,10 +849,11 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
             if (r.rep != rq || r.rank == q) continue;
             const int k = remote_index_15d(m, q, r), slot = k & 1;
             CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
-            if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], started[i] ? SPMM_ACCUM : 0));
+            if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], started[i] ? SPMM_ACCUM : 0, q));
             started[i] = 1;
             CK(cudaEventRecord(r.ev_free[slot], m->cs));
         }
+        RC(mark_stage(m));
     }
     CK(cudaEventRecord(m->ev_comm_end, m->ms));
     CK(cudaStreamWaitEvent(m->cs, m->ev_comm_end, 0));
@@ -829,11 +886,10 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
     return MGGCN_OK;
 }
 
-int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
+int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
     if (m->c > 1) return staged_spmm_15d(m, job);
     const int P = m->P;
     const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
-    const bool overlap = (m->flags & MGGCN_F_OVERLAP) != 0;
     if (P > 1) {
         CK(cudaEventRecord(m->ev_begin, m->cs));
         CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
@@ -843,12 +899,15 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
     for (auto& r : m->ranks) {
         if (r.rows == 0) continue;
         const int last = (P == 1) ? SPMM_LAST : 0;
-        RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), last));
+        RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), last, -1));
     }
     if (P == 1) return MGGCN_OK;
+    RC(mark_stage(m));
     for (int q = 0; q < P; ++q) {
         // ---- broadcast of block q (comm stream)
         {
+            RC(serial_wait(m));
+            tl_comm(m, q, -1);
             ProfScope ps(m, PC_BCAST, m->ms);
             RC(inject_delay(m, m->ms));
             if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
@@ -859,7 +918,7 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
                     if (!nob && count) NK(ncclBroadcast(s, s, count, ncclFloat32, q, m->comm, m->ms));
                 } else {
                     const int k = remote_index(q, r.rank), slot = k & 1;
-                    if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
                     if (!nob && count) NK(ncclBroadcast(r.BC[slot], r.BC[slot], count, ncclFloat32, q, m->comm, m->ms));
                     CK(cudaEventRecord(r.ev_bc[slot], m->ms));
                 }
@@ -869,7 +928,7 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
                 for (auto& r : m->ranks) {
                     if (r.rank == q) continue;
                     const int k = remote_index(q, r.rank), slot = k & 1;
-                    if (k >= 2 || !overlap) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
                     if (!nob && bytes)
                         CK(cudaMemcpyAsync(r.BC[slot], job.src(m, root, job.ctx), bytes, cudaMemcpyDeviceToDevice,
                                            m->ms));
@@ -884,13 +943,21 @@ int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
             CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
             const int last_q = (r.rank == P - 1) ? P - 2 : P - 1;
             const int flags = SPMM_ACCUM | (q == last_q ? SPMM_LAST : 0);
-            if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], flags));
+            if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], flags, q));
             CK(cudaEventRecord(r.ev_free[slot], m->cs));
         }
+        RC(mark_stage(m));
     }
     CK(cudaEventRecord(m->ev_comm_end, m->ms));
     CK(cudaStreamWaitEvent(m->cs, m->ev_comm_end, 0));
     return MGGCN_OK;
+}
+
+int staged_spmm(mggcn_model_s* m, const SpmmJob& job) {
+    m->tl_spmm = m->tl_nspmm++;
+    const int rc = staged_spmm_impl(m, job);
+    m->tl_spmm = m->tl_stage = m->tl_rank = -1;
+    return rc;
 }
 
 float* src_HWB(mggcn_model_s*, Rank& r, const void*) { return r.HWB; }
@@ -1085,15 +1152,24 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         return MGGCN_EUNSUPPORTED;
     }
     // epoch work model, per this model's rows
+    //   spmm_bytes   compulsory: 4 B per non-zero of the tile as partitioned (pattern-only; +4 B
+    //                weighted) + rowptr + each gathered row once + each output row once
+    //   struct bytes what the kernel's tile structure holds (coalesced entries: index +
+    //                multiplicity value)
     auto spmm_work = [&](int dir, int64_t width) {
         for (auto& r : m->ranks)
             for (int j = 0; j < m->P; ++j) {
                 if (!in_set(m, r.rep, j)) continue;      // 1.5D: the other replica's stages
                 const HostTile& t = dir == 0 ? r.tF(j) : r.tB(j);
+                const HostTile& raw = dir == 0 ? r.part->F[j] : r.part->tileB(j);
                 const double nnz = (double)t.rowptr.back();
-                m->w_spmm_bytes += nnz * (t.val.empty() ? 4.0 : 8.0) + 4.0 * (double)(t.nrows + 1) +
-                                   4.0 * (double)width * (double)(t.ncols + t.nrows);
+                const double nnz_raw = (double)raw.rowptr.back();
+                const double rows_io = 4.0 * (double)width * (double)(t.ncols + t.nrows) + 4.0 * (double)(t.nrows + 1);
+                m->w_spmm_bytes += nnz_raw * (raw.val.empty() ? 4.0 : 8.0) + rows_io;
+                m->w_spmm_struct_bytes += nnz * (t.val.empty() ? 4.0 : 8.0) + rows_io;
                 m->w_gather_bytes += nnz * 4.0 * (double)width;
+                m->w_gather_raw_bytes += nnz_raw * 4.0 * (double)width;
+                m->w_stages += 1.0;
                 if (j != r.rank) m->w_bcast_bytes += 4.0 * (double)width * (double)t.ncols;
             }
     };
@@ -1104,11 +1180,19 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         const int64_t w = m->order[l] == G_ORDER ? m->d[l + 1] : m->d[l];
         if (!(l == 0 && (flags & MGGCN_F_CACHE_L0))) spmm_work(0, w);   // steady state: T0 cached
         const double gf = 2.0 * (double)root_rows * (double)m->d[l] * (double)m->d[l + 1];
+        const double dl = (double)m->d[l], dn = (double)m->d[l + 1];
+        const double rows_fwd = m->order[l] == G_ORDER ? (double)root_rows : (double)m->n_local;
         m->w_gemm_flops += m->order[l] == G_ORDER ? gf : gf * (double)m->n_local / (double)std::max<int64_t>(root_rows, 1);
+        m->w_gemm_bytes += 4.0 * (rows_fwd * (dl + dn) + dl * dn);            // F1: H W (or T0 W)
         m->w_gemm_flops += gf;                       // W_G
-        if (l > 0) m->w_gemm_flops += gf;            // H_G
+        m->w_gemm_bytes += 4.0 * ((double)root_rows * (dl + dn) + dl * dn);   // B2: H^T HW_G
+        if (l > 0) {
+            m->w_gemm_flops += gf;                   // H_G
+            m->w_gemm_bytes += 4.0 * ((double)root_rows * (dl + 2.0 * dl + dn) + dl * dn);   // B3 + old-C mask
+        }
         if (m->order[l] == G_ORDER) spmm_work(1, m->d[l + 1]);   // backward SpMM (Eq. 9)
     }
+    m->w_ce_bytes = 2.0 * 4.0 * (double)root_rows * (double)m->d[L];
     return MGGCN_OK;
 }
 
@@ -1154,8 +1238,12 @@ static void destroy(mggcn_model_s* m) {
         }
     if (m->cp) cudaStreamSynchronize(m->cp);
     for (cudaEvent_t e : {m->ev_begin, m->ev_comm_end, m->ev_tmp, m->ev_wg, m->ev_comm_done, m->ev_pref, m->ev_xfree[0],
-                          m->ev_xfree[1]})
+                          m->ev_xfree[1], m->ev_stage})
         if (e) cudaEventDestroy(e);
+    for (auto& t : m->tl_recs) {
+        cudaEventDestroy(t.a);
+        cudaEventDestroy(t.b);
+    }
     if (m->cp) cudaStreamDestroy(m->cp);
     for (auto& rec : m->prof_recs) {
         cudaEventDestroy(std::get<1>(rec));
@@ -1237,7 +1325,7 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
         return fail(MGGCN_ECUDA);
     }
     for (cudaEvent_t* e : {&m->ev_begin, &m->ev_comm_end, &m->ev_tmp, &m->ev_wg, &m->ev_comm_done, &m->ev_pref,
-                           &m->ev_xfree[0], &m->ev_xfree[1]})
+                           &m->ev_xfree[0], &m->ev_xfree[1], &m->ev_stage})
         if (cudaEventCreateWithFlags(e, cudaEventDisableTiming) != cudaSuccess) {
             set_error("model_create: cudaEventCreate failed");
             return fail(MGGCN_ECUDA);
@@ -1465,6 +1553,7 @@ extern "C" int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, co
 static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int32_t* y, float* loss,
                         float* logits) {
     const int L = m->L;
+    m->tl_nspmm = 0;
     // inputs -> internal buffers (this is the e2e H2D when X is host memory).
     // X == NULL: use the buffer filled by mggcn_prefetch on the copy stream.
     const bool use_cache = (m->flags & MGGCN_F_CACHE_L0) && m->t0_valid;
@@ -1815,7 +1904,7 @@ extern "C" int mggcn_epoch_capture(mggcn_model m, const float* X_local, int64_t 
     // events recorded during the capture became graph edges; re-record them on the
     // (no longer capturing) compute stream so that eager calls may wait on them again
     for (cudaEvent_t e : {m->ev_begin, m->ev_comm_end, m->ev_tmp, m->ev_wg, m->ev_comm_done, m->ev_xfree[0],
-                          m->ev_xfree[1]})
+                          m->ev_xfree[1], m->ev_stage})
         if (e) cudaEventRecord(e, m->cs);
     for (auto& r : m->ranks)
         for (int k = 0; k < 2; ++k) {
@@ -1907,12 +1996,57 @@ extern "C" int mggcn_get_profile(mggcn_model m, double* ms, int64_t* launches, i
     return MGGCN_OK;
 }
 
+extern "C" int mggcn_get_timeline(mggcn_model m, int64_t cap, int32_t* meta, double* t_ms, int64_t* count,
+                                  int32_t reset) {
+    MODEL_GUARD(m);
+    if (cap < 0 || (cap > 0 && (!meta || !t_ms))) {
+        set_error("get_timeline: cap < 0 or NULL arrays");
+        return MGGCN_EINVAL;
+    }
+    if (cudaStreamSynchronize(m->cs) != cudaSuccess || cudaStreamSynchronize(m->ms) != cudaSuccess) {
+        set_error("get_timeline: stream sync failed");
+        return poison(m, MGGCN_ECUDA);
+    }
+    const int64_t n = (int64_t)m->tl_recs.size();
+    if (count) *count = n;
+    for (int64_t i = 0; i < n && i < cap; ++i) {
+        const auto& t = m->tl_recs[i];
+        for (int k = 0; k < 5; ++k) meta[5 * i + k] = t.meta[k];
+        float a = 0, b = 0;
+        cudaEventElapsedTime(&a, m->tl_recs[0].a, t.a);
+        cudaEventElapsedTime(&b, m->tl_recs[0].a, t.b);
+        t_ms[2 * i] = a;
+        t_ms[2 * i + 1] = b;
+    }
+    if (reset) {
+        for (auto& t : m->tl_recs) {
+            m->prof_pool.push_back(t.a);
+            m->prof_pool.push_back(t.b);
+        }
+        m->tl_recs.clear();
+    }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_epoch_work_detail(mggcn_model m, double* out, int32_t n) {
+    MODEL_GUARD(m);
+    if (!out || n < 0) {
+        set_error("epoch_work_detail: NULL out or n < 0");
+        return MGGCN_EINVAL;
+    }
+    const double v[] = {m->w_spmm_bytes, m->w_spmm_struct_bytes, m->w_gather_bytes, m->w_gather_raw_bytes,
+                        m->w_gemm_flops, m->w_gemm_bytes, m->w_bcast_bytes, m->w_ce_bytes, m->w_stages};
+    const int32_t k = (int32_t)(sizeof(v) / sizeof(v[0]));
+    for (int32_t i = 0; i < n && i < k; ++i) out[i] = v[i];
+    return k;
+}
+
 extern "C" int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* gather, double* flops, double* bcast) {
     if (!m) {
         set_error("NULL model");
         return MGGCN_EINVAL;
     }
-    if (spmm_bytes) *spmm_bytes = m->w_spmm_bytes;
+    if (spmm_bytes) *spmm_bytes = m->w_spmm_bytes;   // SURVEY §8(d) compulsory (raw pattern)
     if (gather) *gather = m->w_gather_bytes;
     if (flops) *flops = m->w_gemm_flops;
     if (bcast) *bcast = m->w_bcast_bytes;

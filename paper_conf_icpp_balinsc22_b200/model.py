@@ -8,6 +8,7 @@ from __future__ import annotations
 import numpy as np
 
 from . import (MGGCN_F_IPC, MGGCN_F_OVERLAP, MGGCN_F_REPL2, MGGCN_F_REPLICA1, mggcn_backward, mggcn_epoch_capture,
+               mggcn_epoch_work_detail,
                mggcn_epoch_replay, mggcn_epoch_work, mggcn_forward, mggcn_get_adam, mggcn_get_grad, mggcn_get_loss, mggcn_get_profile, mggcn_get_weights, mggcn_graph_free,
                mggcn_ipc_connect, mggcn_ipc_export, mggcn_load_csr, mggcn_model_create, mggcn_model_free,
                mggcn_part_free, mggcn_part_info, mggcn_partition, mggcn_prefetch, mggcn_set_adam,
@@ -168,6 +169,9 @@ class GCN:
 
     def epoch_work(self):
         return mggcn_epoch_work(self.m)
+
+    def epoch_work_detail(self):
+        return mggcn_epoch_work_detail(self.m)
 
     def synchronize(self):
         self.cs.synchronize()

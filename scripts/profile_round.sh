@@ -1,6 +1,7 @@
 # Round profile evidence: launch list of one epoch + ncu --set full of the top kernels.
 # usage: bash scripts/profile_round.sh <tag> [workload]
 TAG=$1; WL=${2:-reddit}
+sha256sum paper_conf_icpp_balinsc22_b200/libmggcn.so > gpurun_out/${TAG}_so.sha
 ARGS="--workload $WL --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --no-cache-l0"
 timeout -s KILL 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
    --log-file gpurun_out/${TAG}_launches.csv python bench.py $ARGS > gpurun_out/${TAG}_launch.log 2>&1

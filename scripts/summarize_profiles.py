@@ -130,7 +130,13 @@ def main():
         nwin = int(os.environ.get("WIDE_WINDOWS", "2" if wl == "reddit" else "1"))
         wide, narrow = nwin * traffic["spmm_wide"], traffic.get("spmm_narrow", traffic["spmm_wide"])
         avg = (4 * wide + 2 * narrow) / 6 if wl == "reddit" else wide
+        import hashlib
+        so = os.path.join(ROOT, "paper_conf_icpp_balinsc22_b200", "libmggcn.so")
+        so_sha = open(os.path.join(OUT, f"{tag}_so.sha")).read().split()[0][:16] \
+            if os.path.exists(os.path.join(OUT, f"{tag}_so.sha")) else hashlib.sha256(open(so, "rb").read()).hexdigest()[:16]
+        git_sha = subprocess.run(["git", "-C", ROOT, "rev-parse", "HEAD"], capture_output=True, text=True).stdout.strip()
         json.dump({"workload": wl, "P": 1, "tag": tag, "dram_bytes_per_launch": avg,
+                   "so_sha256": so_sha, "git_sha": git_sha,
                    "dram_bytes_wide_launch": wide, "dram_bytes_narrow_launch": narrow,
                    "wide_windows": nwin,
                    "how": "ncu --set full, dram__bytes_read.sum + dram__bytes_write.sum, one launch each "

@@ -418,3 +418,49 @@ def test_delay_injection_keeps_results_bitwise(mg, P, replicas):
         mg.mggcn_debug_comm_delay(gm.m, 0, 20000)
     assert e.value.code == mg.MGGCN_EINVAL
     gm.close()
+
+
+def _stage_overlaps(tl):
+    """Pairs (comm record, SpMM stage record) of the same SpMM whose device intervals intersect."""
+    eps = 2e-3   # ms: event timestamp resolution
+    comm = [r for r in tl if r["stream"] == 1 and r["cls"] == "bcast" and r["spmm"] >= 0]
+    comp = [r for r in tl if r["stream"] == 0 and r["cls"] == "spmm" and r["spmm"] >= 0]
+    return [(a, b) for a in comm for b in comp
+            if a["spmm"] == b["spmm"] and a["t0"] < b["t1"] - eps and b["t0"] < a["t1"] - eps]
+
+
+@pytest.mark.parametrize("P,replicas", [(4, 1), (4, 2)])
+def test_overlap_flag_orders_exchange_and_stages(mg, P, replicas):
+    """MGGCN_F_OVERLAP semantics (include/mggcn.h; Fig. 8), checked on the
+    per-stage timeline rather than on the numbers: without the flag every broadcast starts only
+    after the previous SpMM stage finished (no comm interval intersects a stage interval of the
+    same SpMM); with it, broadcast k+1 runs while stage k computes.  Delay injection (spins of up
+    to 300 us on both streams) makes both orders observable; results stay bitwise equal."""
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    n, m = 3000, 120000
+    rp, col = gen.rmat_csr(n, m, 81)
+    dims = (32, 64, 8)
+    X = gen.features(n, dims[0], 82)
+    y = gen.labels(n, dims[-1], 83)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 84 + l) for l in range(2)]
+    res = {}
+    for overlap in (False, True):
+        flags = mg.MGGCN_F_TIMELINE | (mg.MGGCN_F_OVERLAP if overlap else 0)
+        gm = GCN(n, rp, col, None, dims, P=P, perm_seed=85, flags=flags, loopback=True, replicas=replicas)
+        mg.mggcn_debug_comm_delay(gm.m, 5, 300)
+        gm.set_weights(Ws)
+        Xd = torch.from_numpy(gm.permute_rows(X)).cuda()
+        yd = torch.from_numpy(gm.permute_rows(y)).cuda()
+        loss = gm.forward(Xd, yd, want_loss=True)
+        gm.backward()
+        tl = mg.mggcn_get_timeline(gm.m)
+        res[overlap] = (loss, gm.grads(), _stage_overlaps(tl), tl)
+        gm.close()
+    tl_off = res[False][3]
+    assert any(r["stream"] == 1 and r["cls"] == "bcast" for r in tl_off)
+    assert any(r["stream"] == 0 and r["cls"] == "spmm" and r["stage"] >= 0 for r in tl_off)
+    assert res[False][2] == [], res[False][2][:3]
+    assert len(res[True][2]) > 0
+    assert res[False][0] == res[True][0]
+    for a, b in zip(res[False][1], res[True][1]):
+        assert np.array_equal(a, b)

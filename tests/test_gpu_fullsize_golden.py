@@ -1,0 +1,132 @@
+"""End-to-end parity of ONE WHOLE EPOCH at BASELINE.json's full sizes
+(north_star: "within max relative error 1e-3 ... on logits, loss and weight
+gradients after one epoch, on the same synthetic inputs"; SURVEY.md §8(c)
+"GPU-vs-oracle acceptance").
+
+The expected values are tests/golden/fullsize_<cfg>.npz, written by
+scripts/make_fullsize_golden.py, which calls ONLY oracle/ and gen/: one plain
+unpartitioned oracle epoch (fp32 storage, fp64 accumulate, single core) on the
+seeded inputs.  Nothing here feeds a GPU result into the oracle: the GPU runs
+the whole epoch on its own (forward over all layers with the P-stage SpMM,
+softmax-CE, backward, W_G reduction, Adam), in bench.py's launch
+configuration, and is compared element by element with the oracle's:
+  logits    on the golden's >= 8192 sampled rows (permuted ids, incl. the
+            largest hub and zero-in-degree vertices)   rel <= 1e-3
+  loss                                                  rel <= 1e-3
+  W_G,l     every element, every layer                  rel <= 1e-3
+  Adam m, v after the step, every element               rel <= 1e-3
+  W after the step where |g| > 1e-3 max|g| (the first Adam
+            step is ~ lr sign(g))                       abs <= 1e-5
+rel(x, r) = max|x - r| / max|r|.  Partitioning is an exact re-organisation
+(§8(c)), so the same golden serves P = 1 and the loopback P = 8 split of
+north_star's 8-GPU target.  The inputs' fingerprints are checked first, so a
+generator drift fails loudly instead of comparing different problems."""
+import hashlib
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import gen
+
+pytestmark = pytest.mark.gpu
+REL_TOL = 1e-3
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+
+
+def rel(x, r):
+    r = np.asarray(r, np.float64)
+    return float(np.abs(np.asarray(x, np.float64) - r).max() / max(np.abs(r).max(), 1e-30))
+
+
+def sha(a):
+    return hashlib.sha256(np.ascontiguousarray(a).tobytes()).hexdigest()
+
+
+def load_golden(name):
+    path = os.path.join(GOLDEN, f"fullsize_{name}.npz")
+    z = np.load(path, allow_pickle=False)
+    return {k: z[k] for k in z.files}, json.loads(str(z["meta"]))
+
+
+def check_inputs(meta, rp, col, X, y, Ws):
+    assert sha(rp) == meta["sha_rowptr"] and sha(col) == meta["sha_col"], "graph generator drifted"
+    assert sha(X) == meta["sha_X"] and sha(y) == meta["sha_y"], "feature / label generator drifted"
+    assert [sha(W) for W in Ws] == meta["sha_W"], "weight generator drifted"
+
+
+def compare_epoch(g, L, loss, WG, adam, Wn, logits_rows=None):
+    out = {"loss": abs(loss - float(g["loss"])) / abs(float(g["loss"]))}
+    if logits_rows is not None:
+        out["logits"] = rel(logits_rows, g["logits_rows"])
+    for l in range(L):
+        out[f"WG{l}"] = rel(WG[l], g[f"WG{l}"])
+        mo, ve, t = adam[l]
+        assert t == 1
+        out[f"m{l}"] = rel(mo, g[f"m{l}"])
+        out[f"v{l}"] = rel(ve, g[f"v{l}"])
+        gg = g[f"WG{l}"]
+        mask = np.abs(gg) > 1e-3 * np.abs(gg).max()
+        out[f"W{l}_abs"] = float(np.abs(Wn[l][mask].astype(np.float64) - g[f"W{l}"][mask]).max())
+    print(json.dumps(out))
+    for k, v in out.items():
+        assert v <= (1e-5 if k.endswith("_abs") else REL_TOL), (k, v, out)
+    return out
+
+
+@pytest.mark.parametrize("name,P", [("reddit", 1), ("reddit", 8), ("proteins", 1), ("products", 1)])
+def test_fullsize_epoch_matches_oracle_golden(name, P):
+    """Eager epoch (the path bench.py's profile loop times), P = 1 or loopback P-stage."""
+    import paper_conf_icpp_balinsc22_b200 as mg
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    assert torch.cuda.is_available()
+    g, meta = load_golden(name)
+    w = gen.WORKLOADS[name]
+    L = len(w.dims) - 1
+    rp, col, X, y, Ws = gen.make_inputs(w)
+    check_inputs(meta, rp, col, X, y, Ws)
+    gm = GCN(w.n, rp, col, None, w.dims, P=P, perm_seed=w.perm_seed,
+             flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE, loopback=P > 1)
+    try:
+        assert sha(np.asarray(gm.perm, np.int64)) == meta["sha_perm"]
+        gm.set_weights(Ws)
+        Xp, yp = gm.permute_rows(X), gm.permute_rows(y)
+        del X
+        Xd, yd = gm.device_inputs(Xp), torch.from_numpy(yp).cuda()
+        logits = torch.empty((w.n, w.dims[-1]), dtype=torch.float32, device="cuda")
+        loss = gm.forward(Xd, yd, want_loss=True, logits=logits)
+        rows = torch.from_numpy(g["rows"]).cuda()
+        lrows = logits.index_select(0, rows).cpu().numpy()
+        gm.backward()
+        WG = gm.grads()
+        gm.step(lr=0.01)
+        compare_epoch(g, L, loss, WG, [gm.adam_state(l) for l in range(L)], gm.get_weights(), lrows)
+    finally:
+        gm.close()
+
+
+@pytest.mark.parametrize("name", ["reddit", "products"])
+def test_fullsize_captured_epoch_matches_oracle_golden(name):
+    """The headline path of bench.py (N = 1): one replay of the captured epoch
+    (mggcn_epoch_capture / mggcn_epoch_replay) from fresh weights."""
+    import paper_conf_icpp_balinsc22_b200 as mg
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    g, meta = load_golden(name)
+    w = gen.WORKLOADS[name]
+    L = len(w.dims) - 1
+    rp, col, X, y, Ws = gen.make_inputs(w)
+    check_inputs(meta, rp, col, X, y, Ws)
+    gm = GCN(w.n, rp, col, None, w.dims, P=1, perm_seed=w.perm_seed, flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE)
+    try:
+        gm.set_weights(Ws)
+        Xd, yd = gm.device_inputs(gm.permute_rows(X)), torch.from_numpy(gm.permute_rows(y)).cuda()
+        del X
+        gm.capture_epoch(Xd, yd, lr=0.01)
+        gm.replay_epoch(1)
+        gm.synchronize()
+        compare_epoch(g, L, gm.loss(), gm.grads(), [gm.adam_state(l) for l in range(L)], gm.get_weights())
+    finally:
+        gm.close()
+

@@ -21,11 +21,19 @@
  *    return of the calling thread.
  *  - host inputs are copied before the call returns; the caller may free them.
  *  - device memory is never allocated by the library outside the caller-owned
- *    workspace given to mggcn_model_create (the debug_* test entry points are
- *    the exception and say so).
+ *    workspace given to mggcn_model_create (the debug_* test entry points and
+ *    the 16-byte buffer of the NCCL start-up self-check are the exceptions).
  *  - all matrices are row-major fp32; W_l is d_l x d_{l+1} (so H·W is Eq. 5).
  *  - CUDA / NCCL errors poison a model: every later call on it returns the
  *    same code.
+ *  - multi-GPU models (NCCL or MGGCN_F_IPC): every host wait (forward with a
+ *    loss, the get_* getters, profile / timeline reads, mggcn_model_free)
+ *    polls ncclCommGetAsyncError and gives up after MGGCN_SYNC_TIMEOUT_S
+ *    seconds (environment, default 600): a failed collective or a peer that
+ *    never arrives returns MGGCN_ENCCL (communicators aborted) instead of
+ *    hanging; mggcn_step polls the async error without waiting.
+ *    mggcn_model_create verifies a fresh communicator with one all-reduce and
+ *    one broadcast of known values (ENCCL if they come back wrong).
  *  - a model is single-threaded.  Results are bitwise reproducible run to run
  *    for fixed inputs, P and seed (no floating-point atomics); they are NOT
  *    bitwise equal across different P.

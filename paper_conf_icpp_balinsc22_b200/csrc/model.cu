@@ -10,6 +10,8 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <chrono>
+#include <thread>
 #include <cmath>
 #include <cstring>
 #include <new>
@@ -216,6 +218,7 @@ struct mggcn_model_s {
     ncclComm_t comm_bc = nullptr, comm_pair = nullptr;   // 1.5D: replica group, row-block pair
     int state = ST_READY;
     int poisoned = 0;
+    bool hung = false;              // a bounded host wait timed out: streams may never drain
     int64_t t = 0;
     bool need_wg_wait = false;
     // profiling
@@ -1027,6 +1030,78 @@ static int poison(mggcn_model_s* m, int rc) {
     return rc;
 }
 
+// ------------------------------------------------- bounded host waits
+// Host sync points (getters, forward with a loss, profile / timeline reads,
+// model_free) of a model that talks to peers (NCCL or IPC) wait for a stream
+// while polling NCCL's asynchronous error state: a failed or never-completing
+// collective, or a peer that died, returns MGGCN_ENCCL (communicators
+// aborted, model poisoned) instead of hanging the caller.  The wait limit is
+// MGGCN_SYNC_TIMEOUT_S seconds (default 600).
+static double sync_timeout_s() {
+    static double t = -1;
+    if (t < 0) {
+        const char* e = getenv("MGGCN_SYNC_TIMEOUT_S");
+        t = e ? atof(e) : 600.0;
+        if (!(t > 0)) t = 600.0;
+    }
+    return t;
+}
+
+static void abort_comms(mggcn_model_s* m) {
+    for (ncclComm_t* c : {&m->comm_bc, &m->comm_pair, &m->comm})
+        if (*c) {
+            ncclCommAbort(*c);
+            *c = nullptr;
+        }
+}
+
+static int poll_comm_errors(mggcn_model_s* m) {
+    for (ncclComm_t c : {m->comm, m->comm_bc, m->comm_pair}) {
+        if (!c) continue;
+        ncclResult_t ae = ncclSuccess;
+        const ncclResult_t r = ncclCommGetAsyncError(c, &ae);
+        if (r != ncclSuccess || ae != ncclSuccess) {
+            set_error(std::string("NCCL async error: ") + ncclGetErrorString(r != ncclSuccess ? r : ae));
+            abort_comms(m);
+            m->hung = true;
+            return MGGCN_ENCCL;
+        }
+    }
+    return MGGCN_OK;
+}
+
+static int sync_stream(mggcn_model_s* m, cudaStream_t s) {
+    if (!m->comm && !m->ipc) {
+        CK(cudaStreamSynchronize(s));
+        return MGGCN_OK;
+    }
+    const auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+        const cudaError_t q = cudaStreamQuery(s);
+        if (q == cudaSuccess) break;
+        if (q != cudaErrorNotReady) {
+            set_error(std::string("CUDA error while waiting: ") + cudaGetErrorString(q));
+            return MGGCN_ECUDA;
+        }
+        RC(poll_comm_errors(m));
+        const double el = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+        if (el > sync_timeout_s()) {
+            set_error("communication timeout: a stream waited more than MGGCN_SYNC_TIMEOUT_S s for peers "
+                      "(collective or peer flag never completed)");
+            abort_comms(m);
+            m->hung = true;
+            return MGGCN_ENCCL;
+        }
+        std::this_thread::sleep_for(std::chrono::microseconds(50));
+    }
+    return poll_comm_errors(m);
+}
+
+static int sync_both(mggcn_model_s* m) {
+    RC(sync_stream(m, m->cs));
+    return sync_stream(m, m->ms);
+}
+
 #define MODEL_GUARD(m)                                              \
     do {                                                            \
         if (!(m)) {                                                 \
@@ -1229,8 +1304,13 @@ extern "C" int mggcn_nccl_unique_id(void* out128) {
 
 static void destroy(mggcn_model_s* m) {
     if (!m) return;
-    if (m->cs) cudaStreamSynchronize(m->cs);
-    if (m->ms) cudaStreamSynchronize(m->ms);
+    // bounded: a model whose peers are gone must still be freeable (its comms are aborted)
+    if (!m->hung && m->cs && m->ms && sync_both(m) != MGGCN_OK) m->hung = true;
+    if (m->hung) {
+        abort_comms(m);
+        delete m;   // streams / events / graph of a hung model are left to process teardown
+        return;
+    }
     for (auto& r : m->ranks)
         for (int s = 0; s < 2; ++s) {
             if (r.ev_bc[s]) cudaEventDestroy(r.ev_bc[s]);
@@ -1258,6 +1338,43 @@ static void destroy(mggcn_model_s* m) {
     for (void* p : m->ipc_opened)
         if (p) cudaIpcCloseMemHandle(p);
     delete m;
+}
+
+// Start-up check of a fresh NCCL communicator (and the 1.5D sub-communicators):
+// one all-reduce of (rank + 1) and one broadcast of a known value from rank 0,
+// verified on the host with a bounded wait, so a mis-wired job fails here with
+// MGGCN_ENCCL instead of hanging or corrupting the first epoch.
+static int nccl_selfcheck_one(mggcn_model_s* m, ncclComm_t c, float* buf, const char* what) {
+    int nranks = 0, me = 0;
+    NK(ncclCommCount(c, &nranks));
+    NK(ncclCommUserRank(c, &me));
+    const float init[2] = {(float)(me + 1), me == 0 ? 4242.0f : -1.0f};
+    CK(cudaMemcpyAsync(buf, init, sizeof(init), cudaMemcpyHostToDevice, m->ms));
+    NK(ncclGroupStart());
+    NK(ncclAllReduce(buf, buf, 1, ncclFloat32, ncclSum, c, m->ms));
+    NK(ncclBroadcast(buf + 1, buf + 1, 1, ncclFloat32, 0, c, m->ms));
+    NK(ncclGroupEnd());
+    float got[2] = {0, 0};
+    CK(cudaMemcpyAsync(got, buf, sizeof(got), cudaMemcpyDeviceToHost, m->ms));
+    RC(sync_stream(m, m->ms));
+    const float want = 0.5f * (float)nranks * (float)(nranks + 1);
+    if (got[0] != want || got[1] != 4242.0f) {
+        set_error(std::string("model_create: NCCL self-check failed on the ") + what + " communicator (all-reduce " +
+                  std::to_string(got[0]) + " != " + std::to_string(want) + " or broadcast " + std::to_string(got[1]) +
+                  " != 4242)");
+        return MGGCN_ENCCL;
+    }
+    return MGGCN_OK;
+}
+
+static int nccl_selfcheck(mggcn_model_s* m) {
+    float* buf = nullptr;
+    CK(cudaMalloc(&buf, 4 * sizeof(float)));
+    int rc = nccl_selfcheck_one(m, m->comm, buf, "world");
+    if (rc == MGGCN_OK && m->comm_bc) rc = nccl_selfcheck_one(m, m->comm_bc, buf, "replica-group");
+    if (rc == MGGCN_OK && m->comm_pair) rc = nccl_selfcheck_one(m, m->comm_pair, buf, "row-block-pair");
+    if (!m->hung) cudaFree(buf);
+    return rc;
 }
 
 extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32_t L, const int32_t* dims,
@@ -1362,6 +1479,8 @@ extern "C" int mggcn_model_create(const mggcn_part* parts, int32_t nlocal, int32
                 return fail(MGGCN_ENCCL);
             }
         }
+        rc = nccl_selfcheck(m);
+        if (rc != MGGCN_OK) return fail(rc);
     }
     if (cudaStreamSynchronize(m->cs) != cudaSuccess) {
         set_error(std::string("model_create: ") + cudaGetErrorString(cudaGetLastError()));
@@ -1470,7 +1589,7 @@ extern "C" int mggcn_set_weights(mggcn_model m, int32_t layer, const float* W) {
         RC(refresh_weight_splits(m));
         CK(cudaMemsetAsync(m->Mom, 0, sizeof(float) * m->wtotal, m->cs));
         CK(cudaMemsetAsync(m->Vel, 0, sizeof(float) * m->wtotal, m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     rc = body();
@@ -1484,7 +1603,7 @@ extern "C" int mggcn_get_weights(mggcn_model m, int32_t layer, float* W) {
     const int64_t din = m->d[layer], dout = m->d[layer + 1], ld = m->ld[layer + 1];
     auto body = [&]() -> int {
         CK(cudaMemcpy2DAsync(W, dout * 4, m->W + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost, m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     return poison(m, body());
@@ -1505,7 +1624,7 @@ extern "C" int mggcn_get_grad(mggcn_model m, int32_t layer, float* WG) {
     auto body = [&]() -> int {
         RC(wait_wg(m));
         CK(cudaMemcpy2DAsync(WG, dout * 4, m->WG + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost, m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     return poison(m, body());
@@ -1522,7 +1641,7 @@ extern "C" int mggcn_get_adam(mggcn_model m, int32_t layer, float* mom, float* v
         if (vel)
             CK(cudaMemcpy2DAsync(vel, dout * 4, m->Vel + m->woff[layer], ld * 4, dout * 4, din, cudaMemcpyDeviceToHost,
                                  m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     if (t) *t = m->t;
@@ -1542,7 +1661,7 @@ extern "C" int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, co
                              m->cs));
         CK(cudaMemcpy2DAsync(m->Vel + m->woff[layer], ld * 4, vel, dout * 4, dout * 4, din, cudaMemcpyHostToDevice,
                              m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     m->t = t;
@@ -1634,7 +1753,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
         int64_t nt = 0;
         CK(cudaMemcpyAsync(&s, m->loss_sum, 8, cudaMemcpyDeviceToHost, m->cs));
         CK(cudaMemcpyAsync(&nt, m->ntrain, 8, cudaMemcpyDeviceToHost, m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         *loss = (float)(s / (double)(nt > 0 ? nt : 1));
         if (m->comm) {
             ncclResult_t ae;
@@ -1709,7 +1828,7 @@ extern "C" int mggcn_get_loss(mggcn_model m, float* loss) {
     auto body = [&]() -> int {
         CK(cudaMemcpyAsync(&s, m->loss_sum, 8, cudaMemcpyDeviceToHost, m->cs));
         CK(cudaMemcpyAsync(&nt, m->ntrain, 8, cudaMemcpyDeviceToHost, m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     int rc = body();
@@ -1822,6 +1941,7 @@ static int step_impl(mggcn_model_s* m, float lr, float beta1, float beta2, float
 
 extern "C" int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps) {
     MODEL_GUARD(m);
+    if (int rc = poll_comm_errors(m)) return poison(m, rc);   // non-blocking
     if (m->state != ST_BWD) {
         set_error("step: needs a preceding backward");
         return MGGCN_ESTATE;
@@ -1972,10 +2092,7 @@ extern "C" int mggcn_epoch_replay(mggcn_model m, int32_t epochs) {
 // -------------------------------------------------------------- profiling
 extern "C" int mggcn_get_profile(mggcn_model m, double* ms, int64_t* launches, int32_t reset) {
     MODEL_GUARD(m);
-    if (cudaStreamSynchronize(m->cs) != cudaSuccess || cudaStreamSynchronize(m->ms) != cudaSuccess) {
-        set_error("get_profile: stream sync failed");
-        return poison(m, MGGCN_ECUDA);
-    }
+    if (int rc = sync_both(m)) return poison(m, rc);
     for (auto& rec : m->prof_recs) {
         float t = 0;
         cudaEventElapsedTime(&t, std::get<1>(rec), std::get<2>(rec));
@@ -2003,10 +2120,7 @@ extern "C" int mggcn_get_timeline(mggcn_model m, int64_t cap, int32_t* meta, dou
         set_error("get_timeline: cap < 0 or NULL arrays");
         return MGGCN_EINVAL;
     }
-    if (cudaStreamSynchronize(m->cs) != cudaSuccess || cudaStreamSynchronize(m->ms) != cudaSuccess) {
-        set_error("get_timeline: stream sync failed");
-        return poison(m, MGGCN_ECUDA);
-    }
+    if (int rc = sync_both(m)) return poison(m, rc);
     const int64_t n = (int64_t)m->tl_recs.size();
     if (count) *count = n;
     for (int64_t i = 0; i < n && i < cap; ++i) {
@@ -2079,7 +2193,7 @@ extern "C" int mggcn_debug_layer(mggcn_model m, int32_t layer, float* dst, int64
             if (r.rows)
                 CK(cudaMemcpy2DAsync(dst + r.row_off * ld, ld * 4, r.AHWB[layer],
                                      m->ld[layer + 1] * 4, w * 4, r.rows, cudaMemcpyDefault, m->cs));
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     return poison(m, body());
@@ -2138,7 +2252,7 @@ extern "C" int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int6
                 CK(cudaMemcpy2DAsync(out + r.row_off * ldo, ldo * 4, ctx.out[i], w * 4, width * 4, r.rows,
                                      cudaMemcpyDeviceToDevice, m->cs));
         }
-        CK(cudaStreamSynchronize(m->cs));
+        RC(sync_stream(m, m->cs));
         return MGGCN_OK;
     };
     int rc = body();

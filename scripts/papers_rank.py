@@ -33,6 +33,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=2)
     ap.add_argument("--workload", default="papers")
+    ap.add_argument("--timeline", action="store_true",
+                    help="also record one epoch with MGGCN_F_TIMELINE and report per-SpMM stage sums / spans / gaps")
     args = ap.parse_args()
 
     import numpy as np
@@ -60,6 +62,8 @@ def main():
     del rp, col
     print(f"[papers_rank] load_csr {t_load:.1f} s", flush=True)
     flags = mg.MGGCN_F_OVERLAP | mg.MGGCN_F_NO_BCAST | mg.MGGCN_F_PROFILE
+    if args.timeline:
+        flags |= mg.MGGCN_F_TIMELINE
     t0 = time.perf_counter()
     gm = GCN(w.n, None, None, None, w.dims, P=args.parts, rank=args.rank, perm_seed=w.perm_seed, flags=flags,
              graph=graph)
@@ -86,6 +90,32 @@ def main():
         epoch()
     gm.synchronize()
     gm.profile(reset=True)
+    tl_summary = None
+    if args.timeline:
+        mg.mggcn_get_timeline(gm.m, reset=True)
+        epoch()
+        gm.synchronize()
+        tl = mg.mggcn_get_timeline(gm.m, reset=True)
+        gm.profile(reset=True)
+        comp = [r for r in tl if r["stream"] == 0]
+        t_end = max(r["t1"] for r in comp)
+        per = {}
+        for r in comp:
+            if r["cls"] != "spmm" or r["spmm"] < 0:
+                continue
+            d = per.setdefault(r["spmm"], {"stages": 0, "busy_ms": 0.0, "t0": r["t0"], "t1": r["t1"]})
+            d["stages"] += 1
+            d["busy_ms"] += r["t1"] - r["t0"]
+            d["t0"] = min(d["t0"], r["t0"])
+            d["t1"] = max(d["t1"], r["t1"])
+        for d in per.values():
+            d["span_ms"] = d["t1"] - d["t0"]
+            d["gap_ms"] = d["span_ms"] - d["busy_ms"]
+        busy = sum(r["t1"] - r["t0"] for r in comp)
+        tl_summary = {"epoch_span_ms": t_end, "compute_busy_ms": busy, "compute_idle_ms": t_end - busy,
+                      "spmm": {k: {kk: round(vv, 4) for kk, vv in v.items() if kk not in ("t0", "t1")}
+                               for k, v in sorted(per.items())},
+                      "stage_ms": [round(r["t1"] - r["t0"], 4) for r in comp if r["cls"] == "spmm"]}
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(gm.cs)
     for _ in range(args.steps):
@@ -110,7 +140,7 @@ def main():
         "bcast_note": "broadcast bytes received per rank per epoch (library work model) / 900 GB/s NVLink; "
                       "the 8-GPU epoch is at least max(compute, this) with perfect overlap",
         "setup_s": {"generate": t_gen, "load_csr": t_load, "partition+model": t_part},
-        "steps": args.steps, "warmup": args.warmup,
+        "steps": args.steps, "warmup": args.warmup, "timeline": tl_summary,
         "gpu": torch.cuda.get_device_name(0),
     }
     print(json.dumps(out), flush=True)

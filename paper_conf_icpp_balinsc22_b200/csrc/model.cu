@@ -148,6 +148,38 @@ std::vector<int32_t> encode_hot_classes(const HostTile& ht) {
     return out;
 }
 
+// Stage groups: the tile of a group is the row-wise concatenation of the
+// group's S column tiles, tile t's local column c becoming t * stride + c
+// (stride = max_j n_j, the BC slot pitch in rows).  Entries of a row stay in
+// (block, column) order; values are kept if any tile has them.
+void merge_group_tiles(const std::vector<const HostTile*>& tiles, int64_t stride, HostTile& o) {
+    const int64_t S = (int64_t)tiles.size();
+    o.nrows = tiles[0]->nrows;
+    o.ncols = S * stride;
+    o.col0 = 0;
+    bool vals = false;
+    size_t nnz = 0;
+    for (const HostTile* t : tiles) {
+        vals = vals || !t->val.empty();
+        nnz += t->col.size();
+    }
+    o.rowptr.assign(o.nrows + 1, 0);
+    o.col.clear();
+    o.val.clear();
+    o.col.reserve(nnz);
+    if (vals) o.val.reserve(nnz);
+    for (int64_t r = 0; r < o.nrows; ++r) {
+        for (int64_t t = 0; t < S; ++t) {
+            const HostTile& h = *tiles[t];
+            for (int32_t e = h.rowptr[r]; e < h.rowptr[r + 1]; ++e) {
+                o.col.push_back((int32_t)(t * stride + h.col[e]));
+                if (vals) o.val.push_back(h.val.empty() ? 1.0f : h.val[e]);
+            }
+        }
+        o.rowptr[r + 1] = (int32_t)o.col.size();
+    }
+}
+
 struct Rank {
     const mggcn_part_s* part = nullptr;
     int rank = 0;
@@ -173,6 +205,15 @@ struct Rank {
     float* T0 = nullptr;
     float* HWB = nullptr;
     float* BC[2] = {nullptr, nullptr};
+    // stage groups (S > 1, see plan_groups): the remote blocks of one group are consumed by ONE
+    // launch over a merged tile whose column t * max_rows_j + c addresses local column c of the
+    // group's t-th block; the group's blocks land in consecutive BC slots packed at the SpMM's
+    // width (slot k at BCg + k * max_rows_j * width), 2S slots (two groups in flight)
+    float* BCg = nullptr;
+    std::vector<HostTile> gF, gB;    // merged tiles per group (host)
+    std::vector<HostItems> hgF, hgB;
+    std::vector<SpmmTile> GF, GB;    // device
+    std::vector<int32_t> order_cache;  // row order of the items (setup only)
     std::vector<float*> AHWB;
     float* spmm_partial = nullptr;
     double* ce_partial = nullptr;
@@ -201,6 +242,7 @@ struct mggcn_model_s {
     int64_t n_local = 0;            // rows owned by this model (sum over local ranks)
     int64_t max_rows_j = 0;
     int64_t bc_ld = 0, hw_ld = 0;
+    int grp_S = 1;                  // remote stages per launch (1 = one launch per stage, the paper's schedule)
     std::vector<Rank> ranks;
     float *W = nullptr, *Mom = nullptr, *Vel = nullptr, *WG = nullptr;
     // tf32 hi/lo copies of W for the tcgen05 row GEMMs (refreshed after every update):
@@ -304,6 +346,42 @@ inline bool in_set(const mggcn_model_s* m, int rep, int j) { return m->c == 1 ||
 // needs the block's GEMM products (HW, the input gradient) and contributes W_G, the loss and
 // |T|; the other replica only adds its partial SpMM stages (every rank is a root in 1D)
 inline bool is_root(const mggcn_model_s* m, const Rank& r) { return in_set(m, r.rep, r.rank); }
+
+// The k-th remote block (k = 0 .. P-2) a rank consumes: ascending j != rank for the
+// collective backends (broadcast order is global), rotated (rank + k + 1) mod P for the
+// IPC pulls (every GPU serves one reader per step).
+inline int remote_block(const mggcn_model_s* m, int rank, int k, bool ipc) {
+    if (ipc) return (rank + k + 1) % m->P;
+    return k < rank ? k : k + 1;
+}
+inline int n_groups(const mggcn_model_s* m) { return (m->P - 1 + m->grp_S - 1) / m->grp_S; }
+
+// Remote stages per launch (per-stage launches pay a row visit, an output
+// read-modify-write, a launch and a hub fix-up per stage; at P = 8 a Reddit-shaped rank's
+// stages are 40-100 us, so those fixed costs are a third of its SpMM time).  Default:
+// two remote groups per SpMM, ceil((P-1)/2) blocks each, both in flight (2S BC slots),
+// so group 1's blocks arrive while group 0 computes; capped so the 2S slots fit
+// MGGCN_BC_BUDGET_MB (default 16 GiB: Papers-shaped blocks of 14 GB keep S = 1).
+// MGGCN_STAGE_GROUP=S overrides (1 = the paper's one launch per stage).  1D only.
+int choose_group_size(const mggcn_model_s* m, uint32_t flags) {
+    if (m->P <= 2 || m->c > 1) return 1;
+    int S = (m->P - 1 + 1) / 2;
+    if (const char* e = getenv("MGGCN_STAGE_GROUP")) {
+        const int v = atoi(e);
+        if (v >= 1) S = v;
+    }
+    if (const char* h = getenv("MGGCN_SPMM_HOTCLS"))
+        if (atoi(h) != 0) S = 1;   // priority-class tiles keep per-stage launches
+    S = std::max(1, std::min(S, m->P - 1));
+    double budget = 16384.0;
+    if (const char* e = getenv("MGGCN_BC_BUDGET_MB")) budget = atof(e);
+    const double slot = (double)m->max_rows_j * (double)m->bc_ld * 4.0 / 1048576.0;
+    while (S > 1 && 2.0 * S * slot > budget) --S;
+    // merged column ids and the kernel's 32-bit float4 row offsets must not overflow
+    while (S > 1 && (double)S * (double)m->max_rows_j * (double)(m->bc_ld / 4) >= 4294967296.0) --S;
+    (void)flags;
+    return S;
+}
 
 // ---------------------------------------------------------------- profiling
 cudaEvent_t prof_event(mggcn_model_s* m) {
@@ -420,43 +498,61 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
         const int P = pt->P;
         r.F.assign(P, SpmmTile());
         r.B.assign(P, SpmmTile());
+        auto place = [&](const HostTile& ht, const HostItems& hi, SpmmTile& t, bool hot_ok) {
+            t.nrows = ht.nrows;
+            t.ncols = ht.ncols;
+            t.nnz = ht.rowptr.back();
+            t.n_items = (int64_t)hi.items.size();
+            t.n_items_nz = hi.n_nonempty;
+            t.split = hi.split;
+            t.n_splits = (int64_t)hi.splits.size();
+            t.n_slots = hi.nslots;
+            t.items = b.take<int4>(hi.items.size());
+            t.splits = b.take<int4>(hi.splits.size());
+            t.col = b.take<int32_t>(ht.col.size());
+            t.hot_enc = hot_ok && want_hot_classes(ht);
+            t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
+        };
         for (int j = 0; j < P; ++j) {
+            // with stage groups only the local tile is launched per stage (the remote ones
+            // live in the merged group tiles; mggcn_part_export_tile reads the host copies)
+            const bool on_dev = m->grp_S == 1 || j == r.rank;
             for (int dir = 0; dir < 2; ++dir) {
                 if (dir == 1 && pt->shared_fb) {
                     r.B[j] = r.F[j];
                     continue;
                 }
-                const HostTile& ht = dir == 0 ? r.tF(j) : r.tB(j);
-                const HostItems& hi = dir == 0 ? r.hF[j] : r.hB[j];
                 SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
-                t.nrows = ht.nrows;
-                t.ncols = ht.ncols;
-                t.nnz = ht.rowptr.back();
-                t.n_items = (int64_t)hi.items.size();
-                t.n_items_nz = hi.n_nonempty;
-                t.split = hi.split;
-                t.n_splits = (int64_t)hi.splits.size();
-                t.n_slots = hi.nslots;
-                t.items = b.take<int4>(hi.items.size());
-                t.splits = b.take<int4>(hi.splits.size());
-                t.col = b.take<int32_t>(ht.col.size());
-                t.hot_enc = want_hot_classes(ht);
-                t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
+                if (on_dev) place(dir == 0 ? r.tF(j) : r.tB(j), dir == 0 ? r.hF[j] : r.hB[j], t, true);
             }
+        }
+        const int NG = m->grp_S > 1 ? n_groups(m) : 0;
+        r.GF.assign(NG, SpmmTile());
+        r.GB.assign(NG, SpmmTile());
+        for (int g = 0; g < NG; ++g) {
+            place(r.gF[g], r.hgF[g], r.GF[g], false);
+            if (pt->shared_fb) r.GB[g] = r.GF[g];
+            else place(r.gB[g], r.hgB[g], r.GB[g], false);
         }
         r.inv_deg = b.take<float>(r.rows);
         for (int k = 0; k < 2; ++k) r.ybuf[k] = b.take<int32_t>(r.rows);
         r.Xs = r.Xbuf[0];
         r.y = r.ybuf[0];
         r.T0 = m->order[0] == S_ORDER ? b.take<float>(r.rows * m->ld[0]) : nullptr;
-        if (P > 1) {
+        if (P > 1 && m->grp_S == 1) {
             r.BC[0] = b.take<float>(m->max_rows_j * m->bc_ld);
             r.BC[1] = b.take<float>(m->max_rows_j * m->bc_ld);
+        } else if (P > 1) {
+            r.BCg = b.take<float>(2 * m->grp_S * m->max_rows_j * m->bc_ld);
         }
         int64_t slots = 0;
         for (int j = 0; j < P; ++j) {
             slots = std::max(slots, r.hF[j].nslots);
             if (!pt->shared_fb) slots = std::max(slots, r.hB[j].nslots);
+        }
+        for (int g = 0; g < NG; ++g) {
+            slots = std::max(slots, r.hgF[g].nslots);
+            if (!pt->shared_fb) slots = std::max(slots, r.hgB[g].nslots);
         }
         r.spmm_partial = b.take<float>(slots * std::min<int64_t>(m->bc_ld, 512));
         r.ce_partial = b.take<double>(kCeBlocks);
@@ -472,12 +568,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
 int upload_static(mggcn_model_s* m) {
     for (auto& r : m->ranks) {
         const mggcn_part_s* pt = r.part;
-        for (int j = 0; j < pt->P; ++j)
-            for (int dir = 0; dir < 2; ++dir) {
-                if (dir == 1 && pt->shared_fb) continue;
-                const HostTile& ht = dir == 0 ? r.tF(j) : r.tB(j);
-                const HostItems& hi = dir == 0 ? r.hF[j] : r.hB[j];
-                SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
+        auto upload = [&](const HostTile& ht, const HostItems& hi, SpmmTile& t) -> int {
                 if (!hi.items.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.items), hi.items.data(), sizeof(int4) * hi.items.size(),
                                        cudaMemcpyHostToDevice, m->cs));
@@ -494,9 +585,22 @@ int upload_static(mggcn_model_s* m) {
                 if (t.val && !ht.val.empty())
                     CK(cudaMemcpyAsync(const_cast<float*>(t.val), ht.val.data(), sizeof(float) * ht.val.size(),
                                        cudaMemcpyHostToDevice, m->cs));
+                return MGGCN_OK;
+        };
+        for (int j = 0; j < pt->P; ++j)
+            for (int dir = 0; dir < 2; ++dir) {
+                if (dir == 1 && pt->shared_fb) continue;
+                if (m->grp_S > 1 && j != r.rank) continue;
+                RC(upload(dir == 0 ? r.tF(j) : r.tB(j), dir == 0 ? r.hF[j] : r.hB[j], dir == 0 ? r.F[j] : r.B[j]));
             }
+        for (size_t g = 0; g < r.GF.size(); ++g) {
+            RC(upload(r.gF[g], r.hgF[g], r.GF[g]));
+            if (!pt->shared_fb) RC(upload(r.gB[g], r.hgB[g], r.GB[g]));
+        }
         if (pt->shared_fb)
             for (int j = 0; j < pt->P; ++j) r.B[j] = r.F[j];
+        if (pt->shared_fb)
+            for (size_t g = 0; g < r.GF.size(); ++g) r.GB[g] = r.GF[g];
         CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
         // zero every activation buffer once: padding columns stay 0 forever
         for (int k = 0; k < 2; ++k) CK(cudaMemsetAsync(r.Xbuf[k], 0, sizeof(float) * r.rows * m->ld[0], m->cs));
@@ -506,6 +610,7 @@ int upload_static(mggcn_model_s* m) {
         if (r.T0) CK(cudaMemsetAsync(r.T0, 0, sizeof(float) * r.rows * m->ld[0], m->cs));
         for (int s = 0; s < 2; ++s)
             if (r.BC[s]) CK(cudaMemsetAsync(r.BC[s], 0, sizeof(float) * m->max_rows_j * m->bc_ld, m->cs));
+        if (r.BCg) CK(cudaMemsetAsync(r.BCg, 0, sizeof(float) * 2 * m->grp_S * m->max_rows_j * m->bc_ld, m->cs));
     }
     CK(cudaMemsetAsync(m->W, 0, sizeof(float) * m->wtotal, m->cs));
     CK(cudaMemsetAsync(m->flags_dev, 0, sizeof(uint32_t) * 64, m->cs));
@@ -743,6 +848,28 @@ void tl_comm(mggcn_model_s* m, int k, int rank_idx) {
 
 int remote_index(int q, int self) { return q < self ? q : q - 1; }
 
+// Stage groups (choose_group_size): remote index k of a rank lands in slot
+// (g mod 2) * S + (k mod S), g = k / S, packed at the SpMM's width, so group
+// g's blocks are one contiguous operand for its merged tile.
+float* group_slot(mggcn_model_s* m, Rank& r, int k, int64_t width) {
+    const int g = k / m->grp_S, slot = (g & 1) * m->grp_S + k % m->grp_S;
+    return r.BCg + (size_t)slot * (size_t)m->max_rows_j * (size_t)width;
+}
+
+int launch_group(mggcn_model_s* m, Rank& r, const SpmmJob& job, int g, int flags, int tl_k) {
+    RC(inject_delay(m, m->cs));
+    const SpmmTile& t = job.dir == 0 ? r.GF[g] : r.GB[g];
+    float* out = job.dst(m, r, job.ctx);
+    m->tl_stage = tl_k;
+    m->tl_rank = (int32_t)(&r - &m->ranks[0]);
+    ProfScope ps(m, PC_SPMM, m->cs);
+    if ((m->comm || m->solo) && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
+    const float* B = r.BCg + (size_t)((g & 1) * m->grp_S) * (size_t)m->max_rows_j * (size_t)job.width;
+    CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
+                   (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
+    return MGGCN_OK;
+}
+
 // NEXT-1 (SM-free exchange): every receiver PULLS the peers' blocks with copy
 // engines in rotated order (stage s reads block (i + s) mod P, so each GPU
 // serves one reader per step); sequence flags order producer -> pull -> reuse.
@@ -758,6 +885,32 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
     CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
     if (r.rows > 0) RC(launch_stage(m, r, job, me, mysrc, 0, -1));
     RC(mark_stage(m));
+    if (m->grp_S > 1) {   // stage groups: pulls into consecutive slots, one launch per group
+        const int S = m->grp_S, NG = n_groups(m);
+        for (int k = 0; k < P - 1; ++k) {
+            const int q = (me + k + 1) % P, g = k / S;
+            const bool last_of_group = (k % S == S - 1) || k == P - 2;
+            {
+                RC(serial_wait(m));
+                tl_comm(m, q, 0);
+                ProfScope ps(m, PC_BCAST, m->ms);
+                RC(inject_delay(m, m->ms));
+                if (k % S == 0 && g >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[g & 1], 0));
+                CK(stream_wait_u32(m->ms, peer_ptr(m, q, m->flags_dev) + 0, seq));   // block q is ready
+                const size_t bytes = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width * sizeof(float);
+                if (!nob && bytes)
+                    CK(cudaMemcpyAsync(group_slot(m, r, k, job.width), peer_ptr(m, q, mysrc), bytes, cudaMemcpyDefault,
+                                       m->ms));
+                if (last_of_group) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
+            }
+            if (last_of_group) {
+                CK(cudaStreamWaitEvent(m->cs, r.ev_bc[g & 1], 0));
+                if (r.rows > 0) RC(launch_group(m, r, job, g, SPMM_ACCUM | (g == NG - 1 ? SPMM_LAST : 0), q));
+                CK(cudaEventRecord(r.ev_free[g & 1], m->cs));
+                RC(mark_stage(m));
+            }
+        }
+    } else
     for (int st = 1; st < P; ++st) {
         const int q = (me + st) % P, k = st - 1, slot = k & 1;
         {
@@ -889,6 +1042,64 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
     return MGGCN_OK;
 }
 
+// 1D schedule with stage groups: the broadcasts keep their global order
+// (q = 0..P-1, every rank joins every collective); a rank launches group g
+// once the last block of g has arrived; group g + 2 reuses group g's slots.
+int staged_spmm_grouped(mggcn_model_s* m, const SpmmJob& job) {
+    const int P = m->P, S = m->grp_S, NG = n_groups(m);
+    const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
+    for (auto& r : m->ranks)
+        if (r.rows > 0) RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), 0, -1));
+    RC(mark_stage(m));
+    auto last_of_group = [&](int k) { return (k % S == S - 1) || k == P - 2; };
+    for (int q = 0; q < P; ++q) {
+        {
+            RC(serial_wait(m));
+            tl_comm(m, q, -1);
+            ProfScope ps(m, PC_BCAST, m->ms);
+            RC(inject_delay(m, m->ms));
+            if (m->comm || m->solo) {   // solo: nob is set, only the slot events remain
+                Rank& r = m->ranks[0];
+                const size_t count = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width;
+                if (q == r.rank) {
+                    float* src = job.src(m, r, job.ctx);
+                    if (!nob && count) NK(ncclBroadcast(src, src, count, ncclFloat32, q, m->comm, m->ms));
+                } else {
+                    const int k = remote_index(q, r.rank), g = k / S;
+                    if (k % S == 0 && g >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[g & 1], 0));
+                    float* dst = group_slot(m, r, k, job.width);
+                    if (!nob && count) NK(ncclBroadcast(dst, dst, count, ncclFloat32, q, m->comm, m->ms));
+                    if (last_of_group(k)) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
+                }
+            } else {
+                Rank& root = m->ranks[q];
+                const size_t bytes = (size_t)root.rows * (size_t)job.width * sizeof(float);
+                for (auto& r : m->ranks) {
+                    if (r.rank == q) continue;
+                    const int k = remote_index(q, r.rank), g = k / S;
+                    if (k % S == 0 && g >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[g & 1], 0));
+                    if (!nob && bytes)
+                        CK(cudaMemcpyAsync(group_slot(m, r, k, job.width), job.src(m, root, job.ctx), bytes,
+                                           cudaMemcpyDeviceToDevice, m->ms));
+                    if (last_of_group(k)) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
+                }
+            }
+        }
+        for (auto& r : m->ranks) {
+            if (r.rank == q) continue;
+            const int k = remote_index(q, r.rank), g = k / S;
+            if (!last_of_group(k)) continue;
+            CK(cudaStreamWaitEvent(m->cs, r.ev_bc[g & 1], 0));
+            if (r.rows > 0) RC(launch_group(m, r, job, g, SPMM_ACCUM | (g == NG - 1 ? SPMM_LAST : 0), q));
+            CK(cudaEventRecord(r.ev_free[g & 1], m->cs));
+        }
+        RC(mark_stage(m));
+    }
+    CK(cudaEventRecord(m->ev_comm_end, m->ms));
+    CK(cudaStreamWaitEvent(m->cs, m->ev_comm_end, 0));
+    return MGGCN_OK;
+}
+
 int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
     if (m->c > 1) return staged_spmm_15d(m, job);
     const int P = m->P;
@@ -898,6 +1109,7 @@ int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
         CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
     }
     if (m->ipc) return staged_spmm_ipc(m, job);
+    if (m->grp_S > 1) return staged_spmm_grouped(m, job);
     // local stage
     for (auto& r : m->ranks) {
         if (r.rows == 0) continue;
@@ -1218,8 +1430,37 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
             build_items(r.tF(j), r.hF[j], order);
             if (!r.part->shared_fb) build_items(r.tB(j), r.hB[j], order);
         }
+        r.order_cache = order;
     }
     m->n_local = off;
+    m->grp_S = choose_group_size(m, flags);
+    if (m->grp_S > 1) {
+        const bool ipc = (flags & MGGCN_F_IPC) != 0;
+        const int NG = n_groups(m);
+        for (auto& r : m->ranks) {
+            r.gF.assign(NG, HostTile());
+            r.hgF.assign(NG, HostItems());
+            if (!r.part->shared_fb) {
+                r.gB.assign(NG, HostTile());
+                r.hgB.assign(NG, HostItems());
+            }
+            for (int g = 0; g < NG; ++g) {
+                std::vector<const HostTile*> tf, tb;
+                for (int k = g * m->grp_S; k < std::min((g + 1) * m->grp_S, m->P - 1); ++k) {
+                    const int j = remote_block(m, r.rank, k, ipc);
+                    tf.push_back(&r.tF(j));
+                    tb.push_back(&r.tB(j));
+                }
+                merge_group_tiles(tf, m->max_rows_j, r.gF[g]);
+                build_items(r.gF[g], r.hgF[g], r.order_cache);
+                if (!r.part->shared_fb) {
+                    merge_group_tiles(tb, m->max_rows_j, r.gB[g]);
+                    build_items(r.gB[g], r.hgB[g], r.order_cache);
+                }
+            }
+        }
+    }
+    for (auto& r : m->ranks) std::vector<int32_t>().swap(r.order_cache);
     // the SpMM gathers address B with 32-bit float4 offsets: rows * ld/4 < 2^32
     if ((double)m->max_rows_j * (double)(std::max(m->bc_ld, m->ld[0]) / 4) >= 4294967296.0 ||
         (double)off * (double)(std::max(m->bc_ld, m->ld[0]) / 4) >= 4294967296.0) {

@@ -65,10 +65,10 @@ def compare(lib, ref, dims, tol=REL_TOL):
     for l in range(len(dims) - 1):
         mo, ve, t = lib["adam"][l]
         assert t == 1
-        assert rel(mo, ref.m[l]) < tol and rel(ve, ref.v[l]) < 2 * tol
-        # W only where |g| is not tiny (first Adam step ~ lr * sign(g))
+        assert rel(mo, ref.m[l]) < tol and rel(ve, ref.v[l]) < tol
+        # W only where |g| is not tiny (first Adam step ~ lr * sign(g); reading C30)
         g = ref.WG[l]
-        mask = np.abs(g) > 1e-3 * np.abs(g).max()
+        mask = np.abs(g) > max(1e-3 * np.abs(g).max(), 100 * 1e-8)
         np.testing.assert_allclose(lib["W"][l][mask], ref.W[l][mask], rtol=0, atol=1e-5)
 
 
@@ -421,12 +421,15 @@ def test_delay_injection_keeps_results_bitwise(mg, P, replicas):
 
 
 def _stage_overlaps(tl):
-    """Pairs (comm record, SpMM stage record) of the same SpMM whose device intervals intersect."""
+    """Pairs (comm record of block q, SpMM stage record of another block q') of the same SpMM whose
+    device intervals intersect.  (In loopback one comm record holds the copies of block q to every
+    receiver, so a receiver's stage of that same block may start before the record ends.)"""
     eps = 2e-3   # ms: event timestamp resolution
     comm = [r for r in tl if r["stream"] == 1 and r["cls"] == "bcast" and r["spmm"] >= 0]
     comp = [r for r in tl if r["stream"] == 0 and r["cls"] == "spmm" and r["spmm"] >= 0]
     return [(a, b) for a in comm for b in comp
-            if a["spmm"] == b["spmm"] and a["t0"] < b["t1"] - eps and b["t0"] < a["t1"] - eps]
+            if a["spmm"] == b["spmm"] and a["stage"] != b["stage"] and a["t0"] < b["t1"] - eps
+            and b["t0"] < a["t1"] - eps]
 
 
 @pytest.mark.parametrize("P,replicas", [(4, 1), (4, 2)])
@@ -464,3 +467,20 @@ def test_overlap_flag_orders_exchange_and_stages(mg, P, replicas):
     assert res[False][0] == res[True][0]
     for a, b in zip(res[False][1], res[True][1]):
         assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("group", ["1", "3", "7"])
+def test_stage_group_sizes_epoch(mg, monkeypatch, group):
+    """Loopback P = 8 epochs with 1 (the paper's one launch per stage), 3 and 7 remote blocks per
+    launch match the oracle (logits, loss, W_G, Adam) and are bitwise reproducible under delay
+    injection (the group launch waits for the last block of its group, P:939-941 slot rule)."""
+    monkeypatch.setenv("MGGCN_STAGE_GROUP", group)
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    ref = oracle.epoch(oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed), X, y, Ws)
+    a = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 8, w.perm_seed, mg.MGGCN_F_OVERLAP)
+    compare(a, ref, w.dims)
+    b = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 8, w.perm_seed, mg.MGGCN_F_OVERLAP, delay=(9, 150))
+    assert np.array_equal(a["logits"], b["logits"]) and a["loss"] == b["loss"]
+    for u, v in zip(a["W"], b["W"]):
+        assert np.array_equal(u, v)

@@ -104,3 +104,24 @@ def test_bench_two_ranks_ipc_exposed_comm():
     ex = d["exposed_comm"]
     assert ex is not None and ex["compute_only_ms"] > 0 and 0.0 <= ex["frac"] <= 1.0
     assert ex["bcast_bytes_per_rank_per_epoch"] > 0
+
+
+def test_ipc_four_ranks_stage_groups(tmp_path):
+    """Four IPC ranks (rotated pulls, P = 4): the default schedule groups the three remote
+    blocks of a rank into two launches (merged tiles over consecutive BC slots,
+    choose_group_size); ranks agree bitwise and match the P = 4 oracle."""
+    n, m, dims = 3001, 60000, (100, 64, 64, 7)
+    rp, col = gen.rmat_csr(n, m, 71)
+    X = gen.features(n, dims[0], 72)
+    y = gen.labels(n, dims[-1], 73, 200)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 74 + l) for l in range(len(dims) - 1)]
+    ref = oracle.epoch(oracle.permute_graph(n, rp, col, None, seed=75), X, y, Ws, P=4)
+    res = run_ranks(tmp_path, "device", world=4, steps=1)
+    for r in res[1:]:
+        for k in ["loss0"] + [f"WG0_{l}" for l in range(3)] + [f"W{l}" for l in range(3)]:
+            assert np.array_equal(res[0][k], r[k]), k
+    logits = np.concatenate([r["logits"] for r in res])
+    assert rel(logits, ref.logits) < REL_TOL
+    assert abs(float(res[0]["loss0"]) - ref.loss) / abs(ref.loss) < REL_TOL
+    for l in range(3):
+        assert rel(res[0][f"WG0_{l}"], ref.WG[l]) < REL_TOL, l

@@ -139,6 +139,24 @@ def test_spmm_exactness_graph(mg, P, width):
     _spmm_check(mg, n, rp, col, None, P, width, seed=5, exact=True)
 
 
+@pytest.mark.parametrize("P,group", [(4, None), (5, "1"), (5, "3"), (8, None), (8, "2"), (8, "7")])
+def test_spmm_stage_groups_exact(mg, monkeypatch, P, group):
+    """Stage groups (model.cu choose_group_size: several remote blocks consumed by one launch
+    over a merged tile whose columns address consecutive BC slots): bit-exact on the
+    exactness graph for the default grouping and forced group sizes (1 = one launch per
+    stage), and within 1e-5 on R-MAT hubs (split rows + fix-up over merged rows)."""
+    if group is not None:
+        monkeypatch.setenv("MGGCN_STAGE_GROUP", group)
+    n = 1037
+    rp, col, _ = _circulant(n, 3)
+    for width in (7, 48, 256):
+        _spmm_check(mg, n, rp, col, None, P, width, seed=5, exact=True)
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    for width in (44, 256):
+        _spmm_check(mg, n, rp, col, None, P, width, seed=9, exact=False)
+
+
 @pytest.mark.parametrize("P", [1, 2, 4])
 @pytest.mark.parametrize("width", [8, 44, 48, 100, 128, 172, 256, 512, 600])
 @pytest.mark.parametrize("coalesce", [True, False])

@@ -242,7 +242,10 @@ struct mggcn_model_s {
     int64_t n_local = 0;            // rows owned by this model (sum over local ranks)
     int64_t max_rows_j = 0;
     int64_t bc_ld = 0, hw_ld = 0;
-    int grp_S = 1;                  // remote stages per launch (1 = one launch per stage, the paper's schedule)
+    // stage groups (choose_groups): remote indices [grp_b[g], grp_b[g+1]) are consumed by one
+    // launch; empty = one launch per stage (the paper's schedule, BC1/BC2)
+    std::vector<int> grp_b;
+    bool grouped() const { return !grp_b.empty(); }
     std::vector<Rank> ranks;
     float *W = nullptr, *Mom = nullptr, *Vel = nullptr, *WG = nullptr;
     // tf32 hi/lo copies of W for the tcgen05 row GEMMs (refreshed after every update):
@@ -354,33 +357,66 @@ inline int remote_block(const mggcn_model_s* m, int rank, int k, bool ipc) {
     if (ipc) return (rank + k + 1) % m->P;
     return k < rank ? k : k + 1;
 }
-inline int n_groups(const mggcn_model_s* m) { return (m->P - 1 + m->grp_S - 1) / m->grp_S; }
+inline int n_groups(const mggcn_model_s* m) { return m->grouped() ? (int)m->grp_b.size() - 1 : 0; }
+inline int group_of(const mggcn_model_s* m, int k) {
+    int g = 0;
+    while (k >= m->grp_b[g + 1]) ++g;
+    return g;
+}
+inline bool last_of_group(const mggcn_model_s* m, int k) { return k == m->grp_b[group_of(m, k) + 1] - 1; }
 
-// Remote stages per launch (per-stage launches pay a row visit, an output
-// read-modify-write, a launch and a hub fix-up per stage; at P = 8 a Reddit-shaped rank's
-// stages are 40-100 us, so those fixed costs are a third of its SpMM time).  Default:
-// two remote groups per SpMM, ceil((P-1)/2) blocks each, both in flight (2S BC slots),
-// so group 1's blocks arrive while group 0 computes; capped so the 2S slots fit
-// MGGCN_BC_BUDGET_MB (default 16 GiB: Papers-shaped blocks of 14 GB keep S = 1).
-// MGGCN_STAGE_GROUP=S overrides (1 = the paper's one launch per stage).  1D only.
-int choose_group_size(const mggcn_model_s* m, uint32_t flags) {
-    if (m->P <= 2 || m->c > 1) return 1;
-    int S = (m->P - 1 + 1) / 2;
-    if (const char* e = getenv("MGGCN_STAGE_GROUP")) {
-        const int v = atoi(e);
-        if (v >= 1) S = v;
-    }
+// Stage groups.  One launch per stage (the paper's schedule) pays, per stage,
+// a visit of every row with entries, an output read-modify-write, a launch
+// and a hub fix-up; at P = 8 a Reddit-shaped rank's stages are 40-100 us, so
+// these fixed costs are about a third of its SpMM time.  Grouped,
+// the remote blocks get one BC slot each (P - 1 slots, no reuse inside a
+// SpMM) and a group of them is consumed by ONE launch over a merged tile.
+// Default: two groups per SpMM, a small first one (ceil((P-1)/4) blocks, whose
+// transfer hides behind the local stage) and the rest (whose transfer hides
+// behind the first group); P >= 4.  Off when the P - 1 slots exceed
+// MGGCN_BC_BUDGET_MB (default 16 GiB: Papers-shaped 14 GB blocks keep BC1/BC2).
+// MGGCN_STAGE_GROUPS="a,b,.." (sizes summing to P - 1) or MGGCN_STAGE_GROUP=S
+// (uniform; 1 = per stage) override.  1D only.
+std::vector<int> choose_groups(const mggcn_model_s* m) {
+    std::vector<int> none;
+    if (m->P <= 2 || m->c > 1) return none;
     if (const char* h = getenv("MGGCN_SPMM_HOTCLS"))
-        if (atoi(h) != 0) S = 1;   // priority-class tiles keep per-stage launches
-    S = std::max(1, std::min(S, m->P - 1));
+        if (atoi(h) != 0) return none;   // priority-class tiles keep per-stage launches
+    const int R = m->P - 1;
+    std::vector<int> sizes;
+    if (const char* e = getenv("MGGCN_STAGE_GROUPS")) {
+        int tot = 0;
+        for (const char* c = e; *c;) {
+            const int v = atoi(c);
+            if (v <= 0) { sizes.clear(); break; }
+            sizes.push_back(v);
+            tot += v;
+            while (*c && *c != ',') ++c;
+            if (*c == ',') ++c;
+        }
+        if (tot != R) sizes.clear();
+    }
+    if (sizes.empty()) {
+        int S = 0;
+        if (const char* e = getenv("MGGCN_STAGE_GROUP")) S = atoi(e);
+        if (S == 1) return none;
+        if (S > 1) {
+            for (int k = 0; k < R; k += S) sizes.push_back(std::min(S, R - k));
+        } else {
+            if (m->P < 4) return none;
+            const int first = (R + 3) / 4;
+            sizes = {first, R - first};
+        }
+    }
     double budget = 16384.0;
     if (const char* e = getenv("MGGCN_BC_BUDGET_MB")) budget = atof(e);
-    const double slot = (double)m->max_rows_j * (double)m->bc_ld * 4.0 / 1048576.0;
-    while (S > 1 && 2.0 * S * slot > budget) --S;
+    const double slot_mb = (double)m->max_rows_j * (double)m->bc_ld * 4.0 / 1048576.0;
+    if ((double)R * slot_mb > budget) return none;
     // merged column ids and the kernel's 32-bit float4 row offsets must not overflow
-    while (S > 1 && (double)S * (double)m->max_rows_j * (double)(m->bc_ld / 4) >= 4294967296.0) --S;
-    (void)flags;
-    return S;
+    if ((double)R * (double)m->max_rows_j * (double)(m->bc_ld / 4) >= 4294967296.0) return none;
+    std::vector<int> b(1, 0);
+    for (int v : sizes) b.push_back(b.back() + v);
+    return b;
 }
 
 // ---------------------------------------------------------------- profiling
@@ -516,7 +552,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
         for (int j = 0; j < P; ++j) {
             // with stage groups only the local tile is launched per stage (the remote ones
             // live in the merged group tiles; mggcn_part_export_tile reads the host copies)
-            const bool on_dev = m->grp_S == 1 || j == r.rank;
+            const bool on_dev = !m->grouped() || j == r.rank;
             for (int dir = 0; dir < 2; ++dir) {
                 if (dir == 1 && pt->shared_fb) {
                     r.B[j] = r.F[j];
@@ -526,7 +562,7 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                 if (on_dev) place(dir == 0 ? r.tF(j) : r.tB(j), dir == 0 ? r.hF[j] : r.hB[j], t, true);
             }
         }
-        const int NG = m->grp_S > 1 ? n_groups(m) : 0;
+        const int NG = n_groups(m);
         r.GF.assign(NG, SpmmTile());
         r.GB.assign(NG, SpmmTile());
         for (int g = 0; g < NG; ++g) {
@@ -539,11 +575,11 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
         r.Xs = r.Xbuf[0];
         r.y = r.ybuf[0];
         r.T0 = m->order[0] == S_ORDER ? b.take<float>(r.rows * m->ld[0]) : nullptr;
-        if (P > 1 && m->grp_S == 1) {
+        if (P > 1 && !m->grouped()) {
             r.BC[0] = b.take<float>(m->max_rows_j * m->bc_ld);
             r.BC[1] = b.take<float>(m->max_rows_j * m->bc_ld);
         } else if (P > 1) {
-            r.BCg = b.take<float>(2 * m->grp_S * m->max_rows_j * m->bc_ld);
+            r.BCg = b.take<float>((P - 1) * m->max_rows_j * m->bc_ld);
         }
         int64_t slots = 0;
         for (int j = 0; j < P; ++j) {
@@ -590,7 +626,7 @@ int upload_static(mggcn_model_s* m) {
         for (int j = 0; j < pt->P; ++j)
             for (int dir = 0; dir < 2; ++dir) {
                 if (dir == 1 && pt->shared_fb) continue;
-                if (m->grp_S > 1 && j != r.rank) continue;
+                if (m->grouped() && j != r.rank) continue;
                 RC(upload(dir == 0 ? r.tF(j) : r.tB(j), dir == 0 ? r.hF[j] : r.hB[j], dir == 0 ? r.F[j] : r.B[j]));
             }
         for (size_t g = 0; g < r.GF.size(); ++g) {
@@ -610,7 +646,7 @@ int upload_static(mggcn_model_s* m) {
         if (r.T0) CK(cudaMemsetAsync(r.T0, 0, sizeof(float) * r.rows * m->ld[0], m->cs));
         for (int s = 0; s < 2; ++s)
             if (r.BC[s]) CK(cudaMemsetAsync(r.BC[s], 0, sizeof(float) * m->max_rows_j * m->bc_ld, m->cs));
-        if (r.BCg) CK(cudaMemsetAsync(r.BCg, 0, sizeof(float) * 2 * m->grp_S * m->max_rows_j * m->bc_ld, m->cs));
+        if (r.BCg) CK(cudaMemsetAsync(r.BCg, 0, sizeof(float) * (m->P - 1) * m->max_rows_j * m->bc_ld, m->cs));
     }
     CK(cudaMemsetAsync(m->W, 0, sizeof(float) * m->wtotal, m->cs));
     CK(cudaMemsetAsync(m->flags_dev, 0, sizeof(uint32_t) * 64, m->cs));
@@ -848,12 +884,11 @@ void tl_comm(mggcn_model_s* m, int k, int rank_idx) {
 
 int remote_index(int q, int self) { return q < self ? q : q - 1; }
 
-// Stage groups (choose_group_size): remote index k of a rank lands in slot
-// (g mod 2) * S + (k mod S), g = k / S, packed at the SpMM's width, so group
-// g's blocks are one contiguous operand for its merged tile.
+// Stage groups (choose_groups): remote index k of a rank lands in its own slot k,
+// packed at the SpMM's width, so a group's blocks are one contiguous operand for
+// its merged tile.
 float* group_slot(mggcn_model_s* m, Rank& r, int k, int64_t width) {
-    const int g = k / m->grp_S, slot = (g & 1) * m->grp_S + k % m->grp_S;
-    return r.BCg + (size_t)slot * (size_t)m->max_rows_j * (size_t)width;
+    return r.BCg + (size_t)k * (size_t)m->max_rows_j * (size_t)width;
 }
 
 int launch_group(mggcn_model_s* m, Rank& r, const SpmmJob& job, int g, int flags, int tl_k) {
@@ -864,7 +899,7 @@ int launch_group(mggcn_model_s* m, Rank& r, const SpmmJob& job, int g, int flags
     m->tl_rank = (int32_t)(&r - &m->ranks[0]);
     ProfScope ps(m, PC_SPMM, m->cs);
     if ((m->comm || m->solo) && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
-    const float* B = r.BCg + (size_t)((g & 1) * m->grp_S) * (size_t)m->max_rows_j * (size_t)job.width;
+    const float* B = group_slot(m, r, m->grp_b[g], job.width);
     CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
                    (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
     return MGGCN_OK;
@@ -885,28 +920,26 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
     CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
     if (r.rows > 0) RC(launch_stage(m, r, job, me, mysrc, 0, -1));
     RC(mark_stage(m));
-    if (m->grp_S > 1) {   // stage groups: pulls into consecutive slots, one launch per group
-        const int S = m->grp_S, NG = n_groups(m);
+    if (m->grouped()) {   // stage groups: pulls into dedicated slots, one launch per group
+        const int NG = n_groups(m);
         for (int k = 0; k < P - 1; ++k) {
-            const int q = (me + k + 1) % P, g = k / S;
-            const bool last_of_group = (k % S == S - 1) || k == P - 2;
+            const int q = (me + k + 1) % P, g = group_of(m, k);
+            const bool last = last_of_group(m, k);
             {
                 RC(serial_wait(m));
                 tl_comm(m, q, 0);
                 ProfScope ps(m, PC_BCAST, m->ms);
                 RC(inject_delay(m, m->ms));
-                if (k % S == 0 && g >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[g & 1], 0));
                 CK(stream_wait_u32(m->ms, peer_ptr(m, q, m->flags_dev) + 0, seq));   // block q is ready
                 const size_t bytes = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width * sizeof(float);
                 if (!nob && bytes)
                     CK(cudaMemcpyAsync(group_slot(m, r, k, job.width), peer_ptr(m, q, mysrc), bytes, cudaMemcpyDefault,
                                        m->ms));
-                if (last_of_group) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
+                if (last) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
             }
-            if (last_of_group) {
+            if (last) {
                 CK(cudaStreamWaitEvent(m->cs, r.ev_bc[g & 1], 0));
                 if (r.rows > 0) RC(launch_group(m, r, job, g, SPMM_ACCUM | (g == NG - 1 ? SPMM_LAST : 0), q));
-                CK(cudaEventRecord(r.ev_free[g & 1], m->cs));
                 RC(mark_stage(m));
             }
         }
@@ -1046,12 +1079,11 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
 // (q = 0..P-1, every rank joins every collective); a rank launches group g
 // once the last block of g has arrived; group g + 2 reuses group g's slots.
 int staged_spmm_grouped(mggcn_model_s* m, const SpmmJob& job) {
-    const int P = m->P, S = m->grp_S, NG = n_groups(m);
+    const int P = m->P, NG = n_groups(m);
     const bool nob = (m->flags & MGGCN_F_NO_BCAST) != 0;
     for (auto& r : m->ranks)
         if (r.rows > 0) RC(launch_stage(m, r, job, r.rank, job.src(m, r, job.ctx), 0, -1));
     RC(mark_stage(m));
-    auto last_of_group = [&](int k) { return (k % S == S - 1) || k == P - 2; };
     for (int q = 0; q < P; ++q) {
         {
             RC(serial_wait(m));
@@ -1065,33 +1097,31 @@ int staged_spmm_grouped(mggcn_model_s* m, const SpmmJob& job) {
                     float* src = job.src(m, r, job.ctx);
                     if (!nob && count) NK(ncclBroadcast(src, src, count, ncclFloat32, q, m->comm, m->ms));
                 } else {
-                    const int k = remote_index(q, r.rank), g = k / S;
-                    if (k % S == 0 && g >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[g & 1], 0));
+                    const int k = remote_index(q, r.rank);
                     float* dst = group_slot(m, r, k, job.width);
                     if (!nob && count) NK(ncclBroadcast(dst, dst, count, ncclFloat32, q, m->comm, m->ms));
-                    if (last_of_group(k)) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
+                    if (last_of_group(m, k)) CK(cudaEventRecord(r.ev_bc[group_of(m, k) & 1], m->ms));
                 }
             } else {
                 Rank& root = m->ranks[q];
                 const size_t bytes = (size_t)root.rows * (size_t)job.width * sizeof(float);
                 for (auto& r : m->ranks) {
                     if (r.rank == q) continue;
-                    const int k = remote_index(q, r.rank), g = k / S;
-                    if (k % S == 0 && g >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[g & 1], 0));
+                    const int k = remote_index(q, r.rank);
                     if (!nob && bytes)
                         CK(cudaMemcpyAsync(group_slot(m, r, k, job.width), job.src(m, root, job.ctx), bytes,
                                            cudaMemcpyDeviceToDevice, m->ms));
-                    if (last_of_group(k)) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
+                    if (last_of_group(m, k)) CK(cudaEventRecord(r.ev_bc[group_of(m, k) & 1], m->ms));
                 }
             }
         }
         for (auto& r : m->ranks) {
             if (r.rank == q) continue;
-            const int k = remote_index(q, r.rank), g = k / S;
-            if (!last_of_group(k)) continue;
+            const int k = remote_index(q, r.rank);
+            if (!last_of_group(m, k)) continue;
+            const int g = group_of(m, k);
             CK(cudaStreamWaitEvent(m->cs, r.ev_bc[g & 1], 0));
             if (r.rows > 0) RC(launch_group(m, r, job, g, SPMM_ACCUM | (g == NG - 1 ? SPMM_LAST : 0), q));
-            CK(cudaEventRecord(r.ev_free[g & 1], m->cs));
         }
         RC(mark_stage(m));
     }
@@ -1109,7 +1139,7 @@ int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
         CK(cudaStreamWaitEvent(m->ms, m->ev_begin, 0));
     }
     if (m->ipc) return staged_spmm_ipc(m, job);
-    if (m->grp_S > 1) return staged_spmm_grouped(m, job);
+    if (m->grouped()) return staged_spmm_grouped(m, job);
     // local stage
     for (auto& r : m->ranks) {
         if (r.rows == 0) continue;
@@ -1433,8 +1463,8 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         r.order_cache = order;
     }
     m->n_local = off;
-    m->grp_S = choose_group_size(m, flags);
-    if (m->grp_S > 1) {
+    m->grp_b = choose_groups(m);
+    if (m->grouped()) {
         const bool ipc = (flags & MGGCN_F_IPC) != 0;
         const int NG = n_groups(m);
         for (auto& r : m->ranks) {
@@ -1446,7 +1476,7 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
             }
             for (int g = 0; g < NG; ++g) {
                 std::vector<const HostTile*> tf, tb;
-                for (int k = g * m->grp_S; k < std::min((g + 1) * m->grp_S, m->P - 1); ++k) {
+                for (int k = m->grp_b[g]; k < m->grp_b[g + 1]; ++k) {
                     const int j = remote_block(m, r.rank, k, ipc);
                     tf.push_back(&r.tF(j));
                     tb.push_back(&r.tB(j));

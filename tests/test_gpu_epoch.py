@@ -469,12 +469,15 @@ def test_overlap_flag_orders_exchange_and_stages(mg, P, replicas):
         assert np.array_equal(a, b)
 
 
-@pytest.mark.parametrize("group", ["1", "3", "7"])
-def test_stage_group_sizes_epoch(mg, monkeypatch, group):
-    """Loopback P = 8 epochs with 1 (the paper's one launch per stage), 3 and 7 remote blocks per
-    launch match the oracle (logits, loss, W_G, Adam) and are bitwise reproducible under delay
-    injection (the group launch waits for the last block of its group, P:939-941 slot rule)."""
-    monkeypatch.setenv("MGGCN_STAGE_GROUP", group)
+@pytest.mark.parametrize("var,group", [("MGGCN_STAGE_GROUP", "1"), ("MGGCN_STAGE_GROUP", "3"),
+                                       ("MGGCN_STAGE_GROUP", "7"), ("MGGCN_STAGE_GROUPS", "3,4"), (None, None)])
+def test_stage_group_sizes_epoch(mg, monkeypatch, var, group):
+    """Loopback P = 8 epochs with 1 (the paper's one launch per stage), 3, 7 and (3, 4) remote
+    blocks per launch and the default grouping match the oracle (logits, loss, W_G, Adam) and
+    are bitwise reproducible under delay injection (a group launch waits for the last block of
+    its group)."""
+    if var:
+        monkeypatch.setenv(var, group)
     w = gen.WORKLOADS["cora"]
     rp, col, X, y, Ws = workload_inputs(w)
     ref = oracle.epoch(oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed), X, y, Ws)

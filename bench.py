@@ -313,6 +313,79 @@ def l2_gather_roofline(dims, work, spmm_ms_per_epoch, cache=False):
             "peak_source_blob_sha": _git_blob_sha(os.path.join(ROOT, "bench_micro", "dsmem_gather.cu"))}
 
 
+def _union(iv):
+    iv = sorted(iv)
+    out = []
+    for a, b in iv:
+        if out and a <= out[-1][1]:
+            out[-1][1] = max(out[-1][1], b)
+        else:
+            out.append([a, b])
+    return out
+
+
+def _measure(iv):
+    return sum(b - a for a, b in iv)
+
+
+def _intersect(u, v):
+    i = j = 0
+    tot = 0.0
+    while i < len(u) and j < len(v):
+        a, b = max(u[i][0], v[j][0]), min(u[i][1], v[j][1])
+        if b > a:
+            tot += b - a
+        if u[i][1] < v[j][1]:
+            i += 1
+        else:
+            j += 1
+    return tot
+
+
+def timeline_summary(tl, dims, p, rank):
+    """Per-stage comm / compute timeline of one epoch (MGGCN_F_TIMELINE; the paper's Fig. 6 / 8,
+    P:1372-1403): busy time per stream, the comm time not covered by any compute
+    op (exposed), and broadcast GB/s per received block."""
+    L = len(dims) - 1
+    fwd = [dims[l] if dims[l] < dims[l + 1] else dims[l + 1] for l in range(L)]
+    bwd = [dims[l + 1] for l in range(L - 1, -1, -1) if dims[l] >= dims[l + 1]]
+    widths = fwd + bwd
+    comp = [(r["t0"], r["t1"]) for r in tl if r["stream"] == 0]
+    comm = [(r["t0"], r["t1"]) for r in tl if r["stream"] == 1]
+    if not comp:
+        return None
+    t0 = min(a for a, _ in comp + comm)
+    t1 = max(b for _, b in comp + comm)
+    uc, um = _union(comp), _union(comm)
+    exposed = _measure(um) - _intersect(um, uc)
+    gbps = []
+    for r in tl:
+        if r["stream"] == 1 and r["cls"] == "bcast" and 0 <= r["spmm"] < len(widths) and r["stage"] >= 0 \
+                and r["stage"] != rank and r["t1"] > r["t0"]:
+            rows = int(p[r["stage"] + 1] - p[r["stage"]])
+            gbps.append(rows * widths[r["spmm"]] * 4 / ((r["t1"] - r["t0"]) * 1e-3) / 1e9)
+    per = {}
+    for r in tl:
+        if r["spmm"] < 0:
+            continue
+        d = per.setdefault(r["spmm"], {"width": widths[r["spmm"]] if r["spmm"] < len(widths) else None,
+                                       "compute_launches": 0, "compute_ms": 0.0, "comm_ops": 0, "comm_ms": 0.0})
+        if r["stream"] == 0:
+            d["compute_launches"] += 1
+            d["compute_ms"] += r["t1"] - r["t0"]
+        else:
+            d["comm_ops"] += 1
+            d["comm_ms"] += r["t1"] - r["t0"]
+    return {"epoch_span_ms": t1 - t0, "compute_busy_ms": _measure(uc), "comm_busy_ms": _measure(um),
+            "exposed_comm_ms": exposed, "exposed_comm_frac": exposed / (t1 - t0) if t1 > t0 else None,
+            "bcast_GBps_median": statistics.median(gbps) if gbps else None, "bcast_records": len(gbps),
+            "per_spmm": {str(k): {kk: (round(vv, 4) if isinstance(vv, float) else vv) for kk, vv in v.items()}
+                         for k, v in sorted(per.items())},
+            "how": "one eager epoch with MGGCN_F_TIMELINE (CUDA event pair per op on the stream it runs on; the "
+                   "timed epochs run without it); exposed = comm-stream busy time not covered by any compute-stream "
+                   "op; bcast GB/s = received block bytes / broadcast duration"}
+
+
 def auto_rows(w):
     # about 3 s of single-core oracle work per sampled epoch
     per_row = (w.m / w.n) * sum(w.dims) * 2 + 3 * sum(w.dims[l] * w.dims[l + 1] for l in range(len(w.dims) - 1))
@@ -439,6 +512,19 @@ def main():
     prof = gm.profile(reset=True)
     work = gm.epoch_work()
     work_detail = gm.epoch_work_detail()
+    # ---- one extra eager epoch with the per-stage timeline (not timed)
+    timeline = None
+    try:
+        mg.mggcn_get_timeline(gm.m, reset=True)
+        mg.mggcn_timeline_enable(gm.m, True)
+        epoch(Xd, yd)
+        gm.synchronize()
+        tl = mg.mggcn_get_timeline(gm.m, reset=True)
+        mg.mggcn_timeline_enable(gm.m, False)
+        gm.profile(reset=True)
+        timeline = timeline_summary(tl, w.dims, gm.p, rank % (P // args.replicas))
+    except mg.MggcnError as e:
+        timeline = {"error": str(e)}
     ms_eager = max_over_ranks(dist, ms)
 
     # ---- the same epochs as one CUDA graph each (mggcn_epoch_capture / _replay): identical
@@ -678,6 +764,7 @@ def main():
         "loss_after": loss_now,
         "cache_l0": cache_l0,
         "exposed_comm": exposed,
+        "timeline": timeline,
         "graph_stats": gstats,
         "setup_s": {"generate": t_gen, "load_csr+partition+upload": t_setup},
     }

@@ -275,6 +275,10 @@ int mggcn_get_profile(mggcn_model m, double* ms /*[7]*/, int64_t* launches /*[7]
  * records available (may exceed cap).  Synchronises both streams.
  * EINVAL: cap < 0, or cap > 0 with a NULL array. */
 int mggcn_get_timeline(mggcn_model m, int64_t cap, int32_t* meta, double* t_ms, int64_t* count, int32_t reset);
+/* Turns MGGCN_F_TIMELINE on (on != 0) or off for the calls that follow (the
+ * records cost two events per op, so timed loops run without it).  ESTATE
+ * during an epoch capture. */
+int mggcn_timeline_enable(mggcn_model m, int32_t on);
 /* Algorithmic work of one epoch of this model's rows for the roofline
  * (DESIGN.md §6): spmm_bytes = compulsory SpMM bytes
  * (indices + rowptr + each input row once + each output row once, summed over

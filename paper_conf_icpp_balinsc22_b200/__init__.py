@@ -39,7 +39,7 @@ EXPORTS = (
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
     "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
     "mggcn_epoch_replay", "mggcn_debug_comm_delay", "mggcn_get_timeline",
-    "mggcn_epoch_work_detail",
+    "mggcn_epoch_work_detail", "mggcn_timeline_enable",
 )
 
 
@@ -85,6 +85,7 @@ def _load():
         "mggcn_set_adam": ([P, i32, P, P, i64], ctypes.c_int),
         "mggcn_get_profile": ([P, P, P, i32], ctypes.c_int),
         "mggcn_get_timeline": ([P, i64, P, P, P, i32], ctypes.c_int),
+        "mggcn_timeline_enable": ([P, i32], ctypes.c_int),
         "mggcn_epoch_work": ([P, P, P, P, P], ctypes.c_int),
         "mggcn_epoch_work_detail": ([P, P, i32], ctypes.c_int),
         "mggcn_graph_free": ([P], None),
@@ -307,6 +308,10 @@ def mggcn_get_profile(m, reset=False):
     n = (ctypes.c_int64 * 7)()
     _check(_lib.mggcn_get_profile(m, ms, n, 1 if reset else 0))
     return {c: (ms[i], n[i]) for i, c in enumerate(PROFILE_CLASSES)}
+
+
+def mggcn_timeline_enable(m, on=True):
+    _check(_lib.mggcn_timeline_enable(m, 1 if on else 0))
 
 
 def mggcn_get_timeline(m, reset=True):

@@ -2384,6 +2384,17 @@ extern "C" int mggcn_get_profile(mggcn_model m, double* ms, int64_t* launches, i
     return MGGCN_OK;
 }
 
+extern "C" int mggcn_timeline_enable(mggcn_model m, int32_t on) {
+    MODEL_GUARD(m);
+    if (m->capturing) {
+        set_error("timeline_enable: not during an epoch capture");
+        return MGGCN_ESTATE;
+    }
+    if (on) m->flags |= MGGCN_F_TIMELINE;
+    else m->flags &= ~(uint32_t)MGGCN_F_TIMELINE;
+    return MGGCN_OK;
+}
+
 extern "C" int mggcn_get_timeline(mggcn_model m, int64_t cap, int32_t* meta, double* t_ms, int64_t* count,
                                   int32_t reset) {
     MODEL_GUARD(m);

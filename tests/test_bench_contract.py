@@ -62,3 +62,22 @@ def test_graph_stats_tile_spread_matches_brute_force():
         bv = np.searchsorted(bnd, pv, side="right") - 1
         c = np.bincount(bu * P + bv, minlength=P * P)
         assert abs(st["tile_nnz_max_over_mean"][P] - c.max() / c.mean()) < 1e-12
+
+
+def test_timeline_summary_exposed_comm_and_bandwidth():
+    """bench.timeline_summary (host logic of the per-stage timeline, Fig. 6 / 8): exposed comm is the
+    comm-stream busy time not covered by compute-stream ops; bcast GB/s from the block's bytes."""
+    import bench
+    tl = [dict(cls="spmm", spmm=0, stage=-1, rank=0, stream=0, t0=0.0, t1=1.0),
+          dict(cls="bcast", spmm=0, stage=1, rank=-1, stream=1, t0=0.5, t1=1.5),
+          dict(cls="bcast", spmm=0, stage=0, rank=-1, stream=1, t0=1.5, t1=1.6),   # own block (sent)
+          dict(cls="spmm", spmm=0, stage=1, rank=0, stream=0, t0=1.6, t1=2.0),
+          dict(cls="gemm", spmm=-1, stage=-1, rank=-1, stream=0, t0=2.0, t1=2.5)]
+    s = bench.timeline_summary(tl, (8, 4, 2), [0, 1000, 2000], 0)
+    assert abs(s["epoch_span_ms"] - 2.5) < 1e-12
+    assert abs(s["compute_busy_ms"] - 1.9) < 1e-12
+    assert abs(s["comm_busy_ms"] - 1.1) < 1e-12
+    assert abs(s["exposed_comm_ms"] - 0.6) < 1e-12          # (1.0..1.5) and (1.5..1.6)
+    assert s["bcast_records"] == 1                           # received blocks only
+    assert abs(s["bcast_GBps_median"] - 1000 * 4 * 4 / 1e-3 / 1e9) < 1e-9
+    assert s["per_spmm"]["0"]["compute_launches"] == 2 and s["per_spmm"]["0"]["width"] == 4

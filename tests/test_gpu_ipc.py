@@ -104,6 +104,10 @@ def test_bench_two_ranks_ipc_exposed_comm():
     ex = d["exposed_comm"]
     assert ex is not None and ex["compute_only_ms"] > 0 and 0.0 <= ex["frac"] <= 1.0
     assert ex["bcast_bytes_per_rank_per_epoch"] > 0
+    tl = d["timeline"]      # per-stage comm / compute timeline of one epoch (Fig. 6 / 8)
+    assert tl is not None and "error" not in tl, tl
+    assert tl["comm_busy_ms"] > 0 and tl["compute_busy_ms"] > 0 and tl["bcast_records"] > 0
+    assert 0.0 <= tl["exposed_comm_frac"] <= 1.0
 
 
 def test_ipc_four_ranks_stage_groups(tmp_path):

@@ -15,9 +15,10 @@ configuration, and is compared element by element with the oracle's:
   loss                                                  rel <= 1e-3
   W_G,l     every element, every layer                  rel <= 1e-3
   Adam m, v after the step, every element               rel <= 1e-3
-  W after the step where |g| > max(1e-3 max|g|, 100 eps) (SURVEY §8(c):
-            the first Adam step is lr g / (|g| + eps) ~ lr sign(g); DESIGN.md
-            reading C30)                                abs <= 1e-5
+  W after the step where |g| > 1e-3 max|g|, within
+            1e-5 + lr |s(g_gpu) - s(g_ref)|, s(g) = g / (|g| + eps): the first
+            Adam step is exactly W - lr s(g), ill-conditioned where |g| ~ eps
+            (reading C30)
 rel(x, r) = max|x - r| / max|r|.  Partitioning is an exact re-organisation
 (§8(c)), so the same golden serves P = 1 and the loopback P = 8 split of
 north_star's 8-GPU target.  The inputs' fingerprints are checked first, so a
@@ -58,6 +59,17 @@ def check_inputs(meta, rp, col, X, y, Ws):
     assert [sha(W) for W in Ws] == meta["sha_W"], "weight generator drifted"
 
 
+def w_excess(g_ref, g_gpu, W_gpu, W_ref, lr=0.01, eps=1e-8):
+    """Reading C30: after Adam's first step from zero state W1 = W0 - lr g / (|g| + eps) exactly,
+    so where |g_ref| > 1e-3 max|g_ref| the two W may differ by lr |s(g_gpu) - s(g_ref)| (plus
+    fp32 rounding, 1e-5); returns the largest excess over that bound (<= 0 passes)."""
+    gr, gg = np.asarray(g_ref, np.float64), np.asarray(g_gpu, np.float64)
+    mask = np.abs(gr) > 1e-3 * np.abs(gr).max()
+    bound = 1e-5 + lr * np.abs(gg / (np.abs(gg) + eps) - gr / (np.abs(gr) + eps))
+    diff = np.abs(np.asarray(W_gpu, np.float64) - np.asarray(W_ref, np.float64))
+    return float((diff - bound)[mask].max())
+
+
 def compare_epoch(g, L, loss, WG, adam, Wn, logits_rows=None):
     out = {"loss": abs(loss - float(g["loss"])) / abs(float(g["loss"]))}
     if logits_rows is not None:
@@ -68,12 +80,10 @@ def compare_epoch(g, L, loss, WG, adam, Wn, logits_rows=None):
         assert t == 1
         out[f"m{l}"] = rel(mo, g[f"m{l}"])
         out[f"v{l}"] = rel(ve, g[f"v{l}"])
-        gg = g[f"WG{l}"]
-        mask = np.abs(gg) > max(1e-3 * np.abs(gg).max(), 100 * 1e-8)   # reading C30
-        out[f"W{l}_abs"] = float(np.abs(Wn[l][mask].astype(np.float64) - g[f"W{l}"][mask]).max())
+        out[f"W{l}_excess"] = w_excess(g[f"WG{l}"], WG[l], Wn[l], g[f"W{l}"])
     print(json.dumps(out))
     for k, v in out.items():
-        assert v <= (1e-5 if k.endswith("_abs") else REL_TOL), (k, v, out)
+        assert v <= (0.0 if k.endswith("_excess") else REL_TOL), (k, v, out)
     return out
 
 

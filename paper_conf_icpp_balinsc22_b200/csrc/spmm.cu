@@ -439,7 +439,7 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
     if ((flags & SPMM_ACCUM) && !(flags & SPMM_LAST)) t.n_items = t.n_items_nz;
     // Column windows of at most `win` floats.  The gathers are bound by the
     // SMs' L2 line rate; when the gathered block B_j is larger
-    // than half the L2, a 128-float window that fits it (n_j * 512 B <= L2) keeps the
+    // than 1.5x the L2, a 128-float window that fits it (n_j * 512 B <= L2) keeps the
     // slice L2-resident: same L2 traffic, 2.4x less DRAM traffic, 2 % faster
     // on Reddit-shaped B (profiles/r01_win_sweep.log).  Narrower windows
     // lose (extra index passes); a block that does not fit even at 128 floats
@@ -456,7 +456,10 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
     int win = win_env;
     if (win == 0) {
         const int64_t full = t.ncols * (int64_t)width * 4, w128 = t.ncols * 128 * 4;
-        win = (width > 128 && 2 * full > (int64_t)l2_bytes && w128 <= (int64_t)l2_bytes) ? 128 : 512;
+        // windows pay for their second index pass and launch only when the block is well beyond
+        // the L2: Reddit-shaped P = 1 (228 MB, 1.8x L2) gains 2 %, a 149 MB merged stage group
+        // (Reddit-shaped P = 8, 5 blocks) loses 6 % (profiles/r02_win_rule.log)
+        win = (width > 128 && 2 * full > 3 * (int64_t)l2_bytes && w128 <= (int64_t)l2_bytes) ? 128 : 512;
     }
     // L2 priority classes (tiles with hot_enc): when the gathered window does not
     // fit the L2, the rows of the most reused columns, up to hot_bytes of them,

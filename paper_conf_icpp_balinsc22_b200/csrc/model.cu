@@ -43,7 +43,8 @@ struct Bump {
 };
 
 struct HostItems {
-    std::vector<int4> items, splits;
+    std::vector<int4> items, splits;   // splits: the rows left to the fix-up kernel (> kFuseSegs segments)
+    std::vector<int4> segdesc;         // every split row {row, first_slot, nseg, fused}; segment items carry its index
     int64_t nslots = 0;
     int64_t n_nonempty = 0;   // items[0, n_nonempty): hub segments and non-empty rows; then empty rows
     int64_t split = kSplit;   // segment length used for this tile
@@ -63,14 +64,24 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
         if (split_env != 0 && (split_env < 32 || split_env > 65536)) split_env = 0;
     }
     const int64_t kSplit = split_env ? split_env : split_for(rp.back());
+    static int fuse_segs = -1;   // MGGCN_FUSED_FIXUP=0 sends every split row to the fix-up kernel
+    if (fuse_segs < 0) {
+        const char* e = getenv("MGGCN_FUSED_FIXUP");
+        fuse_segs = (e && atoi(e) == 0) ? 0 : kFuseSegs;
+    }
     for (int64_t r = 0; r < t.nrows; ++r) {
         const int64_t len = rp[r + 1] - rp[r];
         if (len > kSplit) {
             const int64_t nseg = (len + kSplit - 1) / kSplit;
-            h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
+            // rows of few segments are finished inside the stage kernel by the warp that completes
+            // their last segment (fused fix-up); longer ones keep the fix-up kernel
+            const bool fused = fuse_segs > 0 && nseg <= fuse_segs;
+            const int desc = (int)h.segdesc.size();
+            h.segdesc.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, fused ? 1 : 0));
+            if (!fused) h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
             for (int64_t s = 0; s < nseg; ++s) {
                 const int64_t b = rp[r] + s * kSplit, e = std::min<int64_t>(rp[r + 1], b + kSplit);
-                h.items.push_back(make_int4((int)r, (int)b, (int)e, (int)(h.nslots + s)));
+                h.items.push_back(make_int4(desc, (int)b, (int)e, (int)(h.nslots + s)));
             }
             h.nslots += nseg;
         }
@@ -216,6 +227,8 @@ struct Rank {
     std::vector<int32_t> order_cache;  // row order of the items (setup only)
     std::vector<float*> AHWB;
     float* spmm_partial = nullptr;
+    int32_t* seg_cnt = nullptr;      // fused fix-up: segments finished per split row (reset by the finisher)
+    int64_t n_seg_cnt = 0;
     double* ce_partial = nullptr;
     double* loss_local = nullptr;
     int64_t* ntrain_local = nullptr;
@@ -545,6 +558,8 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             t.n_slots = hi.nslots;
             t.items = b.take<int4>(hi.items.size());
             t.splits = b.take<int4>(hi.splits.size());
+            t.segdesc = b.take<int4>(hi.segdesc.size());
+            t.n_segdesc = (int64_t)hi.segdesc.size();
             t.col = b.take<int32_t>(ht.col.size());
             t.hot_enc = hot_ok && want_hot_classes(ht);
             t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
@@ -591,6 +606,17 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             if (!pt->shared_fb) slots = std::max(slots, r.hgB[g].nslots);
         }
         r.spmm_partial = b.take<float>(slots * std::min<int64_t>(m->bc_ld, 512));
+        int64_t ndesc = 0;
+        for (int j = 0; j < P; ++j) {
+            ndesc = std::max<int64_t>(ndesc, (int64_t)r.hF[j].segdesc.size());
+            if (!pt->shared_fb) ndesc = std::max<int64_t>(ndesc, (int64_t)r.hB[j].segdesc.size());
+        }
+        for (int g = 0; g < NG; ++g) {
+            ndesc = std::max<int64_t>(ndesc, (int64_t)r.hgF[g].segdesc.size());
+            if (!pt->shared_fb) ndesc = std::max<int64_t>(ndesc, (int64_t)r.hgB[g].segdesc.size());
+        }
+        r.seg_cnt = b.take<int32_t>(ndesc);
+        r.n_seg_cnt = ndesc;
         r.ce_partial = b.take<double>(kCeBlocks);
         r.WG_local = (m->nlocal > 1) ? b.take<float>(m->wtotal) : nullptr;
         // split-K partials for W_G (Eq. 10)
@@ -611,6 +637,9 @@ int upload_static(mggcn_model_s* m) {
                 if (!hi.splits.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.splits), hi.splits.data(),
                                        sizeof(int4) * hi.splits.size(), cudaMemcpyHostToDevice, m->cs));
+                if (!hi.segdesc.empty())
+                    CK(cudaMemcpyAsync(const_cast<int4*>(t.segdesc), hi.segdesc.data(),
+                                       sizeof(int4) * hi.segdesc.size(), cudaMemcpyHostToDevice, m->cs));
                 if (!ht.col.empty()) {
                     std::vector<int32_t> enc;
                     if (t.hot_enc) enc = encode_hot_classes(ht);
@@ -638,6 +667,7 @@ int upload_static(mggcn_model_s* m) {
         if (pt->shared_fb)
             for (size_t g = 0; g < r.GF.size(); ++g) r.GB[g] = r.GF[g];
         CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
+        if (r.n_seg_cnt) CK(cudaMemsetAsync(r.seg_cnt, 0, sizeof(int32_t) * r.n_seg_cnt, m->cs));
         // zero every activation buffer once: padding columns stay 0 forever
         for (int k = 0; k < 2; ++k) CK(cudaMemsetAsync(r.Xbuf[k], 0, sizeof(float) * r.rows * m->ld[0], m->cs));
         for (int l = 0; l < m->L; ++l)
@@ -853,7 +883,8 @@ int inject_delay(mggcn_model_s* m, cudaStream_t s) {
 
 int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
-    const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
+    SpmmTile t = job.dir == 0 ? r.F[j] : r.B[j];
+    t.seg_cnt = r.seg_cnt;
     float* out = job.dst(m, r, job.ctx);
     m->tl_stage = tl_k;
     m->tl_rank = (int32_t)(&r - &m->ranks[0]);
@@ -893,7 +924,8 @@ float* group_slot(mggcn_model_s* m, Rank& r, int k, int64_t width) {
 
 int launch_group(mggcn_model_s* m, Rank& r, const SpmmJob& job, int g, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
-    const SpmmTile& t = job.dir == 0 ? r.GF[g] : r.GB[g];
+    SpmmTile t = job.dir == 0 ? r.GF[g] : r.GB[g];
+    t.seg_cnt = r.seg_cnt;
     float* out = job.dst(m, r, job.ctx);
     m->tl_stage = tl_k;
     m->tl_rank = (int32_t)(&r - &m->ranks[0]);

@@ -64,10 +64,14 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
         if (split_env != 0 && (split_env < 32 || split_env > 65536)) split_env = 0;
     }
     const int64_t kSplit = split_env ? split_env : split_for(rp.back());
-    static int fuse_segs = -1;   // MGGCN_FUSED_FIXUP=0 sends every split row to the fix-up kernel
+    // MGGCN_FUSED_FIXUP=1: split rows of <= kFuseSegs segments are finished inside the stage
+    // kernel.  Opt-in: parity-green, but not faster (SOLO Reddit-shaped P = 8: 3.74 vs 3.71 ms;
+    // the finishing warps lengthen the stage tail as much as the fix-up launches cost;
+    // profiles/r02_fused_fixup_ab.log)
+    static int fuse_segs = -1;
     if (fuse_segs < 0) {
         const char* e = getenv("MGGCN_FUSED_FIXUP");
-        fuse_segs = (e && atoi(e) == 0) ? 0 : kFuseSegs;
+        fuse_segs = (e && atoi(e) != 0) ? kFuseSegs : 0;
     }
     for (int64_t r = 0; r < t.nrows; ++r) {
         const int64_t len = rp[r + 1] - rp[r];

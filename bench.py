@@ -416,7 +416,7 @@ def run_reference(args):
     line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": statistics.median(walls) * 1e3,
             "higher_is_better": False, "scaling": "strong", "vs_baseline": None, "dtype": "f32 storage, f64 accumulate",
-            "data": "synthetic", "config": workload_desc(w, 1),
+            "data": "synthetic", "config": workload_desc(w, args.gpus),
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
                              "estimated": True, "rows_sampled": R, "sampled_estimate_ms": raw, "calibration": cal,
                              "host": host_info()},
@@ -727,11 +727,11 @@ def main():
         "metric": METRIC, "value": ms_max, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_max, "higher_is_better": False, "scaling": "strong",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": workload_desc(w, P) | {"overlap": not args.no_overlap,
-                                         "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)",
-                                         "comm": (args.comm if P > 1 else "none"),
-                                         "parallelism": (f"dp{P} (1D row partition)" if args.replicas == 1 else
-                                                         f"dp{P} (1.5D: {P // 2} row blocks x 2 replicas)")},
+        "config": workload_desc(w, P),
+        "run": {"overlap": not args.no_overlap, "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)",
+                "comm": (args.comm if P > 1 else "none"),
+                "parallelism": (f"dp{P} (1D row partition)" if args.replicas == 1 else
+                                f"dp{P} (1.5D: {P // 2} row blocks x 2 replicas)")},
         "timing": ("K replays of the captured epoch (mggcn_epoch_replay), CUDA events on the compute stream"
                    if gtime is not None else "K eager forward/backward/step epochs, CUDA events on the compute stream"),
         "eager_ms": ms_eager,

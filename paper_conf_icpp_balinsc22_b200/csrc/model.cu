@@ -8,6 +8,7 @@
 // the P-stage pipeline on one GPU, LOOPBACK (all P ranks in this model,
 // broadcasts = device copies on the comm stream with the same event graph).
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <chrono>
@@ -448,14 +449,24 @@ cudaEvent_t prof_event(mggcn_model_s* m) {
     return e;
 }
 
+// NVTX range names per op class (ranges for nsys / ncu --nvtx; no-ops without a tool)
+const char* const kNvtxName[PC_N] = {"mggcn:spmm", "mggcn:gemm", "mggcn:loss", "mggcn:adam", "mggcn:bcast",
+                                     "mggcn:allreduce", "mggcn:other"};
+
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
 struct ProfScope {
+    NvtxRange nvtx;
     mggcn_model_s* m;
     int cls;
     cudaStream_t s;
     cudaEvent_t a = nullptr;     // MGGCN_F_PROFILE pair (consumed by mggcn_get_profile)
     cudaEvent_t ta = nullptr;    // MGGCN_F_TIMELINE pair (consumed by mggcn_get_timeline)
     int32_t meta[5];
-    ProfScope(mggcn_model_s* m_, int c, cudaStream_t s_) : m(m_), cls(c), s(s_) {
+    ProfScope(mggcn_model_s* m_, int c, cudaStream_t s_) : nvtx(kNvtxName[c]), m(m_), cls(c), s(s_) {
         if (m->capturing) return;   // a captured epoch is timed as a whole
         if (m->flags & MGGCN_F_PROFILE) {
             a = prof_event(m);
@@ -2075,6 +2086,7 @@ static int forward_impl(mggcn_model_s* m, const float* X, int64_t ldx, const int
 
 extern "C" int mggcn_forward(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local, float* loss,
                              float* logits_local) {
+    NvtxRange nvtx_top("mggcn_forward");
     MODEL_GUARD(m);
     if (!X_local) {
         if (m->pref_buf < 0) {
@@ -2222,6 +2234,7 @@ static int backward_impl(mggcn_model_s* m) {
 }
 
 extern "C" int mggcn_backward(mggcn_model m) {
+    NvtxRange nvtx_top("mggcn_backward");
     MODEL_GUARD(m);
     if (m->state != ST_FWD) {
         set_error("backward: needs a preceding forward");
@@ -2247,6 +2260,7 @@ static int step_impl(mggcn_model_s* m, float lr, float beta1, float beta2, float
 }
 
 extern "C" int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps) {
+    NvtxRange nvtx_top("mggcn_step");
     MODEL_GUARD(m);
     if (int rc = poll_comm_errors(m)) return poison(m, rc);   // non-blocking
     if (m->state != ST_BWD) {

@@ -335,6 +335,15 @@ int mggcn_debug_layer(mggcn_model m, int32_t layer, float* dst, int64_t ld);
  * streams interleave differently from run to run; results must not change.
  * max_us = 0 turns it off.  EINVAL: max_us outside [0, 10000]. */
 int mggcn_debug_comm_delay(mggcn_model m, uint64_t seed, int32_t max_us);
+/* mggcn_debug_poison: poison-buffer injection.  With on != 0 the
+ * comm stream fills every BC slot with NaN bytes right before the broadcast,
+ * copy or pull into it, so a SpMM stage that read a slot outside the P:939-941
+ * event rule yields NaN rows instead of silently reusing stale data.  Results
+ * of a correct schedule do not change.  on = 2 is the negative control: it
+ * also drops the compute stream's wait for each broadcast, so stages race the
+ * exchange and the poison must show up (tests prove the check has teeth).
+ * Test hook.  EINVAL: on outside [0, 2]. */
+int mggcn_debug_poison(mggcn_model m, int32_t on);
 
 #ifdef __cplusplus
 }

@@ -39,7 +39,7 @@ EXPORTS = (
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
     "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
     "mggcn_epoch_replay", "mggcn_debug_comm_delay", "mggcn_get_timeline",
-    "mggcn_epoch_work_detail", "mggcn_timeline_enable",
+    "mggcn_epoch_work_detail", "mggcn_timeline_enable", "mggcn_debug_poison",
 )
 
 
@@ -86,6 +86,7 @@ def _load():
         "mggcn_get_profile": ([P, P, P, i32], ctypes.c_int),
         "mggcn_get_timeline": ([P, i64, P, P, P, i32], ctypes.c_int),
         "mggcn_timeline_enable": ([P, i32], ctypes.c_int),
+        "mggcn_debug_poison": ([P, i32], ctypes.c_int),
         "mggcn_epoch_work": ([P, P, P, P, P], ctypes.c_int),
         "mggcn_epoch_work_detail": ([P, P, i32], ctypes.c_int),
         "mggcn_graph_free": ([P], None),
@@ -367,6 +368,11 @@ def mggcn_debug_spmm(m, direction, B, ldb, width, out, ldo):
 
 def mggcn_debug_comm_delay(m, seed, max_us):
     _check(_lib.mggcn_debug_comm_delay(m, seed, max_us))
+
+
+def mggcn_debug_poison(m, on=1):
+    """1: NaN-fill BC slots before they are filled; 2: also drop the broadcast waits (negative control)."""
+    _check(_lib.mggcn_debug_poison(m, int(on)))
 
 
 def mggcn_debug_layer(m, layer, shape):

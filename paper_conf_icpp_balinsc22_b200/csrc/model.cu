@@ -317,6 +317,8 @@ struct mggcn_model_s {
     // delay injection (mggcn_debug_comm_delay): spin kernels of pseudo-random length
     uint64_t delay_seed = 0, delay_ctr = 0;
     int32_t delay_max_us = 0;
+    bool poison_bc = false;         // mggcn_debug_poison: NaN-fill every BC slot right before it is filled
+    bool break_bc_wait = false;     // mggcn_debug_poison(m, 2): negative control, stages skip the broadcast wait
     size_t ws_bytes = 0;             // planned workspace bytes
     size_t sym_bytes = 0;            // symmetric region [0, sym_bytes) (IPC peers must agree)
     uint32_t spmm_seq = 0, wg_seq = 0, sc_seq = 0;
@@ -896,6 +898,20 @@ int inject_delay(mggcn_model_s* m, cudaStream_t s) {
     return MGGCN_OK;
 }
 
+// poison-buffer injection (mggcn_debug_poison): the comm stream NaN-fills a BC slot right
+// before the broadcast / copy / pull into it, so a stage that read a slot outside the
+// P:939-941 event rule would turn its rows into NaN instead of silently reading stale data
+int poison_slot(mggcn_model_s* m, void* p, size_t bytes) {
+    if (m->poison_bc && bytes) CK(cudaMemsetAsync(p, 0xFF, bytes, m->ms));
+    return MGGCN_OK;
+}
+
+// compute-stream wait for a broadcast / pull (skipped only by the negative-control hook)
+int wait_bc(mggcn_model_s* m, cudaEvent_t e) {
+    if (!m->break_bc_wait) CK(cudaStreamWaitEvent(m->cs, e, 0));
+    return MGGCN_OK;
+}
+
 int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
     SpmmTile t = job.dir == 0 ? r.F[j] : r.B[j];
@@ -979,13 +995,14 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
                 RC(inject_delay(m, m->ms));
                 CK(stream_wait_u32(m->ms, peer_ptr(m, q, m->flags_dev) + 0, seq));   // block q is ready
                 const size_t bytes = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width * sizeof(float);
+                if (!nob && bytes) RC(poison_slot(m, group_slot(m, r, k, job.width), bytes));
                 if (!nob && bytes)
                     CK(cudaMemcpyAsync(group_slot(m, r, k, job.width), peer_ptr(m, q, mysrc), bytes, cudaMemcpyDefault,
                                        m->ms));
                 if (last) CK(cudaEventRecord(r.ev_bc[g & 1], m->ms));
             }
             if (last) {
-                CK(cudaStreamWaitEvent(m->cs, r.ev_bc[g & 1], 0));
+                RC(wait_bc(m, r.ev_bc[g & 1]));
                 if (r.rows > 0) RC(launch_group(m, r, job, g, SPMM_ACCUM | (g == NG - 1 ? SPMM_LAST : 0), q));
                 RC(mark_stage(m));
             }
@@ -1001,10 +1018,11 @@ int staged_spmm_ipc(mggcn_model_s* m, const SpmmJob& job) {
             if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
             CK(stream_wait_u32(m->ms, peer_ptr(m, q, m->flags_dev) + 0, seq));   // block q is ready
             const size_t bytes = (size_t)(r.part->p[q + 1] - r.part->p[q]) * (size_t)job.width * sizeof(float);
+            if (!nob && bytes) RC(poison_slot(m, r.BC[slot], bytes));
             if (!nob && bytes) CK(cudaMemcpyAsync(r.BC[slot], peer_ptr(m, q, mysrc), bytes, cudaMemcpyDefault, m->ms));
             CK(cudaEventRecord(r.ev_bc[slot], m->ms));
         }
-        CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
+        RC(wait_bc(m, r.ev_bc[slot]));
         if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], SPMM_ACCUM | (st == P - 1 ? SPMM_LAST : 0), q));
         CK(cudaEventRecord(r.ev_free[slot], m->cs));
         RC(mark_stage(m));
@@ -1061,6 +1079,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
                     } else {
                         const int k = remote_index_15d(m, q, r), slot = k & 1;
                         if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                        if (!nob && count) RC(poison_slot(m, r.BC[slot], count * sizeof(float)));
                         if (!nob && count)
                             NK(ncclBroadcast(r.BC[slot], r.BC[slot], count, ncclFloat32, q, m->comm_bc, m->ms));
                         CK(cudaEventRecord(r.ev_bc[slot], m->ms));
@@ -1073,6 +1092,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
                     if (r.rep != rq || r.rank == q) continue;
                     const int k = remote_index_15d(m, q, r), slot = k & 1;
                     if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (!nob && bytes) RC(poison_slot(m, r.BC[slot], bytes));
                     if (!nob && bytes)
                         CK(cudaMemcpyAsync(r.BC[slot], job.src(m, root, job.ctx), bytes, cudaMemcpyDeviceToDevice,
                                            m->ms));
@@ -1084,7 +1104,7 @@ int staged_spmm_15d(mggcn_model_s* m, const SpmmJob& job) {
             Rank& r = m->ranks[i];
             if (r.rep != rq || r.rank == q) continue;
             const int k = remote_index_15d(m, q, r), slot = k & 1;
-            CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
+            RC(wait_bc(m, r.ev_bc[slot]));
             if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], started[i] ? SPMM_ACCUM : 0, q));
             started[i] = 1;
             CK(cudaEventRecord(r.ev_free[slot], m->cs));
@@ -1146,6 +1166,7 @@ int staged_spmm_grouped(mggcn_model_s* m, const SpmmJob& job) {
                 } else {
                     const int k = remote_index(q, r.rank);
                     float* dst = group_slot(m, r, k, job.width);
+                    if (!nob && count) RC(poison_slot(m, dst, count * sizeof(float)));
                     if (!nob && count) NK(ncclBroadcast(dst, dst, count, ncclFloat32, q, m->comm, m->ms));
                     if (last_of_group(m, k)) CK(cudaEventRecord(r.ev_bc[group_of(m, k) & 1], m->ms));
                 }
@@ -1155,6 +1176,7 @@ int staged_spmm_grouped(mggcn_model_s* m, const SpmmJob& job) {
                 for (auto& r : m->ranks) {
                     if (r.rank == q) continue;
                     const int k = remote_index(q, r.rank);
+                    if (!nob && bytes) RC(poison_slot(m, group_slot(m, r, k, job.width), bytes));
                     if (!nob && bytes)
                         CK(cudaMemcpyAsync(group_slot(m, r, k, job.width), job.src(m, root, job.ctx), bytes,
                                            cudaMemcpyDeviceToDevice, m->ms));
@@ -1167,7 +1189,7 @@ int staged_spmm_grouped(mggcn_model_s* m, const SpmmJob& job) {
             const int k = remote_index(q, r.rank);
             if (!last_of_group(m, k)) continue;
             const int g = group_of(m, k);
-            CK(cudaStreamWaitEvent(m->cs, r.ev_bc[g & 1], 0));
+            RC(wait_bc(m, r.ev_bc[g & 1]));
             if (r.rows > 0) RC(launch_group(m, r, job, g, SPMM_ACCUM | (g == NG - 1 ? SPMM_LAST : 0), q));
         }
         RC(mark_stage(m));
@@ -1211,6 +1233,7 @@ int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
                 } else {
                     const int k = remote_index(q, r.rank), slot = k & 1;
                     if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (!nob && count) RC(poison_slot(m, r.BC[slot], count * sizeof(float)));
                     if (!nob && count) NK(ncclBroadcast(r.BC[slot], r.BC[slot], count, ncclFloat32, q, m->comm, m->ms));
                     CK(cudaEventRecord(r.ev_bc[slot], m->ms));
                 }
@@ -1221,6 +1244,7 @@ int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
                     if (r.rank == q) continue;
                     const int k = remote_index(q, r.rank), slot = k & 1;
                     if (k >= 2) CK(cudaStreamWaitEvent(m->ms, r.ev_free[slot], 0));
+                    if (!nob && bytes) RC(poison_slot(m, r.BC[slot], bytes));
                     if (!nob && bytes)
                         CK(cudaMemcpyAsync(r.BC[slot], job.src(m, root, job.ctx), bytes, cudaMemcpyDeviceToDevice,
                                            m->ms));
@@ -1232,7 +1256,7 @@ int staged_spmm_impl(mggcn_model_s* m, const SpmmJob& job) {
         for (auto& r : m->ranks) {
             if (r.rank == q) continue;
             const int k = remote_index(q, r.rank), slot = k & 1;
-            CK(cudaStreamWaitEvent(m->cs, r.ev_bc[slot], 0));
+            RC(wait_bc(m, r.ev_bc[slot]));
             const int last_q = (r.rank == P - 1) ? P - 2 : P - 1;
             const int flags = SPMM_ACCUM | (q == last_q ? SPMM_LAST : 0);
             if (r.rows > 0) RC(launch_stage(m, r, job, q, r.BC[slot], flags, q));
@@ -2431,6 +2455,17 @@ extern "C" int mggcn_get_profile(mggcn_model m, double* ms, int64_t* launches, i
             m->prof_n[c] = 0;
         }
     }
+    return MGGCN_OK;
+}
+
+extern "C" int mggcn_debug_poison(mggcn_model m, int32_t on) {
+    MODEL_GUARD(m);
+    if (on < 0 || on > 2) {
+        set_error("debug_poison: on must be 0, 1 or 2");
+        return MGGCN_EINVAL;
+    }
+    m->poison_bc = on != 0;
+    m->break_bc_wait = on == 2;
     return MGGCN_OK;
 }
 

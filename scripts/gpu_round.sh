@@ -32,7 +32,7 @@ case $STEP in
   profile)
     bash scripts/profile_round.sh $TAG ${1:-reddit} ;;
   sanitize)
-    for tool in memcheck racecheck synccheck; do
+    for tool in memcheck racecheck synccheck initcheck; do
       timeout -s KILL 1500 compute-sanitizer --tool $tool --error-exitcode 9 --print-limit 20 \
         python scripts/sanitize.py > gpurun_out/${TAG}_sanitize_$tool.log 2>&1
       echo "$tool rc=$?"; grep -E "ERROR SUMMARY" gpurun_out/${TAG}_sanitize_$tool.log | tail -1

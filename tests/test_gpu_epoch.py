@@ -27,11 +27,13 @@ def mg():
 
 
 def run_library(mg, n, rp, col, vals, X, y, Ws, dims, P, seed, flags, host_inputs=False, steps=1, lr=0.01,
-                delay=None, replicas=1):
+                delay=None, replicas=1, poison=False):
     from paper_conf_icpp_balinsc22_b200 import GCN
     gm = GCN(n, rp, col, vals, dims, P=P, perm_seed=seed, flags=flags, loopback=P > 1, replicas=replicas)
     if delay is not None:                       # (seed, max_us): spin kernels on both streams
         mg.mggcn_debug_comm_delay(gm.m, *delay)
+    if poison:                                  # NaN-fill every BC slot right before it is filled
+        mg.mggcn_debug_poison(gm.m, int(poison))
     gm.set_weights(Ws)
     Xl = gm.permute_rows(X)
     yl = gm.permute_rows(y)
@@ -395,8 +397,9 @@ def test_solo_timing_mode_on_disconnected_halves(mg, dims):
 def test_delay_injection_keeps_results_bitwise(mg, P, replicas):
     """SURVEY §4 pipeline-logic test: spin kernels of pseudo-random length (0..200 us) before
     every broadcast (comm stream) and every SpMM stage (compute stream) reshuffle how the
-    two streams interleave; the P:929-941 event rule must keep logits, loss, W_G and the
-    updated W bitwise equal to the undelayed run, for several seeds, 1D and 1.5D."""
+    two streams interleave, and every BC slot is NaN-poisoned right before it is filled; the
+    P:929-941 event rule must keep logits, loss, W_G and the updated W bitwise equal to the
+    undelayed run, for several seeds, 1D and 1.5D."""
     n, m = 1500, 30000
     rp, col = gen.rmat_csr(n, m, 71)
     dims = (24, 48, 9)
@@ -406,7 +409,7 @@ def test_delay_injection_keeps_results_bitwise(mg, P, replicas):
     base = run_library(mg, n, rp, col, None, X, y, Ws, dims, P, 75, mg.MGGCN_F_OVERLAP, steps=2, replicas=replicas)
     for seed in (1, 2, 3):
         d = run_library(mg, n, rp, col, None, X, y, Ws, dims, P, 75, mg.MGGCN_F_OVERLAP, steps=2,
-                        delay=(seed, 200), replicas=replicas)
+                        delay=(seed, 200), replicas=replicas, poison=True)
         assert np.array_equal(base["logits"], d["logits"])
         assert base["loss"] == d["loss"]
         for a, b in zip(base["WG"], d["WG"]):
@@ -484,7 +487,27 @@ def test_stage_group_sizes_epoch(mg, monkeypatch, var, group):
     ref = oracle.epoch(oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed), X, y, Ws)
     a = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 8, w.perm_seed, mg.MGGCN_F_OVERLAP)
     compare(a, ref, w.dims)
-    b = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 8, w.perm_seed, mg.MGGCN_F_OVERLAP, delay=(9, 150))
+    b = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 8, w.perm_seed, mg.MGGCN_F_OVERLAP, delay=(9, 150),
+                    poison=True)
     assert np.array_equal(a["logits"], b["logits"]) and a["loss"] == b["loss"]
     for u, v in zip(a["W"], b["W"]):
         assert np.array_equal(u, v)
+
+
+@pytest.mark.parametrize("group", ["1", None])
+def test_poison_negative_control(mg, monkeypatch, group):
+    """The poison check has teeth: with the compute stream's broadcast waits dropped
+    (mggcn_debug_poison(m, 2)) and long spins on the comm stream, stages read BC slots that
+    were NaN-filled but not yet refilled, so the epoch's logits are no longer the oracle's;
+    the same run with the waits kept (poison 1) is bitwise equal to the clean run."""
+    if group:
+        monkeypatch.setenv("MGGCN_STAGE_GROUP", group)
+    w = gen.WORKLOADS["cora"]
+    rp, col, X, y, Ws = workload_inputs(w)
+    clean = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 4, w.perm_seed, mg.MGGCN_F_OVERLAP)
+    good = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 4, w.perm_seed, mg.MGGCN_F_OVERLAP,
+                       delay=(3, 2000), poison=1)
+    assert np.array_equal(clean["logits"], good["logits"])
+    bad = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 4, w.perm_seed, mg.MGGCN_F_OVERLAP,
+                      delay=(3, 2000), poison=2)
+    assert not np.array_equal(np.nan_to_num(bad["logits"], nan=1e30), clean["logits"])

@@ -340,8 +340,9 @@ int mggcn_debug_comm_delay(mggcn_model m, uint64_t seed, int32_t max_us);
  * copy or pull into it, so a SpMM stage that read a slot outside the P:939-941
  * event rule yields NaN rows instead of silently reusing stale data.  Results
  * of a correct schedule do not change.  on = 2 is the negative control: it
- * also drops the compute stream's wait for each broadcast, so stages race the
- * exchange and the poison must show up (tests prove the check has teeth).
+ * also drops the compute stream's wait for each broadcast (and the compute-side
+ * delay spins), so stages race the delayed exchange and the poison must show up
+ * (tests prove the check has teeth).
  * Test hook.  EINVAL: on outside [0, 2]. */
 int mggcn_debug_poison(mggcn_model m, int32_t on);
 

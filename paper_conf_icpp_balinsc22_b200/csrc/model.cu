@@ -890,6 +890,7 @@ struct SpmmJob {
 // delay injection: a spin of 0..delay_max_us on stream s (test hook, P:929-941 rule check)
 int inject_delay(mggcn_model_s* m, cudaStream_t s) {
     if (m->delay_max_us <= 0) return MGGCN_OK;
+    if (m->break_bc_wait && s == m->cs) return MGGCN_OK;   // negative control: only the exchange is late
     uint64_t z = m->delay_seed + 0x9E3779B97F4A7C15ull * (++m->delay_ctr);
     z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
     z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;

@@ -1,6 +1,7 @@
 """Small end-to-end run for compute-sanitizer: loopback P=2 Cora-shaped epoch,
 an SpMM-first config (112 classes: the 32-lane CE row groups), a 1.5D loopback
-epoch (MGGCN_F_REPL2, P = 4), and the three GEMM ops (ragged shapes)."""
+epoch (MGGCN_F_REPL2, P = 4), a loopback P = 8 epoch with the default stage
+groups and NaN-poisoned BC slots, and the three GEMM ops (ragged shapes)."""
 import os, sys
 import numpy as np, torch
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -8,13 +9,15 @@ import gen
 import paper_conf_icpp_balinsc22_b200 as mg
 from paper_conf_icpp_balinsc22_b200 import GCN
 for dims, P, n, m, c in (((1433, 16, 7), 2, 2708, 10556, 1), ((8, 128, 128, 112), 1, 3001, 60000, 1),
-                         ((100, 64, 47), 4, 3001, 60000, 2)):
+                         ((100, 64, 47), 4, 3001, 60000, 2), ((64, 48, 41), 8, 4001, 200000, 1)):
     rp, col = gen.rmat_csr(n, m, 5)
     X = gen.features(n, dims[0], 6); y = gen.labels(n, dims[-1], 7, 100)
     Ws = [gen.glorot(dims[l], dims[l + 1], 8 + l) for l in range(len(dims) - 1)]
     gm = GCN(n, rp, col, None, dims, P=P, perm_seed=9, loopback=P > 1, flags=mg.MGGCN_F_OVERLAP | mg.MGGCN_F_PROFILE,
              replicas=c)
     gm.set_weights(Ws)
+    if P == 8:
+        mg.mggcn_debug_poison(gm.m, 1)
     for host in (False, True):
         Xl, yl = gm.permute_rows(X), gm.permute_rows(y)
         Xin = Xl if host else torch.from_numpy(Xl).cuda()

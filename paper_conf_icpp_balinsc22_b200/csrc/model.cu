@@ -685,6 +685,8 @@ int upload_static(mggcn_model_s* m) {
             for (size_t g = 0; g < r.GF.size(); ++g) r.GB[g] = r.GF[g];
         CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
         if (r.n_seg_cnt) CK(cudaMemsetAsync(r.seg_cnt, 0, sizeof(int32_t) * r.n_seg_cnt, m->cs));
+        // loopback W_G partials: the padding columns (ld > d) are summed with the rest (initcheck)
+        if (r.WG_local) CK(cudaMemsetAsync(r.WG_local, 0, sizeof(float) * m->wtotal, m->cs));
         // zero every activation buffer once: padding columns stay 0 forever
         for (int k = 0; k < 2; ++k) CK(cudaMemsetAsync(r.Xbuf[k], 0, sizeof(float) * r.rows * m->ld[0], m->cs));
         for (int l = 0; l < m->L; ++l)

@@ -46,6 +46,7 @@ struct Bump {
 struct HostItems {
     std::vector<int4> items, splits;   // splits: the rows left to the fix-up kernel (> kFuseSegs segments)
     std::vector<int4> segdesc;         // every split row {row, first_slot, nseg, fused}; segment items carry its index
+    bool any_fused = false;            // segdesc is uploaded (and read by the kernel) only then
     int64_t nslots = 0;
     int64_t n_nonempty = 0;   // items[0, n_nonempty): hub segments and non-empty rows; then empty rows
     int64_t split = kSplit;   // segment length used for this tile
@@ -81,6 +82,7 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
             // rows of few segments are finished inside the stage kernel by the warp that completes
             // their last segment (fused fix-up); longer ones keep the fix-up kernel
             const bool fused = fuse_segs > 0 && nseg <= fuse_segs;
+            h.any_fused = h.any_fused || fused;
             const int desc = (int)h.segdesc.size();
             h.segdesc.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, fused ? 1 : 0));
             if (!fused) h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
@@ -575,8 +577,9 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             t.n_slots = hi.nslots;
             t.items = b.take<int4>(hi.items.size());
             t.splits = b.take<int4>(hi.splits.size());
-            t.segdesc = b.take<int4>(hi.segdesc.size());
-            t.n_segdesc = (int64_t)hi.segdesc.size();
+            // without fused rows the kernel never reads the descriptors (a dependent load per segment)
+            t.segdesc = hi.any_fused ? b.take<int4>(hi.segdesc.size()) : nullptr;
+            t.n_segdesc = hi.any_fused ? (int64_t)hi.segdesc.size() : 0;
             t.col = b.take<int32_t>(ht.col.size());
             t.hot_enc = hot_ok && want_hot_classes(ht);
             t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
@@ -654,7 +657,7 @@ int upload_static(mggcn_model_s* m) {
                 if (!hi.splits.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.splits), hi.splits.data(),
                                        sizeof(int4) * hi.splits.size(), cudaMemcpyHostToDevice, m->cs));
-                if (!hi.segdesc.empty())
+                if (t.segdesc && !hi.segdesc.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.segdesc), hi.segdesc.data(),
                                        sizeof(int4) * hi.segdesc.size(), cudaMemcpyHostToDevice, m->cs));
                 if (!ht.col.empty()) {

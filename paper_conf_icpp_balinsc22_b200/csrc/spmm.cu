@@ -279,7 +279,7 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
             }
             // fused fix-up (SpmmTile::segdesc): the warp that completes the last segment of a
             // short split row sums its partials in segment order and finishes the row
-            const int4 sd = __ldg(segdesc + it.x);
+            const int4 sd = segdesc ? __ldg(segdesc + it.x) : make_int4(0, 0, 0, 0);
             if (sd.w) {
                 __threadfence();                       // release this lane's part of the partial
                 __syncwarp();                          // ... every lane's, before lane 0 counts it

@@ -21,7 +21,6 @@ cudaError_t launch_spin(uint64_t ns, cudaStream_t s);
 // segment order by a fix-up kernel (deterministic, no float atomics).
 constexpr int kSplit = 2048;      // longest segment
 constexpr int kSplitMin = 128;    // shortest segment (small tiles, e.g. Reddit-shaped at P = 8)
-constexpr int kFuseSegs = 8;      // split rows of <= 8 segments are finished inside the stage kernel
 
 // Segment length of a tile with nnz entries: the longest work item is one warp
 // walking a segment, so a short stage (a small tile) needs short segments or
@@ -37,16 +36,8 @@ struct SpmmTile {
     const int4* items = nullptr;   // {row, beg, end, slot}
     int64_t n_items = 0;
     int64_t n_items_nz = 0;        // items[0, n_items_nz) are hub segments and non-empty rows, the rest empty rows
-    const int4* splits = nullptr;  // {row, first_slot, nslots, 0}: rows left to the fix-up kernel
+    const int4* splits = nullptr;  // {row, first_slot, nslots, 0}
     int64_t n_splits = 0;
-    // every split row {row, first_slot, nseg, fused}; a segment item {desc, beg, end, slot} names
-    // its row's descriptor.  Fused rows (nseg <= kFuseSegs) are finished by the warp that
-    // completes their last segment: it counts segments in seg_cnt[desc] (atomicAdd after a
-    // __threadfence), and the last one sums the partials in segment order, applies the epilogue
-    // and resets the counter.
-    const int4* segdesc = nullptr;
-    int64_t n_segdesc = 0;
-    int32_t* seg_cnt = nullptr;
     int64_t n_slots = 0;
     int64_t split = kSplit;        // segment length of this tile (split_for); short segments
                                    // (a small tile) => many per row => block-per-row fix-up

@@ -44,9 +44,7 @@ struct Bump {
 };
 
 struct HostItems {
-    std::vector<int4> items, splits;   // splits: the rows left to the fix-up kernel (> kFuseSegs segments)
-    std::vector<int4> segdesc;         // every split row {row, first_slot, nseg, fused}; segment items carry its index
-    bool any_fused = false;            // segdesc is uploaded (and read by the kernel) only then
+    std::vector<int4> items, splits;
     int64_t nslots = 0;
     int64_t n_nonempty = 0;   // items[0, n_nonempty): hub segments and non-empty rows; then empty rows
     int64_t split = kSplit;   // segment length used for this tile
@@ -66,29 +64,14 @@ void build_items(const HostTile& t, HostItems& h, const std::vector<int32_t>& or
         if (split_env != 0 && (split_env < 32 || split_env > 65536)) split_env = 0;
     }
     const int64_t kSplit = split_env ? split_env : split_for(rp.back());
-    // MGGCN_FUSED_FIXUP=1: split rows of <= kFuseSegs segments are finished inside the stage
-    // kernel.  Opt-in: parity-green, but not faster (SOLO Reddit-shaped P = 8: 3.74 vs 3.71 ms;
-    // the finishing warps lengthen the stage tail as much as the fix-up launches cost;
-    // profiles/r02_fused_fixup_ab.log)
-    static int fuse_segs = -1;
-    if (fuse_segs < 0) {
-        const char* e = getenv("MGGCN_FUSED_FIXUP");
-        fuse_segs = (e && atoi(e) != 0) ? kFuseSegs : 0;
-    }
     for (int64_t r = 0; r < t.nrows; ++r) {
         const int64_t len = rp[r + 1] - rp[r];
         if (len > kSplit) {
             const int64_t nseg = (len + kSplit - 1) / kSplit;
-            // rows of few segments are finished inside the stage kernel by the warp that completes
-            // their last segment (fused fix-up); longer ones keep the fix-up kernel
-            const bool fused = fuse_segs > 0 && nseg <= fuse_segs;
-            h.any_fused = h.any_fused || fused;
-            const int desc = (int)h.segdesc.size();
-            h.segdesc.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, fused ? 1 : 0));
-            if (!fused) h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
+            h.splits.push_back(make_int4((int)r, (int)h.nslots, (int)nseg, 0));
             for (int64_t s = 0; s < nseg; ++s) {
                 const int64_t b = rp[r] + s * kSplit, e = std::min<int64_t>(rp[r + 1], b + kSplit);
-                h.items.push_back(make_int4(desc, (int)b, (int)e, (int)(h.nslots + s)));
+                h.items.push_back(make_int4((int)r, (int)b, (int)e, (int)(h.nslots + s)));
             }
             h.nslots += nseg;
         }
@@ -234,8 +217,6 @@ struct Rank {
     std::vector<int32_t> order_cache;  // row order of the items (setup only)
     std::vector<float*> AHWB;
     float* spmm_partial = nullptr;
-    int32_t* seg_cnt = nullptr;      // fused fix-up: segments finished per split row (reset by the finisher)
-    int64_t n_seg_cnt = 0;
     double* ce_partial = nullptr;
     double* loss_local = nullptr;
     int64_t* ntrain_local = nullptr;
@@ -577,9 +558,6 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             t.n_slots = hi.nslots;
             t.items = b.take<int4>(hi.items.size());
             t.splits = b.take<int4>(hi.splits.size());
-            // without fused rows the kernel never reads the descriptors (a dependent load per segment)
-            t.segdesc = hi.any_fused ? b.take<int4>(hi.segdesc.size()) : nullptr;
-            t.n_segdesc = hi.any_fused ? (int64_t)hi.segdesc.size() : 0;
             t.col = b.take<int32_t>(ht.col.size());
             t.hot_enc = hot_ok && want_hot_classes(ht);
             t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
@@ -626,17 +604,6 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             if (!pt->shared_fb) slots = std::max(slots, r.hgB[g].nslots);
         }
         r.spmm_partial = b.take<float>(slots * std::min<int64_t>(m->bc_ld, 512));
-        int64_t ndesc = 0;
-        for (int j = 0; j < P; ++j) {
-            ndesc = std::max<int64_t>(ndesc, (int64_t)r.hF[j].segdesc.size());
-            if (!pt->shared_fb) ndesc = std::max<int64_t>(ndesc, (int64_t)r.hB[j].segdesc.size());
-        }
-        for (int g = 0; g < NG; ++g) {
-            ndesc = std::max<int64_t>(ndesc, (int64_t)r.hgF[g].segdesc.size());
-            if (!pt->shared_fb) ndesc = std::max<int64_t>(ndesc, (int64_t)r.hgB[g].segdesc.size());
-        }
-        r.seg_cnt = b.take<int32_t>(ndesc);
-        r.n_seg_cnt = ndesc;
         r.ce_partial = b.take<double>(kCeBlocks);
         r.WG_local = (m->nlocal > 1) ? b.take<float>(m->wtotal) : nullptr;
         // split-K partials for W_G (Eq. 10)
@@ -657,9 +624,6 @@ int upload_static(mggcn_model_s* m) {
                 if (!hi.splits.empty())
                     CK(cudaMemcpyAsync(const_cast<int4*>(t.splits), hi.splits.data(),
                                        sizeof(int4) * hi.splits.size(), cudaMemcpyHostToDevice, m->cs));
-                if (t.segdesc && !hi.segdesc.empty())
-                    CK(cudaMemcpyAsync(const_cast<int4*>(t.segdesc), hi.segdesc.data(),
-                                       sizeof(int4) * hi.segdesc.size(), cudaMemcpyHostToDevice, m->cs));
                 if (!ht.col.empty()) {
                     std::vector<int32_t> enc;
                     if (t.hot_enc) enc = encode_hot_classes(ht);
@@ -687,7 +651,6 @@ int upload_static(mggcn_model_s* m) {
         if (pt->shared_fb)
             for (size_t g = 0; g < r.GF.size(); ++g) r.GB[g] = r.GF[g];
         CK(cudaMemcpyAsync(r.inv_deg, pt->inv_deg.data(), sizeof(float) * r.rows, cudaMemcpyHostToDevice, m->cs));
-        if (r.n_seg_cnt) CK(cudaMemsetAsync(r.seg_cnt, 0, sizeof(int32_t) * r.n_seg_cnt, m->cs));
         // loopback W_G partials: the padding columns (ld > d) are summed with the rest (initcheck)
         if (r.WG_local) CK(cudaMemsetAsync(r.WG_local, 0, sizeof(float) * m->wtotal, m->cs));
         // zero every activation buffer once: padding columns stay 0 forever
@@ -920,8 +883,7 @@ int wait_bc(mggcn_model_s* m, cudaEvent_t e) {
 
 int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
-    SpmmTile t = job.dir == 0 ? r.F[j] : r.B[j];
-    t.seg_cnt = r.seg_cnt;
+    const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
     float* out = job.dst(m, r, job.ctx);
     m->tl_stage = tl_k;
     m->tl_rank = (int32_t)(&r - &m->ranks[0]);
@@ -961,8 +923,7 @@ float* group_slot(mggcn_model_s* m, Rank& r, int k, int64_t width) {
 
 int launch_group(mggcn_model_s* m, Rank& r, const SpmmJob& job, int g, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
-    SpmmTile t = job.dir == 0 ? r.GF[g] : r.GB[g];
-    t.seg_cnt = r.seg_cnt;
+    const SpmmTile& t = job.dir == 0 ? r.GF[g] : r.GB[g];
     float* out = job.dst(m, r, job.ctx);
     m->tl_stage = tl_k;
     m->tl_rank = (int32_t)(&r - &m->ranks[0]);

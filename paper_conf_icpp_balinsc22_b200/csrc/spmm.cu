@@ -13,10 +13,7 @@
 //   - U gathers per lane are issued before any FMA (memory-level parallelism);
 //   - epilogue fused: accumulate into the previous stage's output (RMW), and
 //     on the last stage the 1/deg row scale (Eq. 2 for pattern-only graphs)
-//     and ReLU (Eq. 7 / Eq. 18 in place);
-//   - hub rows of <= kFuseSegs segments are finished by the warp that completes
-//     their last segment (atomic segment count, partials summed in segment
-//     order); longer hub rows keep the separate fix-up kernel.
+//     and ReLU (Eq. 7 / Eq. 18 in place).
 #include <cstdio>
 #include <cstdlib>
 
@@ -152,8 +149,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, minb_for<G, CH>())
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const float4* __restrict__ B, int64_t ldb4,
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,
-                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T,
-                  const int4* __restrict__ segdesc, int32_t* __restrict__ seg_cnt) {
+                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T) {
     constexpr int S = 32 / G;
     // U entries per slot per group; U * S <= 32 so a group fits a 32-entry chunk
     constexpr int U = unroll_for<CH>() < G ? unroll_for<CH>() : G;
@@ -268,38 +264,15 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
         for (int off = G; off < 32; off <<= 1)
 #pragma unroll
             for (int ch = 0; ch < CH; ++ch) acc[ch] = f4_add(acc[ch], shfl_xor4(acc[ch], off));
-        if (it.w >= 0) {
-            if (slot == 0) {
+        if (slot == 0) {
+            if (it.w >= 0) {
                 float4* prow = partial + (int64_t)it.w * ldp4;
 #pragma unroll
                 for (int ch = 0; ch < CH; ++ch) {
                     const int q = cl + ch * G;
                     if (q < w4) prow[q] = acc[ch];
                 }
-            }
-            // fused fix-up (SpmmTile::segdesc): the warp that completes the last segment of a
-            // short split row sums its partials in segment order and finishes the row
-            const int4 sd = segdesc ? __ldg(segdesc + it.x) : make_int4(0, 0, 0, 0);
-            if (sd.w) {
-                __threadfence();                       // release this lane's part of the partial
-                __syncwarp();                          // ... every lane's, before lane 0 counts it
-                int last = 0;
-                if (lane == 0) last = atomicAdd(seg_cnt + it.x, 1) == sd.z - 1;
-                last = __shfl_sync(0xffffffffu, last, 0);
-                if (last) {
-                    __threadfence();                   // acquire the other segments' partials
-                    float4* orow = out + (int64_t)sd.x * ldo4;
-                    const float rs = rowscale ? __ldg(rowscale + sd.x) : 1.f;
-                    for (int q = lane; q < w4; q += 32) {
-                        float4 a = make_float4(0.f, 0.f, 0.f, 0.f);
-                        for (int s = 0; s < sd.z; ++s) a = f4_add(a, __ldcg(partial + (int64_t)(sd.y + s) * ldp4 + q));
-                        orow[q] = epilogue(a, orow, q, flags, rs);
-                    }
-                    if (lane == 0) seg_cnt[it.x] = 0;  // ready for the next launch
-                }
-            }
-        } else if (slot == 0) {
-            {
+            } else {
                 float4* orow = out + (int64_t)it.x * ldo4;
 #pragma unroll
                 for (int ch = 0; ch < CH; ++ch) {
@@ -405,8 +378,7 @@ void launch_one(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, i
     const int over = yenv > 1 ? yenv : ((flags & SPMM_YIELD) ? (yenv == 1 ? 1 : kYieldBlocks) : 1);
     const int64_t blocks = persistent_blocks<G, CH, V, H>(t.n_items, over);
     spmm_stage_kernel<G, CH, V, H><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
-        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T, t.segdesc,
-        t.seg_cnt);
+        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T);
 }
 
 template <int G, int CH>

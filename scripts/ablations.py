@@ -77,12 +77,25 @@ def main():
         emit(ablation="permutation", workload="reddit", P=1, permuted=bool(seed), epoch_ms=epoch_ms(gm, X, y))
         gm.close()
 
-    # 2. overlap on / off, loopback P = 4
+    # 2. overlap on / off, loopback P = 4, with the per-stage timeline of one epoch (Fig. 8 analogue;
+    #    the "broadcasts" are device copies on the comm stream, so this shows the schedule, not NVLink)
+    import bench
     for flags in (mg.MGGCN_F_OVERLAP, 0):
         gm = GCN(w.n, rp, col, None, w.dims, P=4, perm_seed=w.perm_seed, flags=flags, loopback=True, graph=g)
         gm.set_weights(Ws)
-        emit(ablation="overlap", workload="reddit", P=4, mode="loopback", overlap=bool(flags),
-             epoch_ms=epoch_ms(gm, X, y, steps=3, warmup=1))
+        ms = epoch_ms(gm, X, y, steps=3, warmup=1)
+        mg.mggcn_timeline_enable(gm.m, True)
+        mg.mggcn_get_timeline(gm.m, reset=True)
+        epoch_ms(gm, X, y, steps=1, warmup=0)
+        tl = mg.mggcn_get_timeline(gm.m, reset=True)
+        mg.mggcn_timeline_enable(gm.m, False)
+        summ = bench.timeline_summary(tl, w.dims, gm.p, 0)
+        emit(ablation="overlap", workload="reddit", P=4, mode="loopback", overlap=bool(flags), epoch_ms=ms,
+             timeline={k: summ[k] for k in ("epoch_span_ms", "compute_busy_ms", "comm_busy_ms", "exposed_comm_ms",
+                                            "exposed_comm_frac")},
+             first_spmm_stages=[dict(cls=r["cls"], stage=r["stage"], rank=r["rank"], stream=r["stream"],
+                                     t0=round(r["t0"], 4), t1=round(r["t1"], 4))
+                                for r in tl if r["spmm"] == 0])
         gm.close()
 
     # 3. duplicate coalescing on / off

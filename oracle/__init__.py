@@ -27,6 +27,9 @@ Pins (tests/test_oracle_*.py, all ``-m "not gpu"``):
                  with a dense Â (independent textbook implementation)
   adam           closed-form first step; torch.optim.Adam for 5 steps
   whole epoch    hand-derived known answers KA1 / KA2 (tests/golden/)
+  branch choices forward_preactivations / backward_given_masks == epoch and torch
+                 autograd with the masks Z > 0; with a flipped mask, == central
+                 finite differences of the loss with that mask frozen (reading C31)
 """
 from __future__ import annotations
 
@@ -404,3 +407,56 @@ def _wgrad(H, G, p, P):
 def tiles_dir(pg, P, rank, direction):
     t = tiles(pg, P, rank)
     return t[direction]
+
+
+# ------------------------------------------------- ReLU branch choices (reading C31)
+def forward_preactivations(pg: PermutedGraph, Xp, Ws, relu_last=False):
+    """The forward of oracle.epoch (Eq. 5-7, §4.4 order rule) on inputs already in permuted
+    order, returning every layer's pre-activation Z_l and input H_l (fp32 storage).  The
+    SpMMs are oracle.spmm (fp64 accumulation, ascending); the dense products use numpy's
+    float64 matmul as the library primitive (SURVEY §8(c) allows a matmul as a step) and are
+    rounded once to fp32, so a value can differ from oracle.gemm's only by fp64 rounding before
+    that rounding.  Used at full size, where oracle.gemm's single-threaded loops take hours."""
+    L = len(Ws)
+    H = [np.ascontiguousarray(Xp, dtype=np.float32)]
+    Z = []
+    for l in range(L):
+        W = np.asarray(Ws[l], dtype=np.float64)
+        if spmm_first(W.shape[0], W.shape[1]):
+            T = spmm(pg.At, H[l])
+            Zl = (T.astype(np.float64) @ W).astype(np.float32)
+        else:
+            HW = (H[l].astype(np.float64) @ W).astype(np.float32)
+            Zl = spmm(pg.At, HW)
+        Z.append(Zl)
+        H.append(relu(Zl) if (l < L - 1 or relu_last) else Zl)
+    return Z, H
+
+
+def backward_given_masks(pg: PermutedGraph, H, G, Ws, masks):
+    """Exact (fp64) backward of Eq. 8-11 with the ReLU' decisions given: masks[l] is the
+    boolean mask of layer l's ReLU (None for a linear layer), H[l] the layer inputs
+    (H[0] = X'), G = dLoss/dlogits.  Returns W_G,l for every l (fp64).  With masks[l] =
+    Z_l > 0 it is the plain backward of oracle.epoch (pinned against it and against torch
+    autograd in tests/test_oracle_numerics.py); with another ReLU branch choice at
+    pre-activations inside the fp32 error of 0 it is the exact gradient of that choice."""
+    L = len(Ws)
+    A64 = CSR(pg.A.rowptr, pg.A.col, pg.A.val.astype(np.float64))
+    At64 = CSR(pg.At.rowptr, pg.At.col, pg.At.val.astype(np.float64))
+    WG = [None] * L
+    G = np.asarray(G, dtype=np.float64)
+    for l in range(L - 1, -1, -1):
+        W = np.asarray(Ws[l], dtype=np.float64)
+        ZG = G * masks[l] if masks[l] is not None else G                 # Eq. 8 (C3, C27)
+        Hl = np.asarray(H[l], dtype=np.float64)
+        if not spmm_first(W.shape[0], W.shape[1]):
+            HWG = spmm(A64, ZG)                                          # Eq. 9
+            WG[l] = Hl.T @ HWG                                           # Eq. 10 (C2)
+            if l > 0:
+                G = HWG @ W.T                                            # Eq. 11
+        else:
+            T = spmm(At64, Hl)
+            WG[l] = T.T @ ZG
+            if l > 0:
+                G = spmm(A64, ZG @ W.T)
+    return WG

@@ -19,7 +19,20 @@ configuration, and is compared element by element with the oracle's:
             1e-5 + lr |s(g_gpu) - s(g_ref)|, s(g) = g / (|g| + eps): the first
             Adam step is exactly W - lr s(g), ill-conditioned where |g| ~ eps
             (reading C30)
-rel(x, r) = max|x - r| / max|r|.  Partitioning is an exact re-organisation
+rel(x, r) = max|x - r| / max|r|.
+
+ReLU branch choices (reading C31): where a pre-activation lies within the fp32
+forward error of 0, both ReLU' decisions are correct fp32 results, and the gradients
+below that ReLU (W_G,l, Adam m, v for l < L-1) depend on the choice; at Products-shaped
+size a few hundred such decisions out of 6.3e8 move W_G,0 by ~1.4e-3 of its max (its
+entries are sums of 2.45 M terms that largely cancel).  When such an entry misses 1e-3
+against the golden, the test checks what is unique and that the rest is valid:
+  (i)  every mask decision of the GPU that differs from an independent reference forward
+       (oracle.forward_preactivations) sits at |Z_ref| <= 1e-6 max|Z_ref|, and they are
+       at most 1e-6 of the entries;
+  (ii) the entry is within 1e-3 of the exact fp64 backward at the GPU's branch choices
+       (oracle.backward_given_masks, on the reference activations).
+Partitioning is an exact re-organisation
 (§8(c)), so the same golden serves P = 1 and the loopback P = 8 split of
 north_star's 8-GPU target.  The inputs' fingerprints are checked first, so a
 generator drift fails loudly instead of comparing different problems."""
@@ -70,7 +83,37 @@ def w_excess(g_ref, g_gpu, W_gpu, W_ref, lr=0.01, eps=1e-8):
     return float((diff - bound)[mask].max())
 
 
-def compare_epoch(g, L, loss, WG, adam, Wn, logits_rows=None):
+def branch_reference(name, gm_masks):
+    """Reading C31: the reference forward (oracle), the audit of the GPU's differing ReLU
+    decisions, and the exact fp64 backward at the GPU's branch choices (W_G, m, v)."""
+    import oracle
+    w = gen.WORKLOADS[name]
+    rp, col, X, y, Ws = gen.make_inputs(w)
+    pg = oracle.permute_graph(w.n, rp, col, None, seed=w.perm_seed)
+    Xp = np.empty_like(X); Xp[pg.perm] = X
+    yp = np.empty_like(y); yp[pg.perm] = y
+    del X
+    Z, H = oracle.forward_preactivations(pg, Xp, Ws)
+    L = len(Ws)
+    audit, masks, Hc = [], [], [Xp]
+    for l in range(L - 1):
+        mref = Z[l] > 0
+        flip = gm_masks[l] != mref
+        mx = float(np.abs(Z[l]).max())
+        worst = float(np.abs(Z[l][flip]).max() / mx) if flip.any() else 0.0
+        audit.append({"layer": l, "flips": int(flip.sum()), "entries": int(flip.size), "max_abs_preact_at_flip": worst})
+        assert worst <= 1e-6 and flip.sum() <= 1e-6 * flip.size, audit[-1]        # C31 (i)
+        masks.append(gm_masks[l])
+        Hc.append(np.where(gm_masks[l], Z[l], 0).astype(np.float32))
+    masks.append(None)
+    ntrain = int((yp >= 0).sum())
+    _, G = oracle.softmax_ce(Z[L - 1].astype(np.float64), yp, ntrain)
+    WGb = oracle.backward_given_masks(pg, Hc, G, Ws, masks)
+    print(json.dumps({"branch_audit": audit}))
+    return {"WG": WGb, "m": [0.1 * w_ for w_ in WGb], "v": [0.001 * w_ * w_ for w_ in WGb]}
+
+
+def compare_epoch(g, L, loss, WG, adam, Wn, logits_rows=None, branch=None):
     out = {"loss": abs(loss - float(g["loss"])) / abs(float(g["loss"]))}
     if logits_rows is not None:
         out["logits"] = rel(logits_rows, g["logits_rows"])
@@ -82,8 +125,18 @@ def compare_epoch(g, L, loss, WG, adam, Wn, logits_rows=None):
         out[f"v{l}"] = rel(ve, g[f"v{l}"])
         out[f"W{l}_excess"] = w_excess(g[f"WG{l}"], WG[l], Wn[l], g[f"W{l}"])
     print(json.dumps(out))
-    for k, v in out.items():
-        assert v <= (0.0 if k.endswith("_excess") else REL_TOL), (k, v, out)
+    failing = [k for k, v in out.items() if v > (0.0 if k.endswith("_excess") else REL_TOL)]
+    below_relu = {f"{p}{l}" for p in ("WG", "m", "v") for l in range(L - 1)}
+    if failing and branch is not None and set(failing) <= below_relu:
+        ref = branch()                                        # reading C31: (i) inside, (ii) here
+        got = {"WG": WG, "m": [a[0] for a in adam], "v": [a[1] for a in adam]}
+        rechk = {k: rel(got[k[:-1]][int(k[-1])], ref[k[:-1]][int(k[-1])]) for k in failing}
+        print(json.dumps({"branch_choice_recheck": rechk}))
+        for k, v in rechk.items():
+            assert v <= REL_TOL, (k, v, out, rechk)
+        return out
+    for k in failing:
+        raise AssertionError((k, out[k], out))
     return out
 
 
@@ -110,10 +163,12 @@ def test_fullsize_epoch_matches_oracle_golden(name, P):
         loss = gm.forward(Xd, yd, want_loss=True, logits=logits)
         rows = torch.from_numpy(g["rows"]).cuda()
         lrows = logits.index_select(0, rows).cpu().numpy()
+        masks = [mg.mggcn_debug_layer(gm.m, l, (w.n, w.dims[l + 1])) > 0 for l in range(L - 1)]   # ReLU decisions
         gm.backward()
         WG = gm.grads()
         gm.step(lr=0.01)
-        compare_epoch(g, L, loss, WG, [gm.adam_state(l) for l in range(L)], gm.get_weights(), lrows)
+        compare_epoch(g, L, loss, WG, [gm.adam_state(l) for l in range(L)], gm.get_weights(), lrows,
+                      branch=lambda: branch_reference(name, masks))
     finally:
         gm.close()
 
@@ -137,7 +192,13 @@ def test_fullsize_captured_epoch_matches_oracle_golden(name):
         gm.capture_epoch(Xd, yd, lr=0.01)
         gm.replay_epoch(1)
         gm.synchronize()
-        compare_epoch(g, L, gm.loss(), gm.grads(), [gm.adam_state(l) for l in range(L)], gm.get_weights())
+        # the captured epoch's ReLU decisions: AHWB_l after the step holds Z_G,l, so re-run the
+        # forward eagerly from the replay's starting weights (bitwise the same kernels)
+        WG, adam, Wn, loss = gm.grads(), [gm.adam_state(l) for l in range(L)], gm.get_weights(), gm.loss()
+        gm.set_weights(Ws)
+        gm.forward(Xd, yd, want_loss=False)
+        masks = [mg.mggcn_debug_layer(gm.m, l, (w.n, w.dims[l + 1])) > 0 for l in range(L - 1)]
+        compare_epoch(g, L, loss, WG, adam, Wn, branch=lambda: branch_reference(name, masks))
     finally:
         gm.close()
 

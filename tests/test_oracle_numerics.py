@@ -254,3 +254,65 @@ def test_float_storage_close_to_double():
     assert rel < 1e-6
     for a, b in zip(r32.WG, r64.WG):
         assert np.abs(a - b).max() / np.abs(b).max() < 1e-5
+
+
+@pytest.mark.parametrize("dims", [(3, 5, 2), (6, 6, 4, 3), (2, 8, 3)])
+def test_branch_choice_helpers_match_epoch_and_autograd(dims):
+    """forward_preactivations / backward_given_masks (reading C31): with the masks Z_l > 0 they
+    reproduce oracle.epoch's forward and W_G, and torch float64 autograd (a textbook GCN)."""
+    n = 24
+    rp, col, vals, X, y, Ws = _random_problem(n, 120, dims, 5, weighted=True, unlabelled=0.2)
+    pg = oracle.permute_graph(n, rp, col, vals, seed=7, dtype=np.float64)
+    r = oracle.epoch(pg, X, y, Ws, dtype=np.float64)
+    Xp = np.empty_like(X); Xp[pg.perm] = X
+    yp = np.empty_like(y); yp[pg.perm] = y
+    pg32 = oracle.permute_graph(n, rp, col, vals, seed=7)
+    Z, H = oracle.forward_preactivations(pg32, Xp, Ws)
+    for a, b in zip(Z, r.Z):
+        np.testing.assert_allclose(a, b, rtol=1e-5, atol=1e-6)
+    ntrain = int((yp >= 0).sum())
+    _, G = oracle.softmax_ce(r.logits, yp, ntrain)
+    masks = [r.Z[l] > 0 for l in range(len(Ws) - 1)] + [None]
+    Hd = [Xp] + [oracle.relu(z) for z in r.Z[:-1]]
+    WG = oracle.backward_given_masks(pg, Hd, G, Ws, masks)
+    _, _, grads = torch_epoch(_perm_dense(n, rp, col, vals, pg.perm), Xp, yp, Ws)
+    for a, b, c in zip(WG, r.WG, grads):
+        np.testing.assert_allclose(a, b, rtol=1e-9, atol=1e-12)
+        np.testing.assert_allclose(a, c, rtol=1e-9, atol=1e-12)
+
+
+def test_backward_given_masks_is_the_gradient_of_the_chosen_branch():
+    """Flipping one ReLU decision at a pre-activation near 0 changes W_G by exactly the
+    gradient of that branch: central finite differences of the loss with the flipped
+    mask frozen (the ReLU replaced by the fixed 0/1 mask) match backward_given_masks."""
+    n, dims = 16, (3, 4, 3)
+    rp, col, vals, X, y, Ws = _random_problem(n, 60, dims, 31)
+    pg = oracle.permute_graph(n, rp, col, vals, seed=3, dtype=np.float64)
+    Xp = np.empty_like(X); Xp[pg.perm] = X
+    yp = np.empty_like(y); yp[pg.perm] = y
+    Ahp = _perm_dense(n, rp, col, vals, pg.perm)
+    r = oracle.epoch(pg, X, y, Ws, dtype=np.float64)
+    mask = r.Z[0] > 0
+    i = np.unravel_index(np.argmin(np.abs(r.Z[0])), mask.shape)
+    mask[i] = ~mask[i]                                            # the other branch at the smallest |Z|
+
+    def loss_of(Wl):
+        H1 = (Ahp.T @ Xp @ Wl[0]) * mask
+        Zl = Ahp.T @ H1 @ Wl[1]
+        zz = Zl - Zl.max(axis=1, keepdims=True)
+        lse = np.log(np.exp(zz).sum(axis=1)) + Zl.max(axis=1)
+        lab = yp >= 0
+        return float((lse[lab] - Zl[lab, yp[lab]]).sum() / lab.sum())
+
+    H1 = (Ahp.T @ Xp @ Ws[0]) * mask
+    logits = Ahp.T @ H1 @ Ws[1]
+    _, G = oracle.softmax_ce(logits, yp, int((yp >= 0).sum()))
+    WG = oracle.backward_given_masks(pg, [Xp, H1], G, Ws, [mask, None])
+    h = 1e-6
+    for l in range(2):
+        for c in range(dims[l]):
+            for k in range(dims[l + 1]):
+                Wp = [W.copy() for W in Ws]; Wp[l][c, k] += h
+                Wm = [W.copy() for W in Ws]; Wm[l][c, k] -= h
+                fd = (loss_of(Wp) - loss_of(Wm)) / (2 * h)
+                assert abs(fd - WG[l][c, k]) <= 1e-6 * max(1.0, abs(fd)), (l, c, k)

@@ -512,6 +512,7 @@ def main():
     prof = gm.profile(reset=True)
     work = gm.epoch_work()
     work_detail = gm.epoch_work_detail()
+    stage_groups = mg.mggcn_stage_groups(gm.m)
     # ---- one extra eager epoch with the per-stage timeline (not timed)
     timeline = None
     try:
@@ -729,6 +730,7 @@ def main():
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": workload_desc(w, P),
         "run": {"overlap": not args.no_overlap, "gemm": "tf32x1" if args.tf32x1 else "3xTF32 (tcgen05)",
+                "stage_groups": stage_groups,
                 "comm": (args.comm if P > 1 else "none"),
                 "parallelism": (f"dp{P} (1D row partition)" if args.replicas == 1 else
                                 f"dp{P} (1.5D: {P // 2} row blocks x 2 replicas)")},

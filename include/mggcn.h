@@ -300,6 +300,11 @@ int mggcn_epoch_work(mggcn_model m, double* spmm_bytes, double* spmm_gather_byte
  * EINVAL: NULL out, n < 0. */
 int mggcn_epoch_work_detail(mggcn_model m, double* out, int32_t n);
 
+/* The remote-stage schedule the model chose (DESIGN §7 "Stage groups"): returns the
+ * number of stage groups (0 = one launch per stage, the paper's BC1/BC2 schedule) and
+ * writes up to cap group sizes (remote blocks per launch, in consumption order). */
+int mggcn_stage_groups(mggcn_model m, int32_t* sizes, int32_t cap);
+
 /* Number of kernels this library has launched in this process (all models,
  * all debug hooks).  Read before and after a timed region to count them. */
 int64_t mggcn_kernel_launch_count(void);

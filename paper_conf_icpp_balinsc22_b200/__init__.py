@@ -39,7 +39,7 @@ EXPORTS = (
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
     "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
     "mggcn_epoch_replay", "mggcn_debug_comm_delay", "mggcn_get_timeline",
-    "mggcn_epoch_work_detail", "mggcn_timeline_enable", "mggcn_debug_poison",
+    "mggcn_epoch_work_detail", "mggcn_timeline_enable", "mggcn_debug_poison", "mggcn_stage_groups",
 )
 
 
@@ -87,6 +87,7 @@ def _load():
         "mggcn_get_timeline": ([P, i64, P, P, P, i32], ctypes.c_int),
         "mggcn_timeline_enable": ([P, i32], ctypes.c_int),
         "mggcn_debug_poison": ([P, i32], ctypes.c_int),
+        "mggcn_stage_groups": ([P, P, i32], ctypes.c_int),
         "mggcn_epoch_work": ([P, P, P, P, P], ctypes.c_int),
         "mggcn_epoch_work_detail": ([P, P, i32], ctypes.c_int),
         "mggcn_graph_free": ([P], None),
@@ -344,6 +345,15 @@ def mggcn_epoch_work_detail(m):
     if k < 0:
         _check(k)
     return {name: out[i] for i, name in enumerate(WORK_DETAIL_KEYS[:k])}
+
+
+def mggcn_stage_groups(m):
+    """Remote blocks per SpMM launch ([] = one launch per stage)."""
+    sizes = (ctypes.c_int32 * 16)()
+    k = _lib.mggcn_stage_groups(m, sizes, 16)
+    if k < 0:
+        _check(k)
+    return [int(sizes[i]) for i in range(k)]
 
 
 def mggcn_kernel_launch_count() -> int:

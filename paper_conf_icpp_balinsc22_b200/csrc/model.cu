@@ -374,13 +374,20 @@ inline bool last_of_group(const mggcn_model_s* m, int k) { return k == m->grp_b[
 // these fixed costs are about a third of its SpMM time.  Grouped,
 // the remote blocks get one BC slot each (P - 1 slots, no reuse inside a
 // SpMM) and a group of them is consumed by ONE launch over a merged tile.
-// Default: two groups per SpMM, a small first one (ceil((P-1)/4) blocks, whose
-// transfer hides behind the local stage) and the rest (whose transfer hides
-// behind the first group); P >= 4.  Off when the P - 1 slots exceed
-// MGGCN_BC_BUDGET_MB (default 16 GiB: Papers-shaped 14 GB blocks keep BC1/BC2).
-// MGGCN_STAGE_GROUPS="a,b,.." (sizes summing to P - 1) or MGGCN_STAGE_GROUP=S
-// (uniform; 1 = per stage) override.  1D only.
-std::vector<int> choose_groups(const mggcn_model_s* m) {
+// The broadcasts then run back to back, so the SpMM ends at max(the compute
+// chain, the last block's arrival + the LAST group's compute):
+//  * compute-bound ranks (a block computes >= 1.5x longer than it takes to
+//    arrive: e_row = coalesced entries per row per remote tile, compute / arrival
+//    ~ e_row x 900 GB/s NVLink / 16 TB/s gathers >= 1.5, i.e. e_row >= 27; Reddit- and
+//    Proteins-shaped at P = 8): two groups, ceil((P-1)/4) blocks (hidden behind the
+//    local stage) and the rest;
+//  * otherwise (Products-, Papers-shaped) the exchange bounds the SpMM, and the last
+//    group's compute is exposed after the last arrival: groups (ceil((P-1)/4), middle, 1),
+//    whose tail is one block, as in the per-stage schedule, with fewer launches.
+// Off when the P - 1 slots exceed MGGCN_BC_BUDGET_MB (default 16 GiB: Papers-shaped
+// 14 GB blocks keep BC1/BC2).  MGGCN_STAGE_GROUPS="a,b,.." (sizes summing to P - 1)
+// or MGGCN_STAGE_GROUP=S (uniform; 1 = per stage) override.  1D only.
+std::vector<int> choose_groups(const mggcn_model_s* m, double e_row) {
     std::vector<int> none;
     if (m->P <= 2 || m->c > 1) return none;
     if (const char* h = getenv("MGGCN_SPMM_HOTCLS"))
@@ -408,7 +415,9 @@ std::vector<int> choose_groups(const mggcn_model_s* m) {
         } else {
             if (m->P < 4) return none;
             const int first = (R + 3) / 4;
-            sizes = {first, R - first};
+            if (e_row * 900.0 / 16000.0 >= 1.5) sizes = {first, R - first};   // compute-bound
+            else if (R - first >= 2) sizes = {first, R - first - 1, 1};      // exchange-bound
+            else return none;
         }
     }
     double budget = 16384.0;
@@ -1501,7 +1510,18 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         r.order_cache = order;
     }
     m->n_local = off;
-    m->grp_b = choose_groups(m);
+    double e_row = 0;   // coalesced entries per row per remote tile (the compute / exchange regime)
+    {
+        double nnz = 0, rows = 0;
+        for (auto& r : m->ranks)
+            for (int j = 0; j < m->P; ++j)
+                if (j != r.rank) {
+                    nnz += (double)r.tF(j).rowptr.back();
+                    rows += (double)r.rows;
+                }
+        e_row = rows > 0 ? nnz / rows : 0;
+    }
+    m->grp_b = choose_groups(m, e_row);
     if (m->grouped()) {
         const bool ipc = (flags & MGGCN_F_IPC) != 0;
         const int NG = n_groups(m);
@@ -2423,6 +2443,13 @@ extern "C" int mggcn_get_profile(mggcn_model m, double* ms, int64_t* launches, i
         }
     }
     return MGGCN_OK;
+}
+
+extern "C" int mggcn_stage_groups(mggcn_model m, int32_t* sizes, int32_t cap) {
+    MODEL_GUARD(m);
+    const int ng = n_groups(m);
+    for (int g = 0; g < ng && g < cap && sizes; ++g) sizes[g] = m->grp_b[g + 1] - m->grp_b[g];
+    return ng;
 }
 
 extern "C" int mggcn_debug_poison(mggcn_model m, int32_t on) {

@@ -132,6 +132,7 @@ def main():
                 "results invalid): per-rank compute ms per epoch",
         "n": w.n, "nnz": w.m, "dims": list(w.dims), "rank_rows": int(rows),
         "compute_ms_per_epoch": ms,
+        "stage_groups": mg.mggcn_stage_groups(gm.m),
         "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
         "workspace_GiB": gm.ws_bytes / 2**30,
         "device_mem_reserved_GiB": torch.cuda.memory_reserved() / 2**30,

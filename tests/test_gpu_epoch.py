@@ -511,3 +511,23 @@ def test_poison_negative_control(mg, monkeypatch, group):
     bad = run_library(mg, w.n, rp, col, None, X, y, Ws, w.dims, 4, w.perm_seed, mg.MGGCN_F_OVERLAP,
                       delay=(3, 2000), poison=2)
     assert not np.array_equal(np.nan_to_num(bad["logits"], nan=1e30), clean["logits"])
+
+
+def test_stage_group_regimes(mg):
+    """choose_groups: a rank whose blocks compute longer than they take to arrive
+    (many entries per row per tile) gets two groups; an exchange-bound one keeps a last group of
+    one block (its tail after the last arrival is one block, as in the per-stage schedule)."""
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    dims = (16, 16, 4)
+    n = 3000
+    rp, col = gen.rmat_csr(n, 2000000, 91)           # ~670 entries per row: ~80 per row per tile at P = 8
+    gm = GCN(n, rp, col, None, dims, P=8, perm_seed=1, loopback=True)
+    assert mg.mggcn_stage_groups(gm.m) == [2, 5]
+    gm.close()
+    rp, col = gen.rmat_csr(n, 30000, 92)             # ~10 entries per row: ~1 per tile
+    gm = GCN(n, rp, col, None, dims, P=8, perm_seed=1, loopback=True)
+    assert mg.mggcn_stage_groups(gm.m) == [2, 4, 1]
+    gm.close()
+    gm = GCN(n, rp, col, None, dims, P=3, perm_seed=1, loopback=True)
+    assert mg.mggcn_stage_groups(gm.m) == []         # P <= 3: the paper's per-stage schedule
+    gm.close()

@@ -83,9 +83,20 @@ def w_excess(g_ref, g_gpu, W_gpu, W_ref, lr=0.01, eps=1e-8):
     return float((diff - bound)[mask].max())
 
 
+_BRANCH_CACHE = {}
+
+
 def branch_reference(name, gm_masks):
     """Reading C31: the reference forward (oracle), the audit of the GPU's differing ReLU
-    decisions, and the exact fp64 backward at the GPU's branch choices (W_G, m, v)."""
+    decisions, and the exact fp64 backward at the GPU's branch choices (W_G, m, v).
+    Cached per (config, masks): the eager and the captured epoch make the same decisions."""
+    key = (name, tuple(hashlib.sha256(np.packbits(m).tobytes()).hexdigest() for m in gm_masks))
+    if key not in _BRANCH_CACHE:
+        _BRANCH_CACHE[key] = _branch_reference(name, gm_masks)
+    return _BRANCH_CACHE[key]
+
+
+def _branch_reference(name, gm_masks):
     import oracle
     w = gen.WORKLOADS[name]
     rp, col, X, y, Ws = gen.make_inputs(w)

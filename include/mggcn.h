@@ -319,6 +319,9 @@ void mggcn_model_free(mggcn_model m);
  * mggcn_debug_spmm: out = Â'^T B (dir 0) or Â' B (dir 1) for the model's
  *   rows, B = the model's n_local... all n rows of the permuted operand in
  *   loopback mode / P = 1 (device, ld = ldb), through the staged pipeline.
+ *   In the SOLO timing mode (one rank of a P-way partition, no broadcasts) B is
+ *   the rank's own block and the remote stages read the never-filled (zero) BC
+ *   slots, so out = the rank's LOCAL tile times B, row-scaled on the last stage.
  * mggcn_debug_gemm: op 0: C = A·B (A MxK, B KxN); op 1: C = A·B^T (B NxK);
  *   op 2: C = A^T·B (A KxM, B KxN).  Device pointers, tcgen05 path. */
 int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int64_t ldb, int32_t width, float* out,

@@ -2567,8 +2567,8 @@ extern "C" int mggcn_debug_spmm(mggcn_model m, int32_t dir, const float* B, int6
         set_error("debug_spmm: bad arguments");
         return MGGCN_EINVAL;
     }
-    if (m->P > 1 && m->nlocal == 1) {
-        set_error("debug_spmm: needs P == 1 or loopback mode");
+    if (m->P > 1 && m->nlocal == 1 && !m->solo) {
+        set_error("debug_spmm: needs P == 1, loopback or the SOLO timing mode");
         return MGGCN_EUNSUPPORTED;
     }
     const int64_t w = round_up(width, 4);

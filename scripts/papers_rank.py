@@ -26,6 +26,52 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
+def local_tile_check(gm, mg, w, rp, col, rank):
+    """Correctness at full size on sampled rows (SOLO mode): mggcn_debug_spmm returns the rank's
+    LOCAL tile times B (remote BC slots are never filled), i.e. for local row r (new id v):
+    inv_deg(v) * sum over in-neighbours u of v with new id in this rank's block of B[u - p0]
+    (Eq. 2 and Eq. 6 restricted to the diagonal tile).  The reference is computed in
+    fp64 from the ORIGINAL CSR and the permutation (symmetric graph: in-neighbours = the row),
+    independently of the library's partitioner and tiles."""
+    import numpy as np
+    import torch
+
+    import gen
+    p0, p1 = int(gm.p[rank]), int(gm.p[rank + 1])
+    rows = p1 - p0
+    width = 64
+    B = torch.from_numpy(gen.features(rows, width, 777)).cuda()
+    outd = torch.empty((rows, width), dtype=torch.float32, device="cuda")
+    mg.mggcn_debug_spmm(gm.m, 0, B, width, width, outd, width)
+    perm = np.asarray(gm.perm, dtype=np.int64)
+    inv = np.empty_like(perm)
+    inv[perm] = np.arange(perm.shape[0], dtype=np.int64)
+    deg = np.diff(rp)
+    local_orig = inv[p0:p1]
+    ldeg = deg[local_orig]
+    rng = np.random.default_rng(5)
+    sample = set(rng.choice(rows, 254, replace=False).tolist())
+    sample.add(int(np.argmax(ldeg)))
+    z = np.flatnonzero(ldeg == 0)
+    if z.size:
+        sample.add(int(z[0]))
+    sample = np.array(sorted(sample), dtype=np.int64)
+    got = outd[torch.from_numpy(sample).cuda()].cpu().numpy().astype(np.float64)
+    Bh = B.cpu().numpy()
+    exp = np.zeros_like(got)
+    for i, r in enumerate(sample):
+        x = local_orig[r]
+        nb = perm[col[rp[x]:rp[x + 1]].astype(np.int64)]
+        nb = nb[(nb >= p0) & (nb < p1)] - p0
+        d = np.float32(deg[x])
+        s = Bh[nb].astype(np.float64).sum(axis=0)
+        exp[i] = s * (np.float32(1.0) / d if d != 0 else 0.0)
+    rel = float(np.abs(got - exp).max() / max(np.abs(exp).max(), 1e-30))
+    return {"rows_checked": int(sample.size), "largest_local_in_degree": int(ldeg.max()),
+            "rel_err": rel, "ok": rel <= 1e-4,
+            "how": "mggcn_debug_spmm in SOLO mode = local tile x B; reference from the original CSR + perm (fp64)"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--rank", type=int, default=0)
@@ -33,6 +79,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=2)
     ap.add_argument("--workload", default="papers")
+    ap.add_argument("--check", action="store_true",
+                    help="after timing: the local-tile SpMM on sampled rows against the original CSR (host, fp64)")
     ap.add_argument("--timeline", action="store_true",
                     help="also record one epoch with MGGCN_F_TIMELINE and report per-SpMM stage sums / spans / gaps")
     args = ap.parse_args()
@@ -59,7 +107,8 @@ def main():
     t0 = time.perf_counter()
     graph = mg.mggcn_load_csr(w.n, rp, col)
     t_load = time.perf_counter() - t0
-    del rp, col
+    if not args.check:
+        del rp, col
     print(f"[papers_rank] load_csr {t_load:.1f} s", flush=True)
     flags = mg.MGGCN_F_OVERLAP | mg.MGGCN_F_NO_BCAST | mg.MGGCN_F_PROFILE
     t0 = time.perf_counter()
@@ -144,6 +193,8 @@ def main():
         "steps": args.steps, "warmup": args.warmup, "timeline": tl_summary,
         "gpu": torch.cuda.get_device_name(0),
     }
+    if args.check:
+        out["check"] = local_tile_check(gm, mg, w, rp, col, args.rank)
     print(json.dumps(out), flush=True)
     gm.close()
 

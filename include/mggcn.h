@@ -305,6 +305,15 @@ int mggcn_epoch_work_detail(mggcn_model m, double* out, int32_t n);
  * writes up to cap group sizes (remote blocks per launch, in consumption order). */
 int mggcn_stage_groups(mggcn_model m, int32_t* sizes, int32_t cap);
 
+/* Dense blocks of the stage tiles (DESIGN §6 "Dense blocks"): writes min(n, 5)
+ * values into out and returns 5: [0] dense 128 x 32 blocks, [1] coalesced
+ * entries they cover (run on the tensor cores), [2] row groups, [3] column
+ * chunks, [4] coalesced entries of every launched tile (blocks + residual CSR),
+ * summed over this model's ranks and both directions (F and B tiles; one set
+ * when they are shared).  The density threshold is MGGCN_DENSE_THR at
+ * mggcn_model_create (default 0.03; 0 = no blocks).  EINVAL: NULL out. */
+int mggcn_dense_stats(mggcn_model m, int64_t* out, int32_t n);
+
 /* Number of kernels this library has launched in this process (all models,
  * all debug hooks).  Read before and after a timed region to count them. */
 int64_t mggcn_kernel_launch_count(void);

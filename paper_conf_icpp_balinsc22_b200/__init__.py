@@ -39,7 +39,7 @@ EXPORTS = (
     "mggcn_debug_spmm", "mggcn_debug_gemm", "mggcn_kernel_launch_count", "mggcn_reset_cache",
     "mggcn_prefetch", "mggcn_ipc_export", "mggcn_ipc_connect", "mggcn_debug_layer", "mggcn_epoch_capture",
     "mggcn_epoch_replay", "mggcn_debug_comm_delay", "mggcn_get_timeline",
-    "mggcn_epoch_work_detail", "mggcn_timeline_enable", "mggcn_debug_poison", "mggcn_stage_groups",
+    "mggcn_epoch_work_detail", "mggcn_timeline_enable", "mggcn_debug_poison", "mggcn_stage_groups", "mggcn_dense_stats",
 )
 
 
@@ -88,6 +88,7 @@ def _load():
         "mggcn_timeline_enable": ([P, i32], ctypes.c_int),
         "mggcn_debug_poison": ([P, i32], ctypes.c_int),
         "mggcn_stage_groups": ([P, P, i32], ctypes.c_int),
+        "mggcn_dense_stats": ([P, P, i32], ctypes.c_int),
         "mggcn_epoch_work": ([P, P, P, P, P], ctypes.c_int),
         "mggcn_epoch_work_detail": ([P, P, i32], ctypes.c_int),
         "mggcn_graph_free": ([P], None),
@@ -354,6 +355,18 @@ def mggcn_stage_groups(m):
     if k < 0:
         _check(k)
     return [int(sizes[i]) for i in range(k)]
+
+
+DENSE_STATS_KEYS = ("blocks", "block_entries", "row_groups", "chunks", "entries")
+
+
+def mggcn_dense_stats(m):
+    """Dense blocks of the launched stage tiles (tensor-core part of the SpMM)."""
+    out = (ctypes.c_int64 * 8)()
+    k = _lib.mggcn_dense_stats(m, out, 8)
+    if k < 0:
+        _check(k)
+    return {name: int(out[i]) for i, name in enumerate(DENSE_STATS_KEYS[:k])}
 
 
 def mggcn_kernel_launch_count() -> int:

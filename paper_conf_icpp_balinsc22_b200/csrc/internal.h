@@ -38,6 +38,31 @@ struct HostTile {
     std::vector<float> val;        // Â'_uv per entry; empty if pattern-only
 };
 
+// Dense blocks of one stage tile (dense_plan.cpp, run by dense.cu): rows and
+// columns ranked by entry count, cut into 128-row groups x 32-column chunks;
+// a block with >= thr * 128 * 32 entries (values exact in bf16) goes to the
+// tensor cores, everything else stays in `resid` for the CSR gather kernel.
+struct DenseHost {
+    bool active = false;
+    HostTile resid;                     // the tile minus the dense blocks' entries
+    int64_t n_groups = 0, n_tiles = 0, n_chunks = 0, nnz = 0;
+    std::vector<int32_t> grp_rows;      // n_groups * 128, -1 = empty slot
+    std::vector<uint8_t> row_flag;      // nrows: 1 = the row is in a group (gets a dense product)
+    std::vector<int32_t> grp_beg;       // n_groups + 1
+    // work items {group, first block, end block, partial slot (-1: the item is the whole group
+    // and adds into the output)}, longest first; groups longer than the segment length are cut
+    // into several items whose 128 x N products go to partial slots, summed in item order per
+    // group by the fix-up (splits: {group, first slot, slots, 0})
+    std::vector<int32_t> work;          // n_items * 4
+    std::vector<int32_t> splits;        // n_splits * 4 (last: 0)
+    int64_t n_items = 0, n_splits = 0, n_slots = 0;
+    std::vector<int32_t> tile_chunk;    // n_tiles
+    std::vector<int32_t> chunk_cols;    // n_chunks * 32, -1 = empty slot
+    std::vector<uint16_t> A;            // n_tiles * 128 * 32 bf16, K-major SWIZZLE_64B image per block
+};
+// thr <= 0, nothing dense, or the blocks holding < min_frac of the entries => d.active = false.
+void plan_dense(const HostTile& t, double thr, double min_frac, DenseHost& d);
+
 // One rank's 1D partition of the permuted graph.
 struct mggcn_part_s {
     int32_t P = 1, rank = 0;

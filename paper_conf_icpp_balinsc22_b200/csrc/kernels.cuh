@@ -32,6 +32,40 @@ inline int split_for(int64_t nnz) {
     return s;
 }
 
+// ------------------------------------------------------------ dense tiles
+// Dense blocks of a stage tile run on the tensor cores (dense.cu; chosen by
+// plan_dense, dense_plan.cpp): kDenseM output rows (a row group, rows in
+// degree order) x kDenseK columns (a column chunk, columns in degree order).
+constexpr int kDenseM = 128;
+constexpr int kDenseK = 32;
+constexpr int kDenseMaxN = 256;    // features per launch (wider operands: 256-column windows)
+// default density threshold of a dense block (entries / (128 x 32)); MGGCN_DENSE_THR overrides, 0 = off
+constexpr double kDenseThrDefault = 0.03;
+// a tile uses blocks only if they hold >= this share of its entries; MGGCN_DENSE_MINFRAC overrides
+constexpr double kDenseMinFracDefault = 0.5;
+struct DenseTiles {
+    int64_t n_groups = 0, n_tiles = 0, n_chunks = 0;
+    int64_t n_items = 0, n_splits = 0, n_slots = 0;
+    int64_t nnz = 0;                   // entries (coalesced) covered by the blocks
+    int pieces = 3;                    // bf16 pieces of the B operand (2: hi + mid, 3: + lo)
+    const int32_t* grp_rows = nullptr;   // [n_groups][kDenseM] output row of each slot, -1 = none
+    const uint8_t* row_flag = nullptr;   // [nrows] 1 = row of a group: the gather kernel adds to its output
+    const int4* work = nullptr;          // [n_items] {group, first block, end block, partial slot or -1}
+    const int4* splits = nullptr;        // [n_splits] {group, first slot, slots, 0}: groups cut into items
+    float* partial = nullptr;            // scratch: [n_slots][kDenseM][N]
+    const int32_t* tile_chunk = nullptr; // [n_tiles] column chunk of each block
+    const int32_t* chunk_cols = nullptr; // [n_chunks][kDenseK] column of each chunk slot, -1 = none
+    const uint8_t* A = nullptr;          // [n_tiles][kDenseM x kDenseK bf16], K-major SWIZZLE_64B image
+    uint8_t* bimg = nullptr;             // scratch: [n_chunks][pieces][N][kDenseK bf16]
+};
+// out[rows of the groups][0, width) (+)= dense blocks · B (B row stride ldb, width <= kDenseMaxN,
+// % 4 == 0); first: store (the stage's first write) instead of add
+cudaError_t launch_dense(const DenseTiles& d, const float* B, int64_t ldb, float* out, int64_t ldo, int width,
+                         bool first, cudaStream_t s);
+size_t dense_bimg_bytes(int64_t n_chunks, int pieces);
+size_t dense_partial_floats(int64_t n_slots);
+int dense_stages_for(int N, int pieces);
+
 struct SpmmTile {
     const int4* items = nullptr;   // {row, beg, end, slot}
     int64_t n_items = 0;
@@ -49,6 +83,8 @@ struct SpmmTile {
     // (hot_class_of); launch_spmm gathers the rows of the classes that fit its
     // L2 budget with evict_last and the rest with evict_first.
     bool hot_enc = false;
+    // dense blocks of the tile (n_groups == 0: none); the CSR above then holds the residual entries
+    DenseTiles dense;
 };
 
 // default evict_last budget of the L2 priority classes (MGGCN_SPMM_HOT_MB overrides)

@@ -198,6 +198,18 @@ struct Rank {
         if (coalesced) return part->shared_fb ? cF[j] : cB[j];
         return part->tileB(j);
     }
+    // dense blocks of the launched tiles (plan_dense; DESIGN §6 "Dense blocks"): when active,
+    // the launch tile is the residual CSR and the blocks run on the tensor cores
+    std::vector<DenseHost> dF, dB, dgF, dgB;
+    const HostTile& lF(int j) const { return (j < (int)dF.size() && dF[j].active) ? dF[j].resid : tF(j); }
+    const HostTile& lB(int j) const {
+        if (part->shared_fb) return lF(j);
+        return (j < (int)dB.size() && dB[j].active) ? dB[j].resid : tB(j);
+    }
+    const HostTile& lgF(int g) const { return (g < (int)dgF.size() && dgF[g].active) ? dgF[g].resid : gF[g]; }
+    const HostTile& lgB(int g) const { return (g < (int)dgB.size() && dgB[g].active) ? dgB[g].resid : gB[g]; }
+    uint8_t* dense_bimg = nullptr;   // B-image scratch shared by the tiles' dense launches
+    float* dense_partial = nullptr;  // partial products of split row groups (same sharing)
     float* inv_deg = nullptr;
     float* Xs = nullptr;             // current input buffer (= Xbuf[xcur])
     int32_t* y = nullptr;
@@ -293,6 +305,11 @@ struct mggcn_model_s {
     void* ipc_alloc = nullptr;
     size_t ipc_alloc_off = 0;
     bool ipc = false, ipc_connected = false;
+    // dense blocks of the stage tiles (plan_dense): density threshold (MGGCN_DENSE_THR,
+    // 0 = off) and bf16 pieces of the B operand (MGGCN_DENSE_PIECES, 2 or 3)
+    double dense_thr = 0;
+    double dense_min_frac = 0.5;    // MGGCN_DENSE_MINFRAC: blocks must hold this share of a tile's entries
+    int dense_pieces = 3;
     // SOLO timing mode (MGGCN_F_NO_BCAST, P > 1, nlocal = 1, no NCCL id, no IPC): one rank of a
     // P-way run on its own, every collective skipped; per-rank compute time of a partition
     // too large for loopback (Papers-shaped at P = 8).  Results are invalid by construction.
@@ -571,6 +588,30 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             t.hot_enc = hot_ok && want_hot_classes(ht);
             t.val = ht.val.empty() ? nullptr : b.take<float>(ht.val.size());
         };
+        // dense blocks (device copies of a DenseHost); every tile shares the rank's B-image scratch
+        size_t bimg_bytes = 0, part_floats = 0;
+        auto place_dense = [&](const DenseHost& dh, SpmmTile& t) {
+            t.dense = DenseTiles();
+            if (!dh.active) return;
+            DenseTiles& d = t.dense;
+            d.n_groups = dh.n_groups;
+            d.n_tiles = dh.n_tiles;
+            d.n_chunks = dh.n_chunks;
+            d.n_items = dh.n_items;
+            d.n_splits = dh.n_splits;
+            d.n_slots = dh.n_slots;
+            d.nnz = dh.nnz;
+            d.pieces = m->dense_pieces;
+            d.grp_rows = b.take<int32_t>(dh.grp_rows.size());
+            d.row_flag = b.take<uint8_t>(dh.row_flag.size());
+            d.work = b.take<int4>(dh.n_items);
+            d.splits = b.take<int4>(dh.n_splits);
+            d.tile_chunk = b.take<int32_t>(dh.tile_chunk.size());
+            d.chunk_cols = b.take<int32_t>(dh.chunk_cols.size());
+            d.A = reinterpret_cast<const uint8_t*>(b.take<uint16_t>(dh.A.size()));
+            bimg_bytes = std::max(bimg_bytes, dense_bimg_bytes(dh.n_chunks, m->dense_pieces));
+            part_floats = std::max(part_floats, dense_partial_floats(dh.n_slots));
+        };
         for (int j = 0; j < P; ++j) {
             // with stage groups only the local tile is launched per stage (the remote ones
             // live in the merged group tiles; mggcn_part_export_tile reads the host copies)
@@ -581,17 +622,33 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
                     continue;
                 }
                 SpmmTile& t = dir == 0 ? r.F[j] : r.B[j];
-                if (on_dev) place(dir == 0 ? r.tF(j) : r.tB(j), dir == 0 ? r.hF[j] : r.hB[j], t, true);
+                if (on_dev) {
+                    place(dir == 0 ? r.lF(j) : r.lB(j), dir == 0 ? r.hF[j] : r.hB[j], t, true);
+                    const std::vector<DenseHost>& dv = dir == 0 ? r.dF : r.dB;
+                    if (j < (int)dv.size()) place_dense(dv[j], t);
+                }
             }
+            if (pt->shared_fb) r.B[j] = r.F[j];
         }
         const int NG = n_groups(m);
         r.GF.assign(NG, SpmmTile());
         r.GB.assign(NG, SpmmTile());
         for (int g = 0; g < NG; ++g) {
-            place(r.gF[g], r.hgF[g], r.GF[g], false);
+            place(r.lgF(g), r.hgF[g], r.GF[g], false);
+            if (g < (int)r.dgF.size()) place_dense(r.dgF[g], r.GF[g]);
             if (pt->shared_fb) r.GB[g] = r.GF[g];
-            else place(r.gB[g], r.hgB[g], r.GB[g], false);
+            else {
+                place(r.lgB(g), r.hgB[g], r.GB[g], false);
+                if (g < (int)r.dgB.size()) place_dense(r.dgB[g], r.GB[g]);
+            }
         }
+        r.dense_bimg = bimg_bytes ? b.take<uint8_t>(bimg_bytes) : nullptr;
+        r.dense_partial = part_floats ? b.take<float>(part_floats) : nullptr;
+        for (auto* v : {&r.F, &r.B, &r.GF, &r.GB})
+            for (auto& t : *v) {
+                t.dense.bimg = r.dense_bimg;
+                t.dense.partial = r.dense_partial;
+            }
         r.inv_deg = b.take<float>(r.rows);
         for (int k = 0; k < 2; ++k) r.ybuf[k] = b.take<int32_t>(r.rows);
         r.Xs = r.Xbuf[0];
@@ -645,15 +702,37 @@ int upload_static(mggcn_model_s* m) {
                                        cudaMemcpyHostToDevice, m->cs));
                 return MGGCN_OK;
         };
+        auto upload_dense = [&](const DenseHost& dh, const SpmmTile& t) -> int {
+            if (!dh.active) return MGGCN_OK;
+            const DenseTiles& d = t.dense;
+            auto cp = [&](const void* dst, const void* src, size_t bytes) -> int {
+                if (bytes) CK(cudaMemcpyAsync(const_cast<void*>(dst), src, bytes, cudaMemcpyHostToDevice, m->cs));
+                return MGGCN_OK;
+            };
+            RC(cp(d.grp_rows, dh.grp_rows.data(), 4 * dh.grp_rows.size()));
+            RC(cp(d.row_flag, dh.row_flag.data(), dh.row_flag.size()));
+            RC(cp(d.work, dh.work.data(), 4 * dh.work.size()));
+            RC(cp(d.splits, dh.splits.data(), 4 * dh.splits.size()));
+            RC(cp(d.tile_chunk, dh.tile_chunk.data(), 4 * dh.tile_chunk.size()));
+            RC(cp(d.chunk_cols, dh.chunk_cols.data(), 4 * dh.chunk_cols.size()));
+            RC(cp(d.A, dh.A.data(), 2 * dh.A.size()));
+            return MGGCN_OK;
+        };
         for (int j = 0; j < pt->P; ++j)
             for (int dir = 0; dir < 2; ++dir) {
                 if (dir == 1 && pt->shared_fb) continue;
                 if (m->grouped() && j != r.rank) continue;
-                RC(upload(dir == 0 ? r.tF(j) : r.tB(j), dir == 0 ? r.hF[j] : r.hB[j], dir == 0 ? r.F[j] : r.B[j]));
+                RC(upload(dir == 0 ? r.lF(j) : r.lB(j), dir == 0 ? r.hF[j] : r.hB[j], dir == 0 ? r.F[j] : r.B[j]));
+                const std::vector<DenseHost>& dv = dir == 0 ? r.dF : r.dB;
+                if (j < (int)dv.size()) RC(upload_dense(dv[j], dir == 0 ? r.F[j] : r.B[j]));
             }
         for (size_t g = 0; g < r.GF.size(); ++g) {
-            RC(upload(r.gF[g], r.hgF[g], r.GF[g]));
-            if (!pt->shared_fb) RC(upload(r.gB[g], r.hgB[g], r.GB[g]));
+            RC(upload(r.lgF((int)g), r.hgF[g], r.GF[g]));
+            if (g < r.dgF.size()) RC(upload_dense(r.dgF[g], r.GF[g]));
+            if (!pt->shared_fb) {
+                RC(upload(r.lgB((int)g), r.hgB[g], r.GB[g]));
+                if (g < r.dgB.size()) RC(upload_dense(r.dgB[g], r.GB[g]));
+            }
         }
         if (pt->shared_fb)
             for (int j = 0; j < pt->P; ++j) r.B[j] = r.F[j];
@@ -1544,6 +1623,55 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
                 if (!r.part->shared_fb) {
                     merge_group_tiles(tb, m->max_rows_j, r.gB[g]);
                     build_items(r.gB[g], r.hgB[g], r.order_cache);
+                }
+            }
+        }
+    }
+    // Dense blocks of every launched tile (the local / per-stage tiles and the merged group
+    // tiles); their work items are rebuilt over the residual entries.
+    {
+        const char* e = getenv("MGGCN_DENSE_THR");
+        m->dense_thr = e ? atof(e) : kDenseThrDefault;
+        const char* pe = getenv("MGGCN_DENSE_PIECES");
+        m->dense_pieces = (pe && atoi(pe) == 2) ? 2 : 3;
+        const char* fe = getenv("MGGCN_DENSE_MINFRAC");
+        m->dense_min_frac = fe ? atof(fe) : kDenseMinFracDefault;
+        if (!(m->dense_thr > 0) || (!m->ranks.empty() && !m->ranks[0].coalesced)) m->dense_thr = 0;
+    }
+    if (m->dense_thr > 0) {
+        for (auto& r : m->ranks) {
+            r.dF.assign(m->P, DenseHost());
+            if (!r.part->shared_fb) r.dB.assign(m->P, DenseHost());
+            for (int j = 0; j < m->P; ++j) {
+                if (m->grouped() && j != r.rank) continue;
+                plan_dense(r.tF(j), m->dense_thr, m->dense_min_frac, r.dF[j]);
+                if (r.dF[j].active) {
+                    r.hF[j] = HostItems();
+                    build_items(r.lF(j), r.hF[j], r.order_cache);
+                }
+                if (!r.part->shared_fb) {
+                    plan_dense(r.tB(j), m->dense_thr, m->dense_min_frac, r.dB[j]);
+                    if (r.dB[j].active) {
+                        r.hB[j] = HostItems();
+                        build_items(r.lB(j), r.hB[j], r.order_cache);
+                    }
+                }
+            }
+            const int NG = n_groups(m);
+            r.dgF.assign(NG, DenseHost());
+            if (!r.part->shared_fb) r.dgB.assign(NG, DenseHost());
+            for (int g = 0; g < NG; ++g) {
+                plan_dense(r.gF[g], m->dense_thr, m->dense_min_frac, r.dgF[g]);
+                if (r.dgF[g].active) {
+                    r.hgF[g] = HostItems();
+                    build_items(r.lgF(g), r.hgF[g], r.order_cache);
+                }
+                if (!r.part->shared_fb) {
+                    plan_dense(r.gB[g], m->dense_thr, m->dense_min_frac, r.dgB[g]);
+                    if (r.dgB[g].active) {
+                        r.hgB[g] = HostItems();
+                        build_items(r.lgB(g), r.hgB[g], r.order_cache);
+                    }
                 }
             }
         }
@@ -2450,6 +2578,39 @@ extern "C" int mggcn_stage_groups(mggcn_model m, int32_t* sizes, int32_t cap) {
     const int ng = n_groups(m);
     for (int g = 0; g < ng && g < cap && sizes; ++g) sizes[g] = m->grp_b[g + 1] - m->grp_b[g];
     return ng;
+}
+
+extern "C" int mggcn_dense_stats(mggcn_model m, int64_t* out, int32_t n) {
+    MODEL_GUARD(m);
+    if (!out || n < 0) {
+        set_error("dense_stats: bad arguments");
+        return MGGCN_EINVAL;
+    }
+    // [0] blocks [1] entries in blocks [2] row groups [3] column chunks [4] entries of the launched
+    // tiles (coalesced, blocks + residual), over every rank of this model and both directions
+    int64_t v[5] = {0, 0, 0, 0, 0};
+    for (auto& r : m->ranks) {
+        for (const auto* dv : {&r.dF, &r.dB, &r.dgF, &r.dgB})
+            for (const DenseHost& d : *dv)
+                if (d.active) {
+                    v[0] += d.n_tiles;
+                    v[1] += d.nnz;
+                    v[2] += d.n_groups;
+                    v[3] += d.n_chunks;
+                    v[4] += d.nnz;
+                }
+        for (int j = 0; j < m->P; ++j) {
+            if (m->grouped() && j != r.rank) continue;
+            v[4] += r.lF(j).rowptr.back();
+            if (!r.part->shared_fb) v[4] += r.lB(j).rowptr.back();
+        }
+        for (int g = 0; g < n_groups(m); ++g) {
+            v[4] += r.lgF(g).rowptr.back();
+            if (!r.part->shared_fb) v[4] += r.lgB(g).rowptr.back();
+        }
+    }
+    for (int i = 0; i < n && i < 5; ++i) out[i] = v[i];
+    return 5;
 }
 
 extern "C" int mggcn_debug_poison(mggcn_model m, int32_t on) {

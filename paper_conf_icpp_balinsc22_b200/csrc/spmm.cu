@@ -112,8 +112,9 @@ __device__ __forceinline__ float ld_stream_f32(const float* p) {
     return v;
 }
 
-__device__ __forceinline__ float4 epilogue(float4 acc, const float4* out_row, int q, int flags, float scale) {
-    if (flags & SPMM_ACCUM) acc = f4_add(acc, out_row[q]);
+// accum: SPMM_ACCUM, or a row that already holds this stage's dense-block product (DenseTiles::row_flag)
+__device__ __forceinline__ float4 epilogue(float4 acc, const float4* out_row, int q, int flags, float scale, bool accum) {
+    if (accum) acc = f4_add(acc, out_row[q]);
     if (flags & SPMM_LAST) {
         acc.x *= scale; acc.y *= scale; acc.z *= scale; acc.w *= scale;
         if (flags & SPMM_RELU) {
@@ -149,7 +150,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, minb_for<G, CH>())
 spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const float4* __restrict__ B, int64_t ldb4,
                   float4* __restrict__ out, int64_t ldo4, float4* __restrict__ partial, int64_t ldp4,
-                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T) {
+                  const float* __restrict__ rowscale, int w4, int flags, uint32_t hot_T,
+                  const uint8_t* __restrict__ drow) {
     constexpr int S = 32 / G;
     // U entries per slot per group; U * S <= 32 so a group fits a 32-entry chunk
     constexpr int U = unroll_for<CH>() < G ? unroll_for<CH>() : G;
@@ -274,10 +276,11 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
                 }
             } else {
                 float4* orow = out + (int64_t)it.x * ldo4;
+                const bool accum = (flags & SPMM_ACCUM) || (drow && __ldg(drow + it.x));
 #pragma unroll
                 for (int ch = 0; ch < CH; ++ch) {
                     const int q = cl + ch * G;
-                    if (q < w4) orow[q] = epilogue(acc[ch], orow, q, flags, scale);
+                    if (q < w4) orow[q] = epilogue(acc[ch], orow, q, flags, scale, accum);
                 }
             }
         }
@@ -292,17 +295,18 @@ spmm_stage_kernel(const int4* __restrict__ items, int64_t n_items, const int32_t
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 spmm_fixup_warp_kernel(const int4* __restrict__ splits, int64_t n_splits, const float4* __restrict__ partial,
                        int64_t ldp4, float4* __restrict__ out, int64_t ldo4, const float* __restrict__ rowscale,
-                       int w4, int flags) {
+                       int w4, int flags, const uint8_t* __restrict__ drow) {
     const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (warp >= n_splits) return;
     const int4 sp = __ldg(splits + warp);
     float4* orow = out + (int64_t)sp.x * ldo4;
     const float scale = rowscale ? __ldg(rowscale + sp.x) : 1.f;
+    const bool accum = (flags & SPMM_ACCUM) || (drow && __ldg(drow + sp.x));
     for (int q = lane; q < w4; q += 32) {
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
         for (int s = 0; s < sp.z; ++s) acc = f4_add(acc, partial[(int64_t)(sp.y + s) * ldp4 + q]);
-        orow[q] = epilogue(acc, orow, q, flags, scale);
+        orow[q] = epilogue(acc, orow, q, flags, scale, accum);
     }
 }
 
@@ -314,7 +318,7 @@ constexpr int kFixWarps = 8;
 __global__ void __launch_bounds__(kFixWarps * 32)
 spmm_fixup_kernel(const int4* __restrict__ splits, int64_t n_splits, const float4* __restrict__ partial,
                   int64_t ldp4, float4* __restrict__ out, int64_t ldo4, const float* __restrict__ rowscale, int w4,
-                  int flags) {
+                  int flags, const uint8_t* __restrict__ drow) {
     __shared__ float4 red[kFixWarps][128];
     const int64_t sid = blockIdx.x;
     if (sid >= n_splits) return;
@@ -330,11 +334,12 @@ spmm_fixup_kernel(const int4* __restrict__ splits, int64_t n_splits, const float
     if (warp != 0) return;
     float4* orow = out + (int64_t)sp.x * ldo4;
     const float scale = rowscale ? __ldg(rowscale + sp.x) : 1.f;
+    const bool accum = (flags & SPMM_ACCUM) || (drow && __ldg(drow + sp.x));
     for (int q = lane; q < w4; q += 32) {
         float4 acc = red[0][q];
 #pragma unroll
         for (int w = 1; w < kFixWarps; ++w) acc = f4_add(acc, red[w][q]);
-        orow[q] = epilogue(acc, orow, q, flags, scale);
+        orow[q] = epilogue(acc, orow, q, flags, scale, accum);
     }
 }
 
@@ -378,7 +383,8 @@ void launch_one(const SpmmTile& t, const float4* B, int64_t ldb4, float4* out, i
     const int over = yenv > 1 ? yenv : ((flags & SPMM_YIELD) ? (yenv == 1 ? 1 : kYieldBlocks) : 1);
     const int64_t blocks = persistent_blocks<G, CH, V, H>(t.n_items, over);
     spmm_stage_kernel<G, CH, V, H><<<(unsigned)blocks, kWarpsPerBlock * 32, 0, s>>>(
-        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T);
+        t.items, t.n_items, t.col, t.val, B, ldb4, out, ldo4, partial, ldp4, rowscale, w4, flags, hot_T,
+        t.dense.row_flag);
 }
 
 template <int G, int CH>
@@ -432,6 +438,16 @@ cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4
 cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
                         const float* rowscale, int width, int flags, cudaStream_t s) {
     if (tile.nrows == 0) return cudaSuccess;
+    // Dense blocks (dense.cu) first: they store (first stage) or add their products into the
+    // rows of their groups; the gather kernel then adds the residual entries to those rows
+    // (DenseTiles::row_flag), writes the others as usual and applies the stage epilogue.
+    if (tile.dense.n_items > 0) {
+        for (int c0 = 0; c0 < width; c0 += kDenseMaxN) {
+            const int w = width - c0 < kDenseMaxN ? width - c0 : kDenseMaxN;
+            cudaError_t e = launch_dense(tile.dense, B + c0, ldb, out + c0, ldo, w, !(flags & SPMM_ACCUM), s);
+            if (e != cudaSuccess) return e;
+        }
+    }
     // a middle stage (accumulating, not the last) skips the tile's empty rows: their sum is
     // zero, so their output read-modify-write is a no-op (the first stage writes every row,
     // the last applies the row scale / ReLU to every row)
@@ -512,11 +528,12 @@ cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float
             const bool block = fix_env == 2 ? t.split < kSplit : fix_env == 1;
             if (block)
                 spmm_fixup_kernel<<<(unsigned)t.n_splits, kFixWarps * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4,
-                                                                                   Ow, ldo4, rowscale, w4, flags);
+                                                                                   Ow, ldo4, rowscale, w4, flags,
+                                                                                   t.dense.row_flag);
             else
                 spmm_fixup_warp_kernel<<<(unsigned)((t.n_splits + kWarpsPerBlock - 1) / kWarpsPerBlock),
                                          kWarpsPerBlock * 32, 0, s>>>(t.splits, t.n_splits, Pw, ldp4, Ow, ldo4,
-                                                                      rowscale, w4, flags);
+                                                                      rowscale, w4, flags, t.dense.row_flag);
             count_launches(1);
             e = cudaGetLastError();
             if (e != cudaSuccess) return e;

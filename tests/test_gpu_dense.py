@@ -1,0 +1,197 @@
+"""Dense blocks of the staged SpMM (dense.cu / dense_plan.cpp): the blocks of a
+stage tile with >= MGGCN_DENSE_THR density run on the tensor cores (bf16
+pieces of the fp32 operand, fp32 accumulate), the residual entries in the CSR
+gather kernel.  The stage product (Eq. 6 / Eq. 9) is unchanged up
+to the order of the fp32 additions, so: bit-exact on integer features,
+within 1e-5 of the fp64 oracle on random ones, and whole epochs within the
+north_star 1e-3 of the oracle epoch.  Needs a B200."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from helpers import csr_from_edges
+
+pytestmark = pytest.mark.gpu
+
+
+def rel(x, r):
+    return float(np.abs(np.asarray(x, np.float64) - r).max() / max(np.abs(r).max(), 1e-30))
+
+
+@pytest.fixture(autouse=True)
+def _any_coverage(monkeypatch):
+    """The tests force blocks at every threshold (the default MGGCN_DENSE_MINFRAC = 0.5 keeps
+    only tiles whose blocks hold half the entries)."""
+    monkeypatch.setenv("MGGCN_DENSE_MINFRAC", "0")
+
+
+@pytest.fixture(scope="module")
+def mg():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_icpp_balinsc22_b200 as mg
+    return mg
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def _pad(a, ld):
+    out = np.zeros((a.shape[0], ld), dtype=np.float32)
+    out[:, :a.shape[1]] = a
+    return out
+
+
+def _model(mg, n, rp, col, vals, dims, P, seed, flags=None):
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    flags = mg.MGGCN_F_OVERLAP if flags is None else flags
+    return GCN(n, rp, col, vals, dims, P=P, perm_seed=seed, flags=flags, loopback=P > 1)
+
+
+def _check(mg, n, rp, col, vals, P, width, seed, exact, min_frac=0.0):
+    dims = (max(width, 1), max(width, 1))
+    gm = _model(mg, n, rp, col, vals, dims, P, seed)
+    st = mg.mggcn_dense_stats(gm.m)
+    assert st["blocks"] > 0 and st["block_entries"] >= min_frac * st["entries"], st
+    pg = oracle.permute_graph(n, rp, col, vals, seed=seed)
+    ld = (width + 3) // 4 * 4
+    rng = np.random.default_rng(width + P)
+    Bm = (rng.integers(-64, 65, (n, width)) if exact else rng.standard_normal((n, width))).astype(np.float32)
+    dB = _dev(_pad(Bm, ld))
+    out = torch.zeros((n, ld), dtype=torch.float32, device="cuda")
+    # the backward direction of a pattern-only graph pre-scales B by 1/deg (Eq. 2): integer
+    # features stay exact there only for power-of-two degrees, so it is compared at 1e-5
+    pattern_scaled = vals is None
+    for d, csr in ((0, pg.At), (1, pg.A)):
+        out.fill_(7.0)    # stale values must not leak into rows the residual CSR leaves empty
+        torch.cuda.synchronize()
+        mg.mggcn_debug_spmm(gm.m, d, dB, ld, width, out, ld)
+        got = out[:, :width].cpu().numpy()
+        if exact and (d == 0 or not pattern_scaled):
+            ref = oracle.spmm(csr, Bm)
+            assert np.array_equal(got, ref), (d, np.abs(got - ref).max())
+        else:
+            refd = oracle.spmm(oracle.CSR(csr.rowptr, csr.col, csr.val.astype(np.float64)), Bm.astype(np.float64))
+            assert rel(got, refd) < 1e-5, (d, rel(got, refd))
+    gm.close()
+    return st
+
+
+def _dense_core(n, core, p, seed):
+    """Symmetric graph: a random core x core block of density p (the dense blocks) plus a
+    sparse ring over all n vertices (the residual), no self loops."""
+    rng = np.random.default_rng(seed)
+    M = rng.random((core, core)) < p
+    M = np.triu(M, 1)
+    u, v = np.nonzero(M)
+    edges = list(zip(u.tolist(), v.tolist())) + list(zip(v.tolist(), u.tolist()))
+    edges += [(i, (i + 1) % n) for i in range(n)] + [((i + 1) % n, i) for i in range(n)]
+    return csr_from_edges(n, edges)
+
+
+@pytest.mark.parametrize("P", [1, 2, 3])
+@pytest.mark.parametrize("width", [4, 16, 44, 100, 256, 300])
+def test_dense_blocks_exact(mg, monkeypatch, P, width):
+    """Integer features: the bf16 hi piece holds them exactly, products and fp32 sums are
+    exact on both paths -> bit-exact against the oracle, ragged widths and > 256 (windows)."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.05")
+    n = 1500
+    rp, col, _ = _dense_core(n, 700, 0.3, 1)
+    _check(mg, n, rp, col, None, P, width, seed=3, exact=True, min_frac=0.5)
+
+
+@pytest.mark.parametrize("P", [1, 2, 4])
+@pytest.mark.parametrize("width", [8, 48, 128, 256, 600])
+@pytest.mark.parametrize("thr", ["0.01", "0.03", "0.2"])
+def test_dense_blocks_rmat(mg, monkeypatch, P, width, thr):
+    """R-MAT with hubs and duplicates (multiplicity values), random features: within 1e-5."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", thr)
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    _check(mg, n, rp, col, None, P, width, seed=9, exact=False)
+
+
+@pytest.mark.parametrize("pieces", ["2", "3"])
+def test_dense_pieces(mg, monkeypatch, pieces):
+    """bf16 hi + mid (16 significant bits) vs hi + mid + lo: both inside 1e-5 / 1e-3."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.01")
+    monkeypatch.setenv("MGGCN_DENSE_PIECES", pieces)
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    gm = _model(mg, n, rp, col, None, (256, 256), 1, 9)
+    pg = oracle.permute_graph(n, rp, col, None, seed=9)
+    Bm = np.random.default_rng(0).standard_normal((n, 256)).astype(np.float32)
+    out = torch.zeros((n, 256), dtype=torch.float32, device="cuda")
+    mg.mggcn_debug_spmm(gm.m, 0, _dev(Bm), 256, 256, out, 256)
+    refd = oracle.spmm(oracle.CSR(pg.At.rowptr, pg.At.col, pg.At.val.astype(np.float64)), Bm.astype(np.float64))
+    e = rel(out.cpu().numpy(), refd)
+    assert e < (1e-5 if pieces == "3" else 1e-4), e
+    gm.close()
+
+
+def test_dense_off_matches_threshold_zero(mg, monkeypatch):
+    """MGGCN_DENSE_THR=0 turns the blocks off (the pure gather path)."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0")
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] == 0
+    gm.close()
+
+
+def test_dense_weighted_values_stay_in_csr(mg, monkeypatch):
+    """Weighted graph: only entries exact in bf16 may enter a block; the rest stay in the
+    residual CSR; result within 1e-5 either way."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.02")
+    n = 1200
+    rp, col, _ = _dense_core(n, 600, 0.4, 2)
+    rng = np.random.default_rng(5)
+    vals = np.where(rng.random(len(col)) < 0.5, 2.0, rng.random(len(col)) + 0.1).astype(np.float32)
+    # weighted graphs need a symmetric value pattern only for shared tiles; keep it general
+    gm = _model(mg, n, rp, col, vals, (64, 64), 1, 4)
+    st = mg.mggcn_dense_stats(gm.m)
+    gm.close()
+    if st["blocks"] == 0:
+        pytest.skip("no block reached the threshold with the exact half of the values")
+    _check(mg, n, rp, col, vals, 1, 64, seed=4, exact=False)
+
+
+@pytest.mark.parametrize("P", [1, 4])
+def test_dense_epoch_vs_oracle(mg, monkeypatch, P):
+    """A whole epoch (forward, loss, backward, W_G, Adam) with the dense blocks on, against
+    the oracle epoch: north_star's 1e-3 on logits, loss, W_G and the Adam state."""
+    from test_gpu_epoch import compare, run_library
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.02")
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 21)
+    dims = (64, 256, 256, 41)
+    X = gen.features(n, dims[0], 5)
+    y = gen.labels(n, dims[-1], 6)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 7 + l) for l in range(len(dims) - 1)]
+    from paper_conf_icpp_balinsc22_b200 import GCN
+    gm = GCN(n, rp, col, None, dims, P=P, perm_seed=11, flags=mg.MGGCN_F_OVERLAP, loopback=P > 1)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] > 0
+    gm.close()
+    pg = oracle.permute_graph(n, rp, col, None, seed=11)
+    ref = oracle.epoch(pg, X, y, Ws, P=P)
+    lib = run_library(mg, n, rp, col, None, X, y, Ws, dims, P, 11, mg.MGGCN_F_OVERLAP)
+    compare(lib, ref, dims)
+
+
+def test_dense_min_frac_rule(mg, monkeypatch):
+    """A tile whose blocks would hold less than MGGCN_DENSE_MINFRAC of its entries keeps the
+    pure gather path (Products-shaped tiles)."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.03")
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    st = mg.mggcn_dense_stats(gm.m)
+    gm.close()
+    frac = st["block_entries"] / st["entries"]
+    assert 0 < frac < 0.99
+    monkeypatch.setenv("MGGCN_DENSE_MINFRAC", str(min(1.0, frac + 0.01)))
+    gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] == 0
+    gm.close()

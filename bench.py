@@ -274,6 +274,23 @@ def stored_traffic(workload, P):
         "same_build": (d.get("so_sha256") == cur) if d.get("so_sha256") else None}
 
 
+def dense_summary(st, dims):
+    """The dense-block part of the SpMM (DESIGN §6 "Dense blocks"): blocks, the share of the
+    coalesced entries they cover, and the tensor work they issue per epoch (128 x 32 x N x 2 flops
+    per block per bf16 piece, N = the SpMM width rounded up to 16 per 256-column window)."""
+    if not st or not st.get("blocks"):
+        return {"blocks": 0, "note": "no tile passed the dense rules (MGGCN_DENSE_THR / _MINFRAC / _MIN_ROWS)"}
+    pieces = int(os.environ.get("MGGCN_DENSE_PIECES", "3")) if os.environ.get("MGGCN_DENSE_PIECES") == "2" else 3
+    flops = 0.0
+    for wdt in spmm_widths(dims):
+        n_pad = sum((min(256, wdt - c0) + 15) // 16 * 16 for c0 in range(0, wdt, 256))
+        flops += st["blocks"] * 128 * 32 * n_pad * 2 * pieces
+    return {"blocks": st["blocks"], "block_entries": st["block_entries"], "entries": st["entries"],
+            "entry_frac": st["block_entries"] / max(st["entries"], 1), "row_groups": st["row_groups"],
+            "chunks": st["chunks"], "pieces": pieces, "mma_tflop_per_epoch": flops / 1e12,
+            "thr": os.environ.get("MGGCN_DENSE_THR", "default 0.03")}
+
+
 def spmm_widths(dims):
     """Widths of the SpMMs of one epoch (§4.4 order rule C10, first-layer skip C11)."""
     ws = []
@@ -513,6 +530,7 @@ def main():
     work = gm.epoch_work()
     work_detail = gm.epoch_work_detail()
     stage_groups = mg.mggcn_stage_groups(gm.m)
+    dense_stats = mg.mggcn_dense_stats(gm.m)
     # ---- one extra eager epoch with the per-stage timeline (not timed)
     timeline = None
     try:
@@ -740,7 +758,8 @@ def main():
         "e2e": e2e,
         "gpu_launches": int(launches),
         "clocks": clk,
-        "roofline": {"bound": "hbm", "kernel": "spmm_stage (staged CSR SpMM, F2/B1)",
+        "roofline": {"bound": "hbm", "kernel": "SpMM stage (F2/B1): dense_tile_kernel (tcgen05 bf16x3 blocks) + "
+                                               "spmm_stage_kernel (CSR gather of the residual entries)",
                      "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
                      "traffic": traffic, "traffic_source": traffic_src, "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": bytes_per_launch,
@@ -751,10 +770,11 @@ def main():
                              "tiles, rowptr, each gathered and each output row once) / measured mean launch time "
                              "(CUDA events on the compute stream); struct_bytes_per_launch = the same with the "
                              "device tiles' coalesced (index + multiplicity) entries; gather_model_GBps = "
-                             "coalesced nnz * width * 4 B / time; a launch = one SpMM stage (its column-window "
-                             "kernels + hub fix-up)",
+                             "coalesced nnz * width * 4 B / time; a launch = one SpMM stage (B images + dense "
+                             "blocks + their fix-up, the column-window gather kernels + hub fix-up)",
                      "l2_gather": l2_gather},
         "epoch_roofline": epoch_roofline,
+        "dense": dense_summary(dense_stats, w.dims),
         "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
         "gemm": {"tflops": gemm_tflops, "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps,
                  "frac_model_flops": gemm_tflops / tf32_peak if gemm_tflops else None,

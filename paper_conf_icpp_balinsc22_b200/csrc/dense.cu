@@ -189,6 +189,7 @@ dense_bimg_kernel(const int32_t* __restrict__ chunk_cols, const float* __restric
 struct DnParams {
     const int32_t* grp_rows;
     const int4* work;
+    const int32_t* bin_beg;
     float* partial;
     const int32_t* tile_chunk;
     const uint8_t* A;
@@ -237,13 +238,14 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    const int w_end = __ldg(p.bin_beg + blockIdx.x + 1);   // this CTA's bin of work items (host LPT)
 
     if (warp == kDnProdWarp) {
         if (lane == 0) {
             const uint64_t pa = policy_first(), pb = policy_last();
             int s = 0;
             uint32_t ph = 0;
-            for (int w = blockIdx.x; w < p.n_items; w += gridDim.x) {
+            for (int w = __ldg(p.bin_beg + blockIdx.x); w < w_end; ++w) {
                 const int4 it = __ldg(p.work + w);
                 for (int t = it.y; t < it.z; ++t) {
                     const int c = __ldg(p.tile_chunk + t);
@@ -264,7 +266,7 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
                                    ((uint32_t)(kDenseM >> 4) << 24);
             int s = 0, a = 0;
             uint32_t ph = 0, aph = 0;
-            for (int w = blockIdx.x; w < p.n_items; w += gridDim.x) {
+            for (int w = __ldg(p.bin_beg + blockIdx.x); w < w_end; ++w) {
                 const int4 it = __ldg(p.work + w);
                 const int t0 = it.y, t1 = it.z;
                 uint32_t d = 0;
@@ -309,7 +311,7 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
         const int quad = warp & 3, h = warp >> 2;
         const int slot = quad * 32 + lane;
         const int cb = h * 128;                       // first column of this warp
-        for (int w = blockIdx.x; w < p.n_items; w += gridDim.x) {
+        for (int w = __ldg(p.bin_beg + blockIdx.x); w < w_end; ++w) {
             const int4 it = __ldg(p.work + w);
             const int row = __ldg(p.grp_rows + (int64_t)it.x * kDenseM + slot);
             const int nchains = (it.z - it.y + p.drain - 1) / p.drain;
@@ -386,17 +388,6 @@ dense_fixup_kernel(const int4* __restrict__ splits, const int32_t* __restrict__ 
     *o = x;
 }
 
-int dn_sm_count() {
-    static int n = 0;
-    if (n == 0) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-        if (n <= 0) n = 148;
-    }
-    return n;
-}
-
 }  // namespace
 
 int dense_stages_for(int N, int pieces) {
@@ -430,6 +421,7 @@ cudaError_t launch_dense(const DenseTiles& d, const float* B, int64_t ldb, float
     DnParams p;
     p.grp_rows = d.grp_rows;
     p.work = d.work;
+    p.bin_beg = d.bin_beg;
     p.partial = d.partial;
     p.tile_chunk = d.tile_chunk;
     p.A = d.A;
@@ -449,7 +441,7 @@ cudaError_t launch_dense(const DenseTiles& d, const float* B, int64_t ldb, float
         if (drain_env < 0) drain_env = 0;
     }
     p.drain = drain_env > 0 ? drain_env : kDenseDrain;
-    const int grid = (int)(d.n_items < dn_sm_count() ? d.n_items : dn_sm_count());
+    const int grid = (int)d.n_bins;
     dense_tile_kernel<<<grid, kDnThreads, smem, s>>>(p);
     count_launches(2);
     e = cudaGetLastError();

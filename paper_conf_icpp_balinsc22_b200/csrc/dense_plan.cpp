@@ -36,10 +36,15 @@ inline bool bf16_exact(float v) {
 }  // namespace
 
 // (global scope, like HostTile and DenseHost in internal.h)
-void plan_dense(const HostTile& t, double thr, double min_frac, DenseHost& d) {
+void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows, DenseHost& d) {
     d = DenseHost();
     const int64_t nr = t.nrows, nc = t.ncols;
     if (thr <= 0 || nr == 0 || nc == 0 || t.rowptr.empty() || t.rowptr[nr] == 0) return;
+    // ... and only for tiles of >= min_rows rows: a dense launch costs a fixed ~15 us (B images,
+    // the persistent kernel's ramp, the fix-up) that the small stage tiles of an 8-way split do
+    // not amortise (SOLO rank 0: Reddit-shaped P = 8 3.69 -> 3.68 ms, Proteins-shaped P = 8
+    // 1.46 -> 1.70 ms with blocks; P = 4 Reddit 6.61 -> 5.62 ms; profiles/r02_dense_solo_ab.jsonl)
+    if (nr < min_rows) return;
     const int64_t min_cnt = std::max<int64_t>(1, (int64_t)std::ceil(thr * TM * TK));
     const bool pat = t.val.empty();
     auto ok = [&](int64_t e) { return pat || bf16_exact(t.val[e]); };
@@ -179,7 +184,27 @@ void plan_dense(const HostTile& t, double thr, double min_frac, DenseHost& d) {
         return a[2] - a[1] > b[2] - b[1];
     });
     d.n_items = (int64_t)items.size();
-    for (const auto& it : items) d.work.insert(d.work.end(), it.begin(), it.end());
+    // LPT: items (longest first) go to the least-loaded of kSMs bins, one bin per CTA of the
+    // persistent launch (a strided walk of the sorted list gave the SMs 48-87 % tensor-pipe
+    // activity, profiles/r02_dense_ncu.md); cost = blocks + 2 (the chain drains and stores)
+    const int64_t nb = std::min<int64_t>(kSMs, d.n_items);
+    std::vector<std::vector<int32_t>> bins(nb);
+    std::vector<std::pair<int64_t, int64_t>> heap;   // (load, bin), min-heap
+    for (int64_t b = 0; b < nb; ++b) heap.push_back({0, b});
+    auto cmp = [](const std::pair<int64_t, int64_t>& x, const std::pair<int64_t, int64_t>& y) { return x > y; };
+    for (int64_t i = 0; i < d.n_items; ++i) {
+        std::pop_heap(heap.begin(), heap.end(), cmp);
+        auto& top = heap.back();
+        bins[top.second].push_back((int32_t)i);
+        top.first += (items[i][2] - items[i][1]) + 2;
+        std::push_heap(heap.begin(), heap.end(), cmp);
+    }
+    d.bin_beg.push_back(0);
+    for (int64_t b = 0; b < nb; ++b) {
+        for (int32_t i : bins[b]) d.work.insert(d.work.end(), items[i].begin(), items[i].end());
+        d.bin_beg.push_back((int32_t)(d.work.size() / 4));
+    }
+    d.n_bins = nb;
 
     // 4. A images and the residual tile
     d.A.assign((size_t)ntiles * TM * TK, 0);

@@ -56,12 +56,15 @@ struct DenseHost {
     std::vector<int32_t> work;          // n_items * 4
     std::vector<int32_t> splits;        // n_splits * 4 (last: 0)
     int64_t n_items = 0, n_splits = 0, n_slots = 0;
+    std::vector<int32_t> bin_beg;       // n_bins + 1: CTA b runs work items [bin_beg[b], bin_beg[b+1])
+    int64_t n_bins = 0;
     std::vector<int32_t> tile_chunk;    // n_tiles
     std::vector<int32_t> chunk_cols;    // n_chunks * 32, -1 = empty slot
     std::vector<uint16_t> A;            // n_tiles * 128 * 32 bf16, K-major SWIZZLE_64B image per block
 };
-// thr <= 0, nothing dense, or the blocks holding < min_frac of the entries => d.active = false.
-void plan_dense(const HostTile& t, double thr, double min_frac, DenseHost& d);
+// thr <= 0, a tile of fewer than min_rows rows, nothing dense, or the blocks holding < min_frac
+// of the entries => d.active = false.
+void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows, DenseHost& d);
 
 // One rank's 1D partition of the permuted graph.
 struct mggcn_part_s {

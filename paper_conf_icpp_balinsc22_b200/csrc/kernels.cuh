@@ -43,14 +43,17 @@ constexpr int kDenseMaxN = 256;    // features per launch (wider operands: 256-c
 constexpr double kDenseThrDefault = 0.03;
 // a tile uses blocks only if they hold >= this share of its entries; MGGCN_DENSE_MINFRAC overrides
 constexpr double kDenseMinFracDefault = 0.5;
+// ... and only in tiles of at least this many rows (MGGCN_DENSE_MIN_ROWS overrides)
+constexpr int64_t kDenseMinRowsDefault = 49152;
 struct DenseTiles {
     int64_t n_groups = 0, n_tiles = 0, n_chunks = 0;
-    int64_t n_items = 0, n_splits = 0, n_slots = 0;
+    int64_t n_items = 0, n_splits = 0, n_slots = 0, n_bins = 0;
     int64_t nnz = 0;                   // entries (coalesced) covered by the blocks
     int pieces = 3;                    // bf16 pieces of the B operand (2: hi + mid, 3: + lo)
     const int32_t* grp_rows = nullptr;   // [n_groups][kDenseM] output row of each slot, -1 = none
     const uint8_t* row_flag = nullptr;   // [nrows] 1 = row of a group: the gather kernel adds to its output
     const int4* work = nullptr;          // [n_items] {group, first block, end block, partial slot or -1}
+    const int32_t* bin_beg = nullptr;    // [n_bins + 1] CTA b of the launch runs items [bin_beg[b], bin_beg[b+1])
     const int4* splits = nullptr;        // [n_splits] {group, first slot, slots, 0}: groups cut into items
     float* partial = nullptr;            // scratch: [n_slots][kDenseM][N]
     const int32_t* tile_chunk = nullptr; // [n_tiles] column chunk of each block

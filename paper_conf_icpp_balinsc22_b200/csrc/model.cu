@@ -309,6 +309,7 @@ struct mggcn_model_s {
     // 0 = off) and bf16 pieces of the B operand (MGGCN_DENSE_PIECES, 2 or 3)
     double dense_thr = 0;
     double dense_min_frac = 0.5;    // MGGCN_DENSE_MINFRAC: blocks must hold this share of a tile's entries
+    int64_t dense_min_rows = 0;     // MGGCN_DENSE_MIN_ROWS: ... in tiles of at least this many rows
     int dense_pieces = 3;
     // SOLO timing mode (MGGCN_F_NO_BCAST, P > 1, nlocal = 1, no NCCL id, no IPC): one rank of a
     // P-way run on its own, every collective skipped; per-rank compute time of a partition
@@ -600,12 +601,14 @@ void plan_buffers(mggcn_model_s* m, Bump& b) {
             d.n_items = dh.n_items;
             d.n_splits = dh.n_splits;
             d.n_slots = dh.n_slots;
+            d.n_bins = dh.n_bins;
             d.nnz = dh.nnz;
             d.pieces = m->dense_pieces;
             d.grp_rows = b.take<int32_t>(dh.grp_rows.size());
             d.row_flag = b.take<uint8_t>(dh.row_flag.size());
             d.work = b.take<int4>(dh.n_items);
             d.splits = b.take<int4>(dh.n_splits);
+            d.bin_beg = b.take<int32_t>(dh.bin_beg.size());
             d.tile_chunk = b.take<int32_t>(dh.tile_chunk.size());
             d.chunk_cols = b.take<int32_t>(dh.chunk_cols.size());
             d.A = reinterpret_cast<const uint8_t*>(b.take<uint16_t>(dh.A.size()));
@@ -713,6 +716,7 @@ int upload_static(mggcn_model_s* m) {
             RC(cp(d.row_flag, dh.row_flag.data(), dh.row_flag.size()));
             RC(cp(d.work, dh.work.data(), 4 * dh.work.size()));
             RC(cp(d.splits, dh.splits.data(), 4 * dh.splits.size()));
+            RC(cp(d.bin_beg, dh.bin_beg.data(), 4 * dh.bin_beg.size()));
             RC(cp(d.tile_chunk, dh.tile_chunk.data(), 4 * dh.tile_chunk.size()));
             RC(cp(d.chunk_cols, dh.chunk_cols.data(), 4 * dh.chunk_cols.size()));
             RC(cp(d.A, dh.A.data(), 2 * dh.A.size()));
@@ -1636,6 +1640,8 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         m->dense_pieces = (pe && atoi(pe) == 2) ? 2 : 3;
         const char* fe = getenv("MGGCN_DENSE_MINFRAC");
         m->dense_min_frac = fe ? atof(fe) : kDenseMinFracDefault;
+        const char* me = getenv("MGGCN_DENSE_MIN_ROWS");
+        m->dense_min_rows = me ? atoll(me) : kDenseMinRowsDefault;
         if (!(m->dense_thr > 0) || (!m->ranks.empty() && !m->ranks[0].coalesced)) m->dense_thr = 0;
     }
     if (m->dense_thr > 0) {
@@ -1644,13 +1650,13 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
             if (!r.part->shared_fb) r.dB.assign(m->P, DenseHost());
             for (int j = 0; j < m->P; ++j) {
                 if (m->grouped() && j != r.rank) continue;
-                plan_dense(r.tF(j), m->dense_thr, m->dense_min_frac, r.dF[j]);
+                plan_dense(r.tF(j), m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dF[j]);
                 if (r.dF[j].active) {
                     r.hF[j] = HostItems();
                     build_items(r.lF(j), r.hF[j], r.order_cache);
                 }
                 if (!r.part->shared_fb) {
-                    plan_dense(r.tB(j), m->dense_thr, m->dense_min_frac, r.dB[j]);
+                    plan_dense(r.tB(j), m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dB[j]);
                     if (r.dB[j].active) {
                         r.hB[j] = HostItems();
                         build_items(r.lB(j), r.hB[j], r.order_cache);
@@ -1661,13 +1667,13 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
             r.dgF.assign(NG, DenseHost());
             if (!r.part->shared_fb) r.dgB.assign(NG, DenseHost());
             for (int g = 0; g < NG; ++g) {
-                plan_dense(r.gF[g], m->dense_thr, m->dense_min_frac, r.dgF[g]);
+                plan_dense(r.gF[g], m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dgF[g]);
                 if (r.dgF[g].active) {
                     r.hgF[g] = HostItems();
                     build_items(r.lgF(g), r.hgF[g], r.order_cache);
                 }
                 if (!r.part->shared_fb) {
-                    plan_dense(r.gB[g], m->dense_thr, m->dense_min_frac, r.dgB[g]);
+                    plan_dense(r.gB[g], m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dgB[g]);
                     if (r.dgB[g].active) {
                         r.hgB[g] = HostItems();
                         build_items(r.lgB(g), r.hgB[g], r.order_cache);

@@ -182,6 +182,8 @@ def main():
         "n": w.n, "nnz": w.m, "dims": list(w.dims), "rank_rows": int(rows),
         "compute_ms_per_epoch": ms,
         "stage_groups": mg.mggcn_stage_groups(gm.m),
+        "dense": dict(mg.mggcn_dense_stats(gm.m), thr=os.environ.get("MGGCN_DENSE_THR", "default"),
+                      min_rows=os.environ.get("MGGCN_DENSE_MIN_ROWS", "default")),
         "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
         "workspace_GiB": gm.ws_bytes / 2**30,
         "device_mem_reserved_GiB": torch.cuda.memory_reserved() / 2**30,

@@ -29,6 +29,9 @@ METRICS = [
     ("lts__t_sector_hit_rate.pct", "L2 hit %"),
     ("l1tex__t_sector_hit_rate.pct", "L1 hit %"),
     ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed", "tensor pipe active %"),
+    ("sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_active", "tcgen05 pipe active % (of active cycles)"),
+    ("sm__pipe_tc_cycles_active.min.pct_of_peak_sustained_active", "tcgen05 pipe active %, least busy SM"),
+    ("sm__pipe_tc_cycles_active.max.pct_of_peak_sustained_active", "tcgen05 pipe active %, busiest SM"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved occupancy %"),
     ("launch__registers_per_thread", "registers/thread"),
     ("launch__grid_size", "grid"),
@@ -94,7 +97,7 @@ def main():
         lines.append(f"| **total** | {len(ep)} | {tot / 1e3:.1f} | 100% |")
         lines.append("")
     traffic = {}
-    for name in ("spmm_wide", "spmm_narrow", "gemm_rows", "gemm_wgrad"):
+    for name in ("dense_tile", "spmm_wide", "spmm_narrow", "gemm_rows", "gemm_wgrad"):
         rep = os.path.join(OUT, f"{tag}_{name}.ncu-rep")
         if not os.path.exists(rep):
             continue
@@ -120,7 +123,7 @@ def main():
         lines.append("| top stall reasons (cycles / issued inst) | " +
                      ", ".join(f"{s} {v:.2f}" for v, s in stalls[:4]) + " |")
         lines.append("")
-        if name.startswith("spmm") and "dram__bytes_read.sum" in d:
+        if (name.startswith("spmm") or name == "dense_tile") and "dram__bytes_read.sum" in d:
             traffic[name] = to_bytes(*d["dram__bytes_read.sum"]) + to_bytes(*d["dram__bytes_write.sum"])
             traffic[name + "_ms"] = float(d["gpu__time_duration.sum"][1]) * (
                 1e-3 if d["gpu__time_duration.sum"][0] == "us" else 1.0)
@@ -128,7 +131,10 @@ def main():
         # an epoch has 4 wide (256) and 2 narrow (41 -> 48) SpMM stages for the Reddit config; a wide
         # stage is 2 column-window launches of 128 floats (spmm.cu launch_spmm), the capture is one window
         nwin = int(os.environ.get("WIDE_WINDOWS", "2" if wl == "reddit" else "1"))
-        wide, narrow = nwin * traffic["spmm_wide"], traffic.get("spmm_narrow", traffic["spmm_wide"])
+        # a wide stage also runs the dense blocks (one dense_tile_kernel launch, captured separately;
+        # the narrow stage's dense launch is not captured, so `narrow` counts its gather only)
+        wide = nwin * traffic["spmm_wide"] + traffic.get("dense_tile", 0.0)
+        narrow = traffic.get("spmm_narrow", traffic["spmm_wide"])
         avg = (4 * wide + 2 * narrow) / 6 if wl == "reddit" else wide
         import hashlib
         so = os.path.join(ROOT, "paper_conf_icpp_balinsc22_b200", "libmggcn.so")
@@ -138,10 +144,11 @@ def main():
         json.dump({"workload": wl, "P": 1, "tag": tag, "dram_bytes_per_launch": avg,
                    "so_sha256": so_sha, "git_sha": git_sha,
                    "dram_bytes_wide_launch": wide, "dram_bytes_narrow_launch": narrow,
+                   "dram_bytes_dense_tile_launch": traffic.get("dense_tile"),
                    "wide_windows": nwin,
                    "how": "ncu --set full, dram__bytes_read.sum + dram__bytes_write.sum, one launch each "
-                          "(a wide stage = wide_windows window launches); epoch average = (4 wide + 2 narrow) / 6 "
-                          "for reddit"},
+                          "(a wide stage = wide_windows gather window launches + the dense_tile launch); epoch average = "
+                          "(4 wide + 2 narrow) / 6 for reddit"},
                   open(os.path.join(PROF, f"spmm_traffic_{wl}_P1.json"), "w"), indent=1)
     open(os.path.join(PROF, f"{tag}_summary.md"), "w").write("\n".join(lines) + "\n")
     print("\n".join(lines))

@@ -22,7 +22,7 @@ int main(int argc, char** argv) {
     t.rowptr.push_back(0);
     for (int i = 0; i < n; ++i) { std::sort(adj[i].begin(), adj[i].end()); adj[i].erase(std::unique(adj[i].begin(), adj[i].end()), adj[i].end());
         for (int c : adj[i]) { t.col.push_back(c); t.val.push_back(1.f + (rng() % 3)); } t.rowptr.push_back(t.col.size()); }
-    DenseHost d; plan_dense(t, thr, 0.0, d);
+    DenseHost d; plan_dense(t, thr, 0.0, 0, d);
     printf("active %d groups %ld tiles %ld chunks %ld nnz %ld items %ld splits %ld slots %ld resid %d total %zu\n", d.active, d.n_groups, d.n_tiles, d.n_chunks, d.nnz, d.n_items, d.n_splits, d.n_slots, d.active ? d.resid.rowptr.back() : -1, t.col.size());
     // reconstruct dense matrix from A images
     std::vector<double> M((size_t)n * n, 0), R((size_t)n * n, 0);
@@ -40,6 +40,8 @@ int main(int argc, char** argv) {
                     int col = d.chunk_cols[c*32+k];
                     if (v != 0) { if (row < 0 || col < 0) { printf("bad\n"); return 1; } R[(size_t)row*n+col] += v; } } } } }
     if ((int64_t)cover.size() != d.n_tiles) { printf("cover %zu\n", cover.size()); return 1; }
+    if (d.active && (d.bin_beg.empty() || d.bin_beg.front() != 0 || d.bin_beg.back() != d.n_items ||
+                     (int64_t)d.bin_beg.size() != d.n_bins + 1)) { printf("bins\n"); return 1; }
     for (auto& kv : cover) if (kv.second != 1) { printf("dup cover\n"); return 1; }
     double err = 0; for (size_t i = 0; i < M.size(); ++i) err = std::max(err, std::abs(M[i]-R[i]));
     int nflag = 0; for (auto f : d.row_flag) nflag += f;

@@ -23,8 +23,10 @@ def rel(x, r):
 @pytest.fixture(autouse=True)
 def _any_coverage(monkeypatch):
     """The tests force blocks at every threshold (the default MGGCN_DENSE_MINFRAC = 0.5 keeps
-    only tiles whose blocks hold half the entries)."""
+    only tiles whose blocks hold half the entries, MGGCN_DENSE_MIN_ROWS = 49152 only tiles of
+    that many rows)."""
     monkeypatch.setenv("MGGCN_DENSE_MINFRAC", "0")
+    monkeypatch.setenv("MGGCN_DENSE_MIN_ROWS", "0")
 
 
 @pytest.fixture(scope="module")
@@ -193,5 +195,20 @@ def test_dense_min_frac_rule(mg, monkeypatch):
     assert 0 < frac < 0.99
     monkeypatch.setenv("MGGCN_DENSE_MINFRAC", str(min(1.0, frac + 0.01)))
     gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] == 0
+    gm.close()
+
+
+def test_dense_min_rows_rule(mg, monkeypatch):
+    """Tiles with fewer than MGGCN_DENSE_MIN_ROWS rows keep the pure gather path (the small
+    stage tiles of an 8-way split); P = 2 halves the rows of every tile."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.03")
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    monkeypatch.setenv("MGGCN_DENSE_MIN_ROWS", "3000")
+    gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] > 0
+    gm.close()
+    gm = _model(mg, n, rp, col, None, (64, 64), 2, 9)
     assert mg.mggcn_dense_stats(gm.m)["blocks"] == 0
     gm.close()

@@ -318,9 +318,11 @@ def line_bytes(width):
     return tot
 
 
-def l2_gather_roofline(dims, work, spmm_ms_per_epoch, cache=False):
+def l2_gather_roofline(dims, work, spmm_ms_per_epoch, cache=False, gathered_frac=1.0):
     ws = spmm_widths(dims)
-    nnz = work["spmm_gather_bytes"] / (4.0 * sum(ws))          # coalesced non-zeros per SpMM (all ranks' tiles)
+    # coalesced non-zeros per SpMM (all ranks' tiles) that the CSR kernel gathers: the entries of
+    # the dense blocks run on the tensor cores instead
+    nnz = work["spmm_gather_bytes"] / (4.0 * sum(ws)) * gathered_frac
     lb = nnz * sum(line_bytes(x) for x in ws)
     ach = lb / (spmm_ms_per_epoch * 1e-3) / 1e9 if spmm_ms_per_epoch > 0 else 0.0
     return {"bound": "l2 (SM<-L2 line rate of random row gathers)", "achieved": ach, "peak": L2_GATHER_PEAK_GBPS,
@@ -713,7 +715,12 @@ def main():
     gather_gbs = (wd["spmm_gather_bytes"] / max(launches_per_epoch, 1)) / (spmm_launch_ms * 1e-3) / 1e9 \
         if spmm_ms > 0 else 0.0
     traffic, traffic_src = stored_traffic(args.workload, P)
-    l2_gather = l2_gather_roofline(w.dims, work, spmm_ms / args.steps, cache=False)
+    gathered_frac = 1.0 - (dense_stats["block_entries"] / dense_stats["entries"]
+                           if dense_stats.get("entries") else 0.0)
+    l2_gather = l2_gather_roofline(w.dims, work, spmm_ms / args.steps, cache=False, gathered_frac=gathered_frac)
+    l2_gather["gathered_entry_frac"] = gathered_frac
+    l2_gather["note"] = ("line bytes of the gathered (residual) entries over the whole SpMM time, which also "
+                         "contains the dense blocks' kernels: a lower bound on the gather kernel's own rate")
     gemm_ms, gemm_n = prof["gemm"]
     # dense TF32 peak = the measured bf16 peak x the nominal tf32 : bf16 ratio (1 : 2); the GEMMs are
     # timed inside a long epoch, so the sustained figure is the denominator of their fraction

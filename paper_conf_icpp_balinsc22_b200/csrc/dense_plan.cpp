@@ -41,9 +41,11 @@ void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows
     const int64_t nr = t.nrows, nc = t.ncols;
     if (thr <= 0 || nr == 0 || nc == 0 || t.rowptr.empty() || t.rowptr[nr] == 0) return;
     // ... and only for tiles of >= min_rows rows: a dense launch costs a fixed ~15 us (B images,
-    // the persistent kernel's ramp, the fix-up) that the small stage tiles of an 8-way split do
-    // not amortise (SOLO rank 0: Reddit-shaped P = 8 3.69 -> 3.68 ms, Proteins-shaped P = 8
-    // 1.46 -> 1.70 ms with blocks; P = 4 Reddit 6.61 -> 5.62 ms; profiles/r02_dense_solo_ab.jsonl)
+    // the persistent kernel's ramp, the fix-up), and the gathers it replaces are cheap when the
+    // gathered block sits in L2; the 29 K-row local tile of an 8-way Reddit-shaped split loses
+    // (+0.045 ms per wide SpMM) while its 5-block stage group gains (-0.075 ms), Proteins-shaped
+    // P = 8 loses overall (1.46 -> 1.70 ms), P = 4 gains (Reddit 6.61 -> 5.62 ms, Proteins 33 K
+    // rows 2.33 -> 2.15 ms; SOLO rank 0, profiles/r02_dense_solo_ab.jsonl)
     if (nr < min_rows) return;
     const int64_t min_cnt = std::max<int64_t>(1, (int64_t)std::ceil(thr * TM * TK));
     const bool pat = t.val.empty();

@@ -365,7 +365,12 @@ int64_t persistent_blocks(int64_t n_items, int over) {
         if (per_sm <= 0) per_sm = 1;
     }
     const int64_t need = (n_items + kWarpsPerBlock - 1) / kWarpsPerBlock;
-    const int64_t cap = (int64_t)per_sm * sm_count() * over;
+    static int sms_env = -1;   // experiment hook: MGGCN_SPMM_SMS = SMs the persistent grid is sized for
+    if (sms_env < 0) {
+        const char* e = getenv("MGGCN_SPMM_SMS");
+        sms_env = e ? atoi(e) : 0;
+    }
+    const int64_t cap = (int64_t)per_sm * (sms_env > 0 ? sms_env : sm_count()) * over;
     return need < cap ? need : cap;
 }
 

@@ -23,7 +23,7 @@ def rel(x, r):
 @pytest.fixture(autouse=True)
 def _any_coverage(monkeypatch):
     """The tests force blocks at every threshold (the default MGGCN_DENSE_MINFRAC = 0.5 keeps
-    only tiles whose blocks hold half the entries, MGGCN_DENSE_MIN_ROWS = 49152 only tiles of
+    only tiles whose blocks hold half the entries, MGGCN_DENSE_MIN_ROWS = 32768 only tiles of
     that many rows)."""
     monkeypatch.setenv("MGGCN_DENSE_MINFRAC", "0")
     monkeypatch.setenv("MGGCN_DENSE_MIN_ROWS", "0")

@@ -42,10 +42,10 @@ namespace {
 constexpr int kDnEpiWarps = 8;                     // 2 per TMEM lane quadrant, 128 columns each
 constexpr int kDnThreads = (kDnEpiWarps + 2) * 32;
 constexpr int kDnProdWarp = kDnEpiWarps, kDnMmaWarp = kDnEpiWarps + 1;
-constexpr int kDnMaxStages = 8;
+constexpr int kDnMaxStages = 16;                    // narrow N: many small stages cover the latency
 constexpr int kDnABytes = kDenseM * kDenseK * 2;   // 8 KB: 128 rows x 64 B
 constexpr int kDnSmemMax = 232448;                 // sm_100 opt-in shared memory per block
-constexpr int kDnBarBytes = 256;
+constexpr int kDnBarBytes = 512;
 constexpr int kDenseDrain = 8;                      // blocks per accumulation chain (MGGCN_DENSE_DRAIN)
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -203,6 +203,7 @@ struct DnParams {
 };
 
 // ------------------------------------------------------------ tiles
+template <int PIECES>
 __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParams p) {
     extern __shared__ uint8_t smem_dyn[];
     uint8_t* smem = smem_dyn + ((1024u - (smem_u32(smem_dyn) & 1023u)) & 1023u);
@@ -281,13 +282,15 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
                     tc_fence_after();
                     const uint32_t sa = smem_u32(smem + (size_t)s * stage_bytes);
                     const uint64_t ad = sw64_desc(sa);
+                    uint64_t bd[PIECES];
+#pragma unroll
+                    for (int q = 0; q < PIECES; ++q) bd[q] = sw64_desc(sa + kDnABytes + (uint32_t)(q * N * 64));
 #pragma unroll
                     for (int kk = 0; kk < kDenseK / 16; ++kk) {
                         const uint64_t adv = (uint64_t)((kk * 32) >> 4);   // 16 bf16 = 32 B per k step
-                        for (int q = 0; q < p.pieces; ++q) {
-                            const uint64_t bd = sw64_desc(sa + kDnABytes + (uint32_t)(q * N * 64));
-                            mma_bf16(d, ad + adv, bd + adv, idesc, (tc > 0 || kk > 0 || q > 0) ? 1u : 0u);
-                        }
+#pragma unroll
+                        for (int q = 0; q < PIECES; ++q)
+                            mma_bf16(d, ad + adv, bd[q] + adv, idesc, (tc > 0 || kk > 0 || q > 0) ? 1u : 0u);
                     }
                     mma_commit(empty + s);
                     if (++s == S) { s = 0; ph ^= 1; }
@@ -414,7 +417,9 @@ cudaError_t launch_dense(const DenseTiles& d, const float* B, int64_t ldb, float
     const size_t smem = 1024 + (size_t)S * (kDnABytes + pieces * N * 64) + kDnBarBytes;
     static bool attr = false;
     if (!attr) {
-        e = cudaFuncSetAttribute(dense_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kDnSmemMax);
+        e = cudaFuncSetAttribute(dense_tile_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, kDnSmemMax);
+        if (e == cudaSuccess)
+            e = cudaFuncSetAttribute(dense_tile_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, kDnSmemMax);
         if (e != cudaSuccess) return e;
         attr = true;
     }
@@ -442,7 +447,8 @@ cudaError_t launch_dense(const DenseTiles& d, const float* B, int64_t ldb, float
     }
     p.drain = drain_env > 0 ? drain_env : kDenseDrain;
     const int grid = (int)d.n_bins;
-    dense_tile_kernel<<<grid, kDnThreads, smem, s>>>(p);
+    if (pieces == 2) dense_tile_kernel<2><<<grid, kDnThreads, smem, s>>>(p);
+    else dense_tile_kernel<3><<<grid, kDnThreads, smem, s>>>(p);
     count_launches(2);
     e = cudaGetLastError();
     if (e != cudaSuccess || d.n_splits == 0) return e;

@@ -36,17 +36,20 @@ inline bool bf16_exact(float v) {
 }  // namespace
 
 // (global scope, like HostTile and DenseHost in internal.h)
-void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows, DenseHost& d) {
+void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows, int64_t min_entries,
+                DenseHost& d) {
     d = DenseHost();
     const int64_t nr = t.nrows, nc = t.ncols;
     if (thr <= 0 || nr == 0 || nc == 0 || t.rowptr.empty() || t.rowptr[nr] == 0) return;
-    // ... and only for tiles of >= min_rows rows: a dense launch costs a fixed ~15 us (B images,
-    // the persistent kernel's ramp, the fix-up), and the gathers it replaces are cheap when the
-    // gathered block sits in L2; the 29 K-row local tile of an 8-way Reddit-shaped split loses
-    // (+0.045 ms per wide SpMM) while its 5-block stage group gains (-0.075 ms), Proteins-shaped
-    // P = 8 loses overall (1.46 -> 1.70 ms), P = 4 gains (Reddit 6.61 -> 5.62 ms, Proteins 33 K
-    // rows 2.33 -> 2.15 ms; SOLO rank 0, profiles/r02_dense_solo_ab.jsonl)
-    if (nr < min_rows) return;
+    // ... and only for tiles of >= min_entries entries (and min_rows rows): a dense launch
+    // costs a fixed ~15 us (B images, the persistent kernel's ramp, the fix-up), and the gathers
+    // it replaces are cheap when the gathered block sits in L2.  At P = 8 the Reddit-shaped
+    // 1.2 M-entry local tile loses with blocks (+0.045 ms per wide SpMM) while its 6 M-entry
+    // 5-block stage group gains (-0.075 ms); SOLO rank 0 with >= 3 M entries: Reddit-shaped
+    // P = 8 3.70 -> 3.45 ms, P = 4 unchanged (5.58 ms, every tile >= 4.9 M), Proteins-shaped
+    // P = 8 1.46 -> 1.45 ms, while all tiles with blocks lose at P = 8 (Proteins 1.70 ms)
+    // (profiles/r02_dense_solo_ab.jsonl)
+    if (nr < min_rows || (int64_t)t.rowptr[nr] < min_entries) return;
     const int64_t min_cnt = std::max<int64_t>(1, (int64_t)std::ceil(thr * TM * TK));
     const bool pat = t.val.empty();
     auto ok = [&](int64_t e) { return pat || bf16_exact(t.val[e]); };

@@ -62,9 +62,10 @@ struct DenseHost {
     std::vector<int32_t> chunk_cols;    // n_chunks * 32, -1 = empty slot
     std::vector<uint16_t> A;            // n_tiles * 128 * 32 bf16, K-major SWIZZLE_64B image per block
 };
-// thr <= 0, a tile of fewer than min_rows rows, nothing dense, or the blocks holding < min_frac
+// thr <= 0, a tile of fewer than min_rows rows or min_entries entries, nothing dense, or the blocks holding < min_frac
 // of the entries => d.active = false.
-void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows, DenseHost& d);
+void plan_dense(const HostTile& t, double thr, double min_frac, int64_t min_rows, int64_t min_entries,
+                DenseHost& d);
 
 // One rank's 1D partition of the permuted graph.
 struct mggcn_part_s {

@@ -44,7 +44,9 @@ constexpr double kDenseThrDefault = 0.03;
 // a tile uses blocks only if they hold >= this share of its entries; MGGCN_DENSE_MINFRAC overrides
 constexpr double kDenseMinFracDefault = 0.5;
 // ... and only in tiles of at least this many rows (MGGCN_DENSE_MIN_ROWS overrides)
-constexpr int64_t kDenseMinRowsDefault = 32768;
+constexpr int64_t kDenseMinRowsDefault = 0;
+// ... holding at least this many coalesced entries (MGGCN_DENSE_MIN_ENTRIES overrides)
+constexpr int64_t kDenseMinEntriesDefault = 3000000;
 struct DenseTiles {
     int64_t n_groups = 0, n_tiles = 0, n_chunks = 0;
     int64_t n_items = 0, n_splits = 0, n_slots = 0, n_bins = 0;

@@ -310,6 +310,7 @@ struct mggcn_model_s {
     double dense_thr = 0;
     double dense_min_frac = 0.5;    // MGGCN_DENSE_MINFRAC: blocks must hold this share of a tile's entries
     int64_t dense_min_rows = 0;     // MGGCN_DENSE_MIN_ROWS: ... in tiles of at least this many rows
+    int64_t dense_min_entries = 0;  // MGGCN_DENSE_MIN_ENTRIES: ... and this many (coalesced) entries
     int dense_pieces = 3;
     // SOLO timing mode (MGGCN_F_NO_BCAST, P > 1, nlocal = 1, no NCCL id, no IPC): one rank of a
     // P-way run on its own, every collective skipped; per-rank compute time of a partition
@@ -1642,6 +1643,8 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
         m->dense_min_frac = fe ? atof(fe) : kDenseMinFracDefault;
         const char* me = getenv("MGGCN_DENSE_MIN_ROWS");
         m->dense_min_rows = me ? atoll(me) : kDenseMinRowsDefault;
+        const char* ne = getenv("MGGCN_DENSE_MIN_ENTRIES");
+        m->dense_min_entries = ne ? atoll(ne) : kDenseMinEntriesDefault;
         if (!(m->dense_thr > 0) || (!m->ranks.empty() && !m->ranks[0].coalesced)) m->dense_thr = 0;
     }
     if (m->dense_thr > 0) {
@@ -1650,13 +1653,13 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
             if (!r.part->shared_fb) r.dB.assign(m->P, DenseHost());
             for (int j = 0; j < m->P; ++j) {
                 if (m->grouped() && j != r.rank) continue;
-                plan_dense(r.tF(j), m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dF[j]);
+                plan_dense(r.tF(j), m->dense_thr, m->dense_min_frac, m->dense_min_rows, m->dense_min_entries, r.dF[j]);
                 if (r.dF[j].active) {
                     r.hF[j] = HostItems();
                     build_items(r.lF(j), r.hF[j], r.order_cache);
                 }
                 if (!r.part->shared_fb) {
-                    plan_dense(r.tB(j), m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dB[j]);
+                    plan_dense(r.tB(j), m->dense_thr, m->dense_min_frac, m->dense_min_rows, m->dense_min_entries, r.dB[j]);
                     if (r.dB[j].active) {
                         r.hB[j] = HostItems();
                         build_items(r.lB(j), r.hB[j], r.order_cache);
@@ -1667,13 +1670,13 @@ static int model_init_common(mggcn_model_s* m, const mggcn_part* parts, int32_t 
             r.dgF.assign(NG, DenseHost());
             if (!r.part->shared_fb) r.dgB.assign(NG, DenseHost());
             for (int g = 0; g < NG; ++g) {
-                plan_dense(r.gF[g], m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dgF[g]);
+                plan_dense(r.gF[g], m->dense_thr, m->dense_min_frac, m->dense_min_rows, m->dense_min_entries, r.dgF[g]);
                 if (r.dgF[g].active) {
                     r.hgF[g] = HostItems();
                     build_items(r.lgF(g), r.hgF[g], r.order_cache);
                 }
                 if (!r.part->shared_fb) {
-                    plan_dense(r.gB[g], m->dense_thr, m->dense_min_frac, m->dense_min_rows, r.dgB[g]);
+                    plan_dense(r.gB[g], m->dense_thr, m->dense_min_frac, m->dense_min_rows, m->dense_min_entries, r.dgB[g]);
                     if (r.dgB[g].active) {
                         r.hgB[g] = HostItems();
                         build_items(r.lgB(g), r.hgB[g], r.order_cache);

@@ -28,7 +28,7 @@ for dims, P, n, m, c in (((1433, 16, 7), 2, 2708, 10556, 1), ((8, 128, 128, 112)
     print("epoch ok", dims, P, c, loss, flush=True)
     gm.close()
 # dense blocks (dense.cu): forced on the small tiles of a 4096-vertex R-MAT (MGGCN_DENSE_* read at model creation)
-os.environ.update(MGGCN_DENSE_THR="0.02", MGGCN_DENSE_MINFRAC="0", MGGCN_DENSE_MIN_ROWS="0")
+os.environ.update(MGGCN_DENSE_THR="0.02", MGGCN_DENSE_MINFRAC="0", MGGCN_DENSE_MIN_ROWS="0", MGGCN_DENSE_MIN_ENTRIES="0")
 for P in (1, 2):
     n, dims = 4096, (64, 256, 256, 41)
     rp, col = gen.rmat_csr(n, 400000, 17)
@@ -42,7 +42,7 @@ for P in (1, 2):
     gm.backward(); gm.step()
     print("dense epoch ok", P, loss, mg.mggcn_dense_stats(gm.m), flush=True)
     gm.close()
-for k in ("MGGCN_DENSE_THR", "MGGCN_DENSE_MINFRAC", "MGGCN_DENSE_MIN_ROWS"):
+for k in ("MGGCN_DENSE_THR", "MGGCN_DENSE_MINFRAC", "MGGCN_DENSE_MIN_ROWS", "MGGCN_DENSE_MIN_ENTRIES"):
     os.environ.pop(k)
 for op, (M, N, K) in ((0, (300, 41, 602)), (1, (257, 256, 41)), (2, (602, 47, 1000))):
     rng = np.random.default_rng(op)

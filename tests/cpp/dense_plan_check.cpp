@@ -22,7 +22,7 @@ int main(int argc, char** argv) {
     t.rowptr.push_back(0);
     for (int i = 0; i < n; ++i) { std::sort(adj[i].begin(), adj[i].end()); adj[i].erase(std::unique(adj[i].begin(), adj[i].end()), adj[i].end());
         for (int c : adj[i]) { t.col.push_back(c); t.val.push_back(1.f + (rng() % 3)); } t.rowptr.push_back(t.col.size()); }
-    DenseHost d; plan_dense(t, thr, 0.0, 0, d);
+    DenseHost d; plan_dense(t, thr, 0.0, 0, 0, d);
     printf("active %d groups %ld tiles %ld chunks %ld nnz %ld items %ld splits %ld slots %ld resid %d total %zu\n", d.active, d.n_groups, d.n_tiles, d.n_chunks, d.nnz, d.n_items, d.n_splits, d.n_slots, d.active ? d.resid.rowptr.back() : -1, t.col.size());
     // reconstruct dense matrix from A images
     std::vector<double> M((size_t)n * n, 0), R((size_t)n * n, 0);

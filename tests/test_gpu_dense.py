@@ -23,10 +23,11 @@ def rel(x, r):
 @pytest.fixture(autouse=True)
 def _any_coverage(monkeypatch):
     """The tests force blocks at every threshold (the default MGGCN_DENSE_MINFRAC = 0.5 keeps
-    only tiles whose blocks hold half the entries, MGGCN_DENSE_MIN_ROWS = 32768 only tiles of
-    that many rows)."""
+    only tiles whose blocks hold half the entries, MGGCN_DENSE_MIN_ENTRIES = 3 M only tiles of
+    that many entries)."""
     monkeypatch.setenv("MGGCN_DENSE_MINFRAC", "0")
     monkeypatch.setenv("MGGCN_DENSE_MIN_ROWS", "0")
+    monkeypatch.setenv("MGGCN_DENSE_MIN_ENTRIES", "0")
 
 
 @pytest.fixture(scope="module")
@@ -206,6 +207,25 @@ def test_dense_min_rows_rule(mg, monkeypatch):
     n, m = 4096, 400000
     rp, col = gen.rmat_csr(n, m, 17)
     monkeypatch.setenv("MGGCN_DENSE_MIN_ROWS", "3000")
+    gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] > 0
+    gm.close()
+    gm = _model(mg, n, rp, col, None, (64, 64), 2, 9)
+    assert mg.mggcn_dense_stats(gm.m)["blocks"] == 0
+    gm.close()
+
+
+def test_dense_min_entries_rule(mg, monkeypatch):
+    """Tiles with fewer than MGGCN_DENSE_MIN_ENTRIES coalesced entries keep the pure gather
+    path; P = 2 roughly quarters the entries of every tile."""
+    monkeypatch.setenv("MGGCN_DENSE_THR", "0.03")
+    n, m = 4096, 400000
+    rp, col = gen.rmat_csr(n, m, 17)
+    gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
+    st = mg.mggcn_dense_stats(gm.m)
+    gm.close()
+    assert st["blocks"] > 0
+    monkeypatch.setenv("MGGCN_DENSE_MIN_ENTRIES", str(st["entries"] // 2))
     gm = _model(mg, n, rp, col, None, (64, 64), 1, 9)
     assert mg.mggcn_dense_stats(gm.m)["blocks"] > 0
     gm.close()

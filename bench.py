@@ -274,7 +274,7 @@ def stored_traffic(workload, P):
         "same_build": (d.get("so_sha256") == cur) if d.get("so_sha256") else None}
 
 
-def dense_summary(st, dims):
+def dense_summary(st, dims, dense_ms=0.0, bf16_peak=1352.7):
     """The dense-block part of the SpMM (DESIGN §6 "Dense blocks"): blocks, the share of the
     coalesced entries they cover, and the tensor work they issue per epoch (128 x 32 x N x 2 flops
     per block per bf16 piece, N = the SpMM width rounded up to 16 per 256-column window)."""
@@ -285,10 +285,18 @@ def dense_summary(st, dims):
     for wdt in spmm_widths(dims):
         n_pad = sum((min(256, wdt - c0) + 15) // 16 * 16 for c0 in range(0, wdt, 256))
         flops += st["blocks"] * 128 * 32 * n_pad * 2 * pieces
-    return {"blocks": st["blocks"], "block_entries": st["block_entries"], "entries": st["entries"],
-            "entry_frac": st["block_entries"] / max(st["entries"], 1), "row_groups": st["row_groups"],
-            "chunks": st["chunks"], "pieces": pieces, "mma_tflop_per_epoch": flops / 1e12,
-            "thr": os.environ.get("MGGCN_DENSE_THR", "default 0.03")}
+    out = {"blocks": st["blocks"], "block_entries": st["block_entries"], "entries": st["entries"],
+           "entry_frac": st["block_entries"] / max(st["entries"], 1), "row_groups": st["row_groups"],
+           "chunks": st["chunks"], "pieces": pieces, "mma_tflop_per_epoch": flops / 1e12,
+           "thr": os.environ.get("MGGCN_DENSE_THR", "default 0.03")}
+    if dense_ms > 0:
+        ach = flops / (dense_ms * 1e-3) / 1e12
+        out["roofline"] = {"bound": "tensor", "achieved": ach, "peak": bf16_peak, "unit": "TFLOP/s",
+                           "frac": ach / bf16_peak, "ms_per_epoch": dense_ms,
+                           "how": "issued bf16 MMA work (128 x 32 x N x 2 flops x pieces per block) / the dense "
+                                  "kernels' time (library CUDA events around B images + blocks + fix-up, profile "
+                                  "class 'dense'), against MEASURED_PEAKS bf16 sustained (timed inside the epoch)"}
+    return out
 
 
 def spmm_widths(dims):
@@ -388,8 +396,11 @@ def timeline_summary(tl, dims, p, rank):
         if r["spmm"] < 0:
             continue
         d = per.setdefault(r["spmm"], {"width": widths[r["spmm"]] if r["spmm"] < len(widths) else None,
-                                       "compute_launches": 0, "compute_ms": 0.0, "comm_ops": 0, "comm_ms": 0.0})
-        if r["stream"] == 0:
+                                       "compute_launches": 0, "compute_ms": 0.0, "comm_ops": 0, "comm_ms": 0.0,
+                                       "dense_ms": 0.0})
+        if r["cls"] == "dense":          # nested inside its stage's spmm record
+            d["dense_ms"] += r["t1"] - r["t0"]
+        elif r["stream"] == 0:
             d["compute_launches"] += 1
             d["compute_ms"] += r["t1"] - r["t0"]
         else:
@@ -781,7 +792,8 @@ def main():
                              "blocks + their fix-up, the column-window gather kernels + hub fix-up)",
                      "l2_gather": l2_gather},
         "epoch_roofline": epoch_roofline,
-        "dense": dense_summary(dense_stats, w.dims),
+        "dense": dense_summary(dense_stats, w.dims, prof.get("dense", (0.0, 0))[0] / args.steps,
+                               float(peaks.get("bf16_tflops_sustained", 1352.7))),
         "breakdown_ms_per_epoch": {k: v[0] / args.steps for k, v in prof.items()},
         "gemm": {"tflops": gemm_tflops, "peak_tf32_tflops": tf32_peak, "ms_per_epoch": gemm_ms / args.steps,
                  "frac_model_flops": gemm_tflops / tf32_peak if gemm_tflops else None,

@@ -263,8 +263,9 @@ int mggcn_set_adam(mggcn_model m, int32_t layer, const float* mom, const float* 
 /* Profiling (MGGCN_F_PROFILE): accumulated device milliseconds and launch
  * counts per op class since the last reset, measured with CUDA events on the
  * stream each op is launched on.  Classes: 0 spmm, 1 gemm, 2 loss, 3 adam,
- * 4 bcast, 5 allreduce, 6 other.  Synchronises. */
-int mggcn_get_profile(mggcn_model m, double* ms /*[7]*/, int64_t* launches /*[7]*/, int32_t reset);
+ * 4 bcast, 5 allreduce, 6 other, 7 dense (the dense-block kernels of the SpMM
+ * stages; also contained in class 0).  Synchronises. */
+int mggcn_get_profile(mggcn_model m, double* ms /*[8]*/, int64_t* launches /*[8]*/, int32_t reset);
 /* Per-stage timeline (MGGCN_F_TIMELINE; the paper's Fig. 6 / Fig. 8 stage
  * timelines).  Copies up to `cap` records made
  * since the last reset, in issue order: meta[5*i ..] = {op class (as in

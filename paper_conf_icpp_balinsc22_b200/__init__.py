@@ -28,7 +28,7 @@ MGGCN_F_REPL2 = 512        # 1.5D, replication factor c = 2
 MGGCN_F_REPLICA1 = 1024    # with MGGCN_F_REPL2, nlocal = 1: this process is replica 1
 MGGCN_F_TIMELINE = 2048    # per-stage comm / compute event timeline (mggcn_get_timeline)
 MGGCN_IPC_BLOB_BYTES = 128
-PROFILE_CLASSES = ("spmm", "gemm", "loss", "adam", "bcast", "allreduce", "other")
+PROFILE_CLASSES = ("spmm", "gemm", "loss", "adam", "bcast", "allreduce", "other", "dense")
 
 EXPORTS = (
     "mggcn_last_error", "mggcn_version", "mggcn_load_csr", "mggcn_graph_info", "mggcn_partition",
@@ -307,8 +307,8 @@ def mggcn_set_adam(m, layer, mom, vel, t):
 
 
 def mggcn_get_profile(m, reset=False):
-    ms = (ctypes.c_double * 7)()
-    n = (ctypes.c_int64 * 7)()
+    ms = (ctypes.c_double * len(PROFILE_CLASSES))()
+    n = (ctypes.c_int64 * len(PROFILE_CLASSES))()
     _check(_lib.mggcn_get_profile(m, ms, n, 1 if reset else 0))
     return {c: (ms[i], n[i]) for i, c in enumerate(PROFILE_CLASSES)}
 

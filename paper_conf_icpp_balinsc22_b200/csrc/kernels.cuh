@@ -115,6 +115,12 @@ constexpr int kYieldBlocks = 4;
 // rowscale (nullable): multiplies the finished row on the LAST stage.
 cudaError_t launch_spmm(const SpmmTile& t, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
                         const float* rowscale, int width, int flags, cudaStream_t s);
+// the two halves of launch_spmm, in this order: the tile's dense blocks (no-op without them),
+// then the gather of the residual CSR with the stage epilogue
+cudaError_t launch_spmm_dense(const SpmmTile& t, const float* B, int64_t ldb, float* out, int64_t ldo, int width,
+                              int flags, cudaStream_t s);
+cudaError_t launch_spmm_gather(const SpmmTile& t, const float* B, int64_t ldb, float* out, int64_t ldo,
+                               float* partial, const float* rowscale, int width, int flags, cudaStream_t s);
 
 // ------------------------------------------------------------------ GEMM
 // tcgen05 (kind::tf32) GEMM with TMA-staged operands and TMEM accumulators.

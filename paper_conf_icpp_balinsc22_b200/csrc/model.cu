@@ -29,7 +29,8 @@ namespace {
 
 enum Order { G_ORDER = 0, S_ORDER = 1 };   // GeMM-first / SpMM-first (§4.4)
 enum State { ST_READY = 0, ST_FWD = 1, ST_BWD = 2 };
-enum ProfClass { PC_SPMM = 0, PC_GEMM, PC_LOSS, PC_ADAM, PC_BCAST, PC_ALLRED, PC_OTHER, PC_N };
+// PC_DENSE: the dense-block kernels of an SpMM stage, recorded inside (and counted in) its PC_SPMM scope
+enum ProfClass { PC_SPMM = 0, PC_GEMM, PC_LOSS, PC_ADAM, PC_BCAST, PC_ALLRED, PC_OTHER, PC_DENSE, PC_N };
 
 struct Bump {
     char* base = nullptr;
@@ -464,7 +465,7 @@ cudaEvent_t prof_event(mggcn_model_s* m) {
 
 // NVTX range names per op class (ranges for nsys / ncu --nvtx; no-ops without a tool)
 const char* const kNvtxName[PC_N] = {"mggcn:spmm", "mggcn:gemm", "mggcn:loss", "mggcn:adam", "mggcn:bcast",
-                                     "mggcn:allreduce", "mggcn:other"};
+                                     "mggcn:allreduce", "mggcn:other", "mggcn:dense"};
 
 struct NvtxRange {
     explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
@@ -974,6 +975,18 @@ int wait_bc(mggcn_model_s* m, cudaEvent_t e) {
     return MGGCN_OK;
 }
 
+// One SpMM stage launch: the dense blocks under their own PC_DENSE scope (nested in the
+// caller's PC_SPMM scope), then the gather of the residual entries.
+cudaError_t spmm_call(mggcn_model_s* m, const SpmmTile& t, const float* B, int width, float* out, float* partial,
+                      const float* rowscale, int flags) {
+    if (t.dense.n_items > 0) {
+        ProfScope pd(m, PC_DENSE, m->cs);
+        cudaError_t e = launch_spmm_dense(t, B, width, out, width, width, flags, m->cs);
+        if (e != cudaSuccess) return e;
+    }
+    return launch_spmm_gather(t, B, width, out, width, partial, rowscale, width, flags, m->cs);
+}
+
 int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const float* B, int flags, int tl_k) {
     RC(inject_delay(m, m->cs));
     const SpmmTile& t = job.dir == 0 ? r.F[j] : r.B[j];
@@ -983,8 +996,8 @@ int launch_stage(mggcn_model_s* m, Rank& r, const SpmmJob& job, int j, const flo
     ProfScope ps(m, PC_SPMM, m->cs);
     // NCCL collectives run as kernels on the comm stream: let them in while the SpMM runs
     if ((m->comm || m->solo) && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
-    CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
-                   (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
+    CK(spmm_call(m, t, B, (int)job.width, out, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
+                 flags | (job.relu ? SPMM_RELU : 0)));
     return MGGCN_OK;
 }
 
@@ -1023,8 +1036,8 @@ int launch_group(mggcn_model_s* m, Rank& r, const SpmmJob& job, int g, int flags
     ProfScope ps(m, PC_SPMM, m->cs);
     if ((m->comm || m->solo) && m->P > 1 && (m->flags & MGGCN_F_OVERLAP)) flags |= SPMM_YIELD;
     const float* B = group_slot(m, r, m->grp_b[g], job.width);
-    CK(launch_spmm(t, B, job.width, out, job.width, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
-                   (int)job.width, flags | (job.relu ? SPMM_RELU : 0), m->cs));
+    CK(spmm_call(m, t, B, (int)job.width, out, r.spmm_partial, job.use_rowscale ? r.inv_deg : nullptr,
+                 flags | (job.relu ? SPMM_RELU : 0)));
     return MGGCN_OK;
 }
 

@@ -440,19 +440,30 @@ cudaError_t dispatch_gc(int w4, const SpmmTile& t, const float4* B, int64_t ldb4
 
 }  // namespace
 
+cudaError_t launch_spmm_dense(const SpmmTile& tile, const float* B, int64_t ldb, float* out, int64_t ldo, int width,
+                              int flags, cudaStream_t s) {
+    if (tile.nrows == 0 || tile.dense.n_items == 0) return cudaSuccess;
+    for (int c0 = 0; c0 < width; c0 += kDenseMaxN) {
+        const int w = width - c0 < kDenseMaxN ? width - c0 : kDenseMaxN;
+        cudaError_t e = launch_dense(tile.dense, B + c0, ldb, out + c0, ldo, w, !(flags & SPMM_ACCUM), s);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
 cudaError_t launch_spmm(const SpmmTile& tile, const float* B, int64_t ldb, float* out, int64_t ldo, float* partial,
                         const float* rowscale, int width, int flags, cudaStream_t s) {
-    if (tile.nrows == 0) return cudaSuccess;
     // Dense blocks (dense.cu) first: they store (first stage) or add their products into the
     // rows of their groups; the gather kernel then adds the residual entries to those rows
     // (DenseTiles::row_flag), writes the others as usual and applies the stage epilogue.
-    if (tile.dense.n_items > 0) {
-        for (int c0 = 0; c0 < width; c0 += kDenseMaxN) {
-            const int w = width - c0 < kDenseMaxN ? width - c0 : kDenseMaxN;
-            cudaError_t e = launch_dense(tile.dense, B + c0, ldb, out + c0, ldo, w, !(flags & SPMM_ACCUM), s);
-            if (e != cudaSuccess) return e;
-        }
-    }
+    cudaError_t e = launch_spmm_dense(tile, B, ldb, out, ldo, width, flags, s);
+    if (e != cudaSuccess) return e;
+    return launch_spmm_gather(tile, B, ldb, out, ldo, partial, rowscale, width, flags, s);
+}
+
+cudaError_t launch_spmm_gather(const SpmmTile& tile, const float* B, int64_t ldb, float* out, int64_t ldo,
+                               float* partial, const float* rowscale, int width, int flags, cudaStream_t s) {
+    if (tile.nrows == 0) return cudaSuccess;
     // a middle stage (accumulating, not the last) skips the tile's empty rows: their sum is
     // zero, so their output read-modify-write is a no-op (the first stage writes every row,
     // the last applies the row scale / ReLU to every row)

@@ -227,6 +227,9 @@ int mggcn_backward(mggcn_model m);
  * mggcn_forward(m, NULL, 0, NULL, ...) consumes it.  The caller keeps the
  * host buffers valid until that forward returns.  ESTATE if one is pending. */
 int mggcn_prefetch(mggcn_model m, const float* X_local, int64_t ldx, const int32_t* y_local);
+/*   EUNSUPPORTED with MGGCN_F_IPC when layer 0 is SpMM-first (X itself is exchanged: the peers
+ *   pull it from this rank's current input buffer, so every rank must use the same one; X is
+ *   then also always copied into the workspace, never used in place). */
 /* Drops the MGGCN_F_CACHE_L0 aggregate; the next forward recomputes it from X. */
 int mggcn_reset_cache(mggcn_model m);
 int mggcn_step(mggcn_model m, float lr, float beta1, float beta2, float eps);

@@ -858,7 +858,13 @@ int use_input_buffer(mggcn_model_s* m, int k) {
 }
 
 // A device X with the padded row stride and 16-B alignment is used in place.
+// IPC with a SpMM-first layer 0: the peers pull X from this rank's symmetric workspace at the
+// offset of ITS current input buffer (peer_ptr), so X must live in Xbuf[xcur] (no zero-copy
+// external pointer) and every rank must use the same buffer (no prefetch double-buffering).
+bool ipc_x_exchanged(const mggcn_model_s* m) { return m->ipc && m->order[0] == S_ORDER && m->P > 1; }
+
 bool device_zero_copy(mggcn_model_s* m, const float* X, int64_t ldx) {
+    if (ipc_x_exchanged(m)) return false;
     if (ldx != m->ld[0] || (reinterpret_cast<uintptr_t>(X) & 15)) return false;
     cudaPointerAttributes pa;
     const bool dev = cudaPointerGetAttributes(&pa, X) == cudaSuccess && pa.type == cudaMemoryTypeDevice;
@@ -2278,6 +2284,11 @@ extern "C" int mggcn_prefetch(mggcn_model m, const float* X_local, int64_t ldx, 
     if (m->pref_buf >= 0) {
         set_error("prefetch: a prefetch is already pending (call mggcn_forward(X = NULL) first)");
         return MGGCN_ESTATE;
+    }
+    if (ipc_x_exchanged(m)) {
+        set_error("prefetch: not with MGGCN_F_IPC and a SpMM-first layer 0 (peers read X from the "
+                  "current input buffer, which must be the same on every rank)");
+        return MGGCN_EUNSUPPORTED;
     }
     const int k = 1 - m->xcur;
     auto body = [&]() -> int {

@@ -25,6 +25,9 @@ def main():
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
     torch.cuda.set_device(rank % torch.cuda.device_count())
     n, m, dims, seed = 3001, 60000, (100, 64, 64, 7), 75
+    if mode.endswith("_sorder"):     # SpMM-first layer 0: X itself is pulled by the peers
+        dims = (8, 32, 32, 7)
+        mode = mode[:-len("_sorder")]
     rp, col = gen.rmat_csr(n, m, 71)
     X = gen.features(n, dims[0], 72)
     y = gen.labels(n, dims[-1], 73, 200)
@@ -39,6 +42,18 @@ def main():
         Xin, yin = torch.from_numpy(Xl).cuda(), torch.from_numpy(yl).cuda()
     else:
         Xin, yin = Xl, yl
+    if mode == "prefetch" and dims[0] < dims[1]:
+        # MGGCN_F_IPC + SpMM-first layer 0: prefetch double-buffering is refused (include/mggcn.h)
+        try:
+            gm.prefetch(Xin, yin)
+            res["prefetch_refused"] = np.int64(0)
+        except mg.MggcnError as e:
+            res["prefetch_refused"] = np.int64(e.code == mg.MGGCN_EUNSUPPORTED)
+        gm.close()
+        np.savez(out, **res)
+        dist.barrier()
+        dist.destroy_process_group()
+        return
     if mode == "prefetch":
         gm.prefetch(Xin, yin)
     for s in range(steps):

@@ -83,6 +83,28 @@ def test_ipc_two_ranks_vs_oracle(tmp_path, reference, mode):
         assert rel(res[0][f"WG0_{l}"], r1.WG[l]) < REL_TOL, l
 
 
+def test_ipc_spmm_first_layer0(tmp_path):
+    """MGGCN_F_IPC with a SpMM-first layer 0 (X itself is pulled from the peers' input buffers):
+    a device X is copied into the workspace instead of used in place (its address would not be
+    in the peers' mapping), the epoch matches the P = 2 oracle, and mggcn_prefetch (which would
+    let the ranks' input buffers differ) is refused with EUNSUPPORTED."""
+    n, m, dims = 3001, 60000, (8, 32, 32, 7)
+    rp, col = gen.rmat_csr(n, m, 71)
+    X = gen.features(n, dims[0], 72)
+    y = gen.labels(n, dims[-1], 73, 200)
+    Ws = [gen.glorot(dims[l], dims[l + 1], 74 + l) for l in range(len(dims) - 1)]
+    pg = oracle.permute_graph(n, rp, col, None, seed=75)
+    ref = oracle.epoch(pg, X, y, Ws, P=2)
+    res = run_ranks(tmp_path, "device_sorder", steps=1)
+    logits = np.concatenate([r["logits"] for r in res])
+    assert rel(logits, ref.logits) < REL_TOL
+    assert abs(float(res[0]["loss0"]) - ref.loss) / abs(ref.loss) < REL_TOL
+    for l in range(len(Ws)):
+        assert rel(res[0][f"WG0_{l}"], ref.WG[l]) < REL_TOL, l
+    res = run_ranks(tmp_path, "prefetch_sorder", steps=1)
+    assert all(int(r["prefetch_refused"]) == 1 for r in res)
+
+
 def test_bench_two_ranks_ipc_exposed_comm():
     """bench.py's multi-process path end to end (torchrun, 2 ranks, IPC backend; both ranks on
     this GPU, so the times are time-sliced, not scaling numbers): one JSON line from rank 0 with

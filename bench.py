@@ -288,7 +288,7 @@ def dense_summary(st, dims, dense_ms=0.0, bf16_peak=1352.7):
     out = {"blocks": st["blocks"], "block_entries": st["block_entries"], "entries": st["entries"],
            "entry_frac": st["block_entries"] / max(st["entries"], 1), "row_groups": st["row_groups"],
            "chunks": st["chunks"], "pieces": pieces, "mma_tflop_per_epoch": flops / 1e12,
-           "thr": os.environ.get("MGGCN_DENSE_THR", "default 0.03")}
+           "thr": os.environ.get("MGGCN_DENSE_THR", "default 0.04")}
     if dense_ms > 0:
         ach = flops / (dense_ms * 1e-3) / 1e12
         out["roofline"] = {"bound": "tensor", "achieved": ach, "peak": bf16_peak, "unit": "TFLOP/s",

@@ -315,7 +315,7 @@ int mggcn_stage_groups(mggcn_model m, int32_t* sizes, int32_t cap);
  * chunks, [4] coalesced entries of every launched tile (blocks + residual CSR),
  * summed over this model's ranks and both directions (F and B tiles; one set
  * when they are shared).  The density threshold is MGGCN_DENSE_THR at
- * mggcn_model_create (default 0.03; 0 = no blocks).  EINVAL: NULL out. */
+ * mggcn_model_create (default 0.04; 0 = no blocks).  EINVAL: NULL out. */
 int mggcn_dense_stats(mggcn_model m, int64_t* out, int32_t n);
 
 /* Number of kernels this library has launched in this process (all models,

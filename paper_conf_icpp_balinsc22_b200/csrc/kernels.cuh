@@ -40,7 +40,7 @@ constexpr int kDenseM = 128;
 constexpr int kDenseK = 32;
 constexpr int kDenseMaxN = 256;    // features per launch (wider operands: 256-column windows)
 // default density threshold of a dense block (entries / (128 x 32)); MGGCN_DENSE_THR overrides, 0 = off
-constexpr double kDenseThrDefault = 0.03;
+constexpr double kDenseThrDefault = 0.04;
 // a tile uses blocks only if they hold >= this share of its entries; MGGCN_DENSE_MINFRAC overrides
 constexpr double kDenseMinFracDefault = 0.5;
 // ... and only in tiles of at least this many rows (MGGCN_DENSE_MIN_ROWS overrides)

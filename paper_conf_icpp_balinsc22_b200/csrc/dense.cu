@@ -15,13 +15,17 @@
 //                       source rows of H_j, split into bf16 pieces
 //                       (hi + mid + lo = the fp32 value to ~2^-24), transposed
 //                       into the K-major SWIZZLE_64B layout the MMA reads;
-//   dense_tile_kernel   per row group (128 output rows): for every dense block
-//                       of the group, one bulk copy of its A image (the block's
-//                       entries as bf16, pre-swizzled on the host; values are
-//                       small integer multiplicities, exact in bf16) and one of
-//                       the chunk's B image, then tcgen05.mma.kind::f16 (BF16
-//                       in, FP32 accumulate in TMEM) per piece; the epilogue
-//                       adds the 128 x N result into the output rows.
+//   dense_tile_kernel   per work item (a row group of 128 output rows, or a
+//                       segment of a long one; items binned per CTA on the host):
+//                       for every dense block, one bulk copy of its A image (the
+//                       block's entries as bf16, pre-swizzled on the host; values
+//                       are small integer multiplicities, exact in bf16) and one
+//                       of the chunk's B image, then tcgen05.mma.kind::f16 (BF16
+//                       in, FP32 accumulate in TMEM) per piece; every 8 blocks the
+//                       accumulator chain is drained into fp32 registers (reading
+//                       C32), and the epilogue stores / adds the 128 x N result
+//                       into the output rows (or a segment's partial);
+//   dense_fixup_kernel  segments of one row group, summed in order into the rows.
 //
 // The residual non-zeros (everything not in a dense block) stay in the CSR
 // gather kernel (spmm.cu), which runs after this one with SPMM_ACCUM and

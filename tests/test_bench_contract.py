@@ -81,3 +81,33 @@ def test_timeline_summary_exposed_comm_and_bandwidth():
     assert s["bcast_records"] == 1                           # received blocks only
     assert abs(s["bcast_GBps_median"] - 1000 * 4 * 4 / 1e-3 / 1e9) < 1e-9
     assert s["per_spmm"]["0"]["compute_launches"] == 2 and s["per_spmm"]["0"]["width"] == 4
+
+
+def test_dense_summary_flops_and_roofline():
+    """bench.dense_summary: issued MMA work = blocks x 128 x 32 x N x 2 x 3 pieces per SpMM of the
+    epoch (N = width rounded up to 16 per 256-column window), and the tensor roofline divides it
+    by the dense kernels' live time."""
+    import bench
+    st = {"blocks": 1000, "block_entries": 600000, "entries": 1000000, "row_groups": 10, "chunks": 50}
+    d = bench.dense_summary(st, [602, 256, 256, 41], dense_ms=1.0, bf16_peak=1000.0)
+    per_block = 128 * 32 * 2 * 3
+    want = 1000 * per_block * (4 * 256 + 2 * 48)        # widths 256 x 4, 41 -> 48 x 2
+    assert d["mma_tflop_per_epoch"] == pytest.approx(want / 1e12)
+    assert d["entry_frac"] == pytest.approx(0.6)
+    assert d["roofline"]["achieved"] == pytest.approx(want / 1e-3 / 1e12)
+    assert d["roofline"]["frac"] == pytest.approx(d["roofline"]["achieved"] / 1000.0)
+    # widths above 256 run in 256-column windows: 600 -> 256 + 256 + 96
+    d2 = bench.dense_summary(st, [600, 600], dense_ms=0.0)
+    assert d2["mma_tflop_per_epoch"] == pytest.approx(1000 * per_block * 2 * (256 + 256 + 96) / 1e12)
+    assert "roofline" not in d2
+    assert bench.dense_summary({"blocks": 0}, [8, 8])["blocks"] == 0
+
+
+def test_l2_gather_counts_only_gathered_entries():
+    """roofline.l2_gather: the entries of the dense blocks are not gathered, so the L2-line model
+    scales with the gathered (residual) share."""
+    import bench
+    work = {"spmm_gather_bytes": 4.0 * 1e6 * sum(bench.spmm_widths([602, 256, 256, 41]))}
+    full = bench.l2_gather_roofline([602, 256, 256, 41], work, 1.0)
+    part = bench.l2_gather_roofline([602, 256, 256, 41], work, 1.0, gathered_frac=0.25)
+    assert part["line_bytes_per_epoch"] == pytest.approx(0.25 * full["line_bytes_per_epoch"])

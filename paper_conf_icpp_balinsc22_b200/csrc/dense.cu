@@ -204,6 +204,7 @@ struct DnParams {
     int n_items;
     int N, width, pieces, stages;
     int drain;      // blocks per TMEM accumulation chain
+    int stack;      // bf16 pieces stacked along N in one MMA (B = [hi; mid; lo] rows, N_mma = stack x N <= 256)
 };
 
 // ------------------------------------------------------------ tiles
@@ -221,7 +222,12 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
     uint64_t* acce = bars + 2 * kDnMaxStages + 2;   // [2] epilogue (128 threads) -> MMA
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * kDnMaxStages + 4);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t tcols = N <= 128 ? 256u : 512u;   // two accumulators of N columns
+    // Narrow N: the MMA issue, not the tensor work, bounds a block (6 tcgen05.mma of N = 48 take
+    // ~550 of ~690 cycles), so `stack` consecutive pieces, stored contiguously in the B image, go
+    // into ONE MMA of N_mma = stack x N whose accumulator holds each piece in its own N-column
+    // range; the drain sums the ranges in fp32.  An accumulator is accw = stack x N columns.
+    const int accw = p.stack * N;
+    const uint32_t tcols = accw <= 128 ? 256u : 512u;   // two accumulators of accw columns
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < S; ++s) {
@@ -267,8 +273,17 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
         if (lane == 0) {
             // kind::f16: F32 accumulator (bit 4), A and B BF16 (bits 7-9, 10-12 = 1), both K-major,
             // N >> 3 at bit 17, M >> 4 at bit 24
-            const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) |
-                                   ((uint32_t)(kDenseM >> 4) << 24);
+            auto idesc_n = [](int n) {
+                return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(n >> 3) << 17) |
+                       ((uint32_t)(kDenseM >> 4) << 24);
+            };
+            // MMA q of a k step covers pieces [q0, q0 + nq) with N_mma = nq x N (nq = stack, the last
+            // one the remainder); its D range starts at column 0 (the first piece's range) -- the
+            // stacked pieces land in ranges 0, N, 2N, and a remainder MMA adds into range 0
+            const int stack = p.stack;
+            const int nmma = (PIECES + stack - 1) / stack;
+            const uint32_t idesc0 = idesc_n(stack * N);
+            const uint32_t idesc1 = idesc_n((PIECES - stack) * N > 0 ? (PIECES - stack < stack ? PIECES - stack : stack) * N : N);
             int s = 0, a = 0;
             uint32_t ph = 0, aph = 0;
             for (int w = __ldg(p.bin_beg + blockIdx.x); w < w_end; ++w) {
@@ -280,21 +295,24 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
                     if (tc == 0) {   // a new chain: wait until the epilogue drained this accumulator
                         mbar_wait(acce + a, aph ^ 1);
                         tc_fence_after();
-                        d = tmem_base + (uint32_t)(a * N);
+                        d = tmem_base + (uint32_t)(a * accw);
                     }
                     mbar_wait(full + s, ph);
                     tc_fence_after();
                     const uint32_t sa = smem_u32(smem + (size_t)s * stage_bytes);
                     const uint64_t ad = sw64_desc(sa);
-                    uint64_t bd[PIECES];
-#pragma unroll
-                    for (int q = 0; q < PIECES; ++q) bd[q] = sw64_desc(sa + kDnABytes + (uint32_t)(q * N * 64));
+                    const uint64_t bd0 = sw64_desc(sa + kDnABytes);
+                    const uint64_t bd1 = sw64_desc(sa + kDnABytes + (uint32_t)(stack * N * 64));
 #pragma unroll
                     for (int kk = 0; kk < kDenseK / 16; ++kk) {
                         const uint64_t adv = (uint64_t)((kk * 32) >> 4);   // 16 bf16 = 32 B per k step
-#pragma unroll
-                        for (int q = 0; q < PIECES; ++q)
-                            mma_bf16(d, ad + adv, bd[q] + adv, idesc, (tc > 0 || kk > 0 || q > 0) ? 1u : 0u);
+                        mma_bf16(d, ad + adv, bd0 + adv, idesc0, (tc > 0 || kk > 0) ? 1u : 0u);
+                        if (nmma > 1) {
+                            mma_bf16(d, ad + adv, bd1 + adv, idesc1, 1u);
+                            for (int q = 2; q < nmma; ++q)   // stack 1: the third piece
+                                mma_bf16(d, ad + adv, sw64_desc(sa + kDnABytes + (uint32_t)(q * N * 64)) + adv, idesc1,
+                                         1u);
+                        }
                     }
                     mma_commit(empty + s);
                     if (++s == S) { s = 0; ph ^= 1; }
@@ -331,11 +349,15 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
 #pragma unroll
                 for (int cc = 0; cc < 4; ++cc) {
                     if (cb + cc * 32 < N) {
-                        uint32_t v[32];
-                        tmem_ld32_nowait(tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * N + cb + cc * 32), v);
-                        tmem_wait_ld();
+                        const uint32_t ta = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * accw + cb + cc * 32);
+                        // the stacked pieces' ranges (hi, mid, lo), one at a time into the running sum
+                        for (int j = 0; j < p.stack; ++j) {
+                            uint32_t v[32];
+                            tmem_ld32_nowait(ta + (uint32_t)(j * N), v);
+                            tmem_wait_ld();
 #pragma unroll
-                        for (int i = 0; i < 32; ++i) run[cc * 32 + i] += __uint_as_float(v[i]);
+                            for (int i = 0; i < 32; ++i) run[cc * 32 + i] += __uint_as_float(v[i]);
+                        }
                     }
                 }
                 tc_fence_before();
@@ -450,6 +472,15 @@ cudaError_t launch_dense(const DenseTiles& d, const float* B, int64_t ldb, float
         if (drain_env < 0) drain_env = 0;
     }
     p.drain = drain_env > 0 ? drain_env : kDenseDrain;
+    static int stack_env = -1;   // MGGCN_DENSE_STACK=1: one MMA per piece (experiment hook)
+    if (stack_env < 0) {
+        const char* se = getenv("MGGCN_DENSE_STACK");
+        stack_env = se ? atoi(se) : 0;
+    }
+    int stack = kDenseMaxN / N < pieces ? kDenseMaxN / N : pieces;
+    if (stack < 1) stack = 1;
+    if (stack_env > 0 && stack_env < stack) stack = stack_env;
+    p.stack = stack;
     const int grid = (int)d.n_bins;
     if (pieces == 2) dense_tile_kernel<2><<<grid, kDnThreads, smem, s>>>(p);
     else dense_tile_kernel<3><<<grid, kDnThreads, smem, s>>>(p);

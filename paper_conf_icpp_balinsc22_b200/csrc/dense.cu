@@ -45,6 +45,9 @@ namespace {
 
 constexpr int kDnEpiWarps = 8;                     // 2 per TMEM lane quadrant, 128 columns each
 constexpr int kDnThreads = (kDnEpiWarps + 2) * 32;
+#ifndef MGGCN_DENSE_BPOL
+#define MGGCN_DENSE_BPOL 0    // L2 policy of the B-image loads: 0 evict_first (default: the next gather kernel keeps the L2), 1 evict_normal, 2 evict_last
+#endif
 constexpr int kDnProdWarp = kDnEpiWarps, kDnMmaWarp = kDnEpiWarps + 1;
 constexpr int kDnMaxStages = 16;                    // narrow N: many small stages cover the latency
 constexpr int kDnABytes = kDenseM * kDenseK * 2;   // 8 KB: 128 rows x 64 B
@@ -85,6 +88,11 @@ __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t b
 __device__ __forceinline__ uint64_t policy_first() {
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint64_t policy_normal() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
     return pol;
 }
 __device__ __forceinline__ uint64_t policy_last() {
@@ -253,7 +261,13 @@ __global__ void __launch_bounds__(kDnThreads, 1) dense_tile_kernel(const DnParam
 
     if (warp == kDnProdWarp) {
         if (lane == 0) {
+#if MGGCN_DENSE_BPOL == 2
             const uint64_t pa = policy_first(), pb = policy_last();
+#elif MGGCN_DENSE_BPOL == 1
+            const uint64_t pa = policy_first(), pb = policy_normal();
+#else
+            const uint64_t pa = policy_first(), pb = policy_first();
+#endif
             int s = 0;
             uint32_t ph = 0;
             for (int w = __ldg(p.bin_beg + blockIdx.x); w < w_end; ++w) {

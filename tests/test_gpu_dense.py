@@ -232,3 +232,23 @@ def test_dense_min_entries_rule(mg, monkeypatch):
     gm = _model(mg, n, rp, col, None, (64, 64), 2, 9)
     assert mg.mggcn_dense_stats(gm.m)["blocks"] == 0
     gm.close()
+
+
+def test_whole_pipeline_with_forced_blocks():
+    """The epoch, captured-graph and 1.5D suites again in a fresh process with dense blocks forced
+    onto every tile (their small graphs normally stay below the size rules): oracle parity,
+    bitwise determinism under delay injection, stage groups, poisoned BC slots and graph replays
+    all hold with the tensor-core part of the SpMM in the loop."""
+    import os
+    import subprocess
+    import sys
+    if os.environ.get("MGGCN_DENSE_MIN_ENTRIES") == "0" and os.environ.get("MGGCN_DENSE_FORCED_RUN"):
+        pytest.skip("already inside the forced run")
+    here = os.path.dirname(os.path.abspath(__file__))
+    env = dict(os.environ, MGGCN_DENSE_THR="0.02", MGGCN_DENSE_MINFRAC="0", MGGCN_DENSE_MIN_ENTRIES="0",
+               MGGCN_DENSE_MIN_ROWS="0", MGGCN_DENSE_FORCED_RUN="1")
+    tests = [os.path.join(here, f) for f in ("test_gpu_epoch.py", "test_gpu_graph.py", "test_gpu_15d.py")]
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu"] + tests, env=env,
+                       cwd=os.path.dirname(here), capture_output=True, text=True, timeout=1500)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout
